@@ -1,0 +1,496 @@
+/*
+ * oracle/oracle.c -- plain, slow, obviously-correct CPU reference of the hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  The product path
+ * (paper_conf_ispass_mehrabilcslo21_b200/, include/spmm.h) never links or calls it,
+ * and the two share no code, header, table or helper.
+ *
+ * Source of every definition: /root/reference/PAPER.md, cited as P:L<n> with its
+ * section; readings of silent/ambiguous passages are SURVEY.md §8(c) c5 A1-A23 and
+ * are listed in DESIGN.md §"Readings".  Floating point is float64 (the paper's
+ * kernel is FP32; the oracle is the exact reference the tolerance of
+ * BASELINE.json north_star is measured against).
+ *
+ * Pins (tests/test_oracle_*.py, -m "not gpu"): numpy dense matmul and scipy.sparse
+ * for SpMM; hand-worked examples E1/E2 (tests/golden/); paper arithmetic P:L88,
+ * P:L92; stencil closed forms; brute-force local-optimality
+ * checkers for every greedy step; permutation invariants.
+ * Parity unpinned: none of the functions below (oracle_mlp_forward is pinned
+ * against a torch forward; the predictor's TRAINING is not an oracle function).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <math.h>
+
+/* policy ids: same numbering as the C-ABI enum (an integer protocol, not shared code) */
+enum {
+    P_IDENTITY = 0, P_NNZ_SORT = 1, P_PLAIN_SORT = 2, P_CTA_AWARE = 3, P_HYBRID_1 = 4, P_HYBRID_2_1 = 5,
+    P_FLIPPED = 6, P_LPT = 7, P_WARP_AWARE = 8, P_HYBRID_2_2 = 9, P_HYBRID_2_3 = 10, P_DCSR = 11
+};
+
+/* ------------------------------------------------------------------------------------
+ * CSR validity (§II.A): rowidx[0]=0, rowidx[M]=nnz, non-decreasing; 0<=col<N;
+ * columns strictly increasing within a row (reading A15).  Returns 0 if valid.
+ * ---------------------------------------------------------------------------------- */
+int oracle_validate_csr(int64_t M, int64_t N, int64_t nnz, const int64_t *rowidx, const int32_t *colidx) {
+    if (M < 0 || N < 0 || nnz < 0) return 1;
+    if (rowidx[0] != 0 || rowidx[M] != nnz) return 2;
+    for (int64_t i = 0; i < M; ++i) {
+        if (rowidx[i + 1] < rowidx[i]) return 3;
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j) {
+            if (colidx[j] < 0 || colidx[j] >= N) return 4;
+            if (j > rowidx[i] && colidx[j] <= colidx[j - 1]) return 5;
+        }
+    }
+    return 0;
+}
+
+/* ------------------------------------------------------------------------------------
+ * c1. SpMM (Alg.1 "Input: CSR A[M][N], float B[N][K]; Output: float C[M][K]").
+ * For each requested original row i and each k:
+ *   C[i][k]     = sum_{j=rowidx[i]}^{rowidx[i+1]-1} value[j]*B[colidx[j]][k]   (float64, ascending j)
+ *   bound[i][k] = sum |value[j]|*|B[colidx[j]][k]|
+ * rows == NULL -> all M rows, output row r at C[r*K]; else output row t at C[t*K].
+ * ---------------------------------------------------------------------------------- */
+void oracle_spmm_rows(int64_t M, const int64_t *rowidx, const int32_t *colidx, const float *value,
+                      const float *B, int64_t K, const int64_t *rows, int64_t nrows, double *C, double *bound) {
+    int64_t n = rows ? nrows : M;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t t = 0; t < n; ++t) {
+        int64_t i = rows ? rows[t] : t;
+        for (int64_t k = 0; k < K; ++k) {
+            double acc = 0.0, bnd = 0.0;
+            for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j) {
+                double a = (double)value[j], b = (double)B[(int64_t)colidx[j] * K + k];
+                acc += a * b;
+                bnd += fabs(a) * fabs(b);
+            }
+            C[t * K + k] = acc;
+            if (bound) bound[t * K + k] = bnd;
+        }
+    }
+}
+
+/* ------------------------------------------------------------------------------------
+ * Row quantities.
+ *   nnz_i = rowidx[i+1]-rowidx[i]
+ *   wl_i  = ceil(nnz_i / nt)  "warp load"                (§II.C)
+ *   blocks_i = sorted unique { colidx[j] div bw }        (§III.B: bit b of the row mask
+ *              is set iff block b of bw=32 consecutive columns holds a non-zero)
+ *   ham(a,b) = |blocks_a| + |blocks_b| - 2|blocks_a ∩ blocks_b|  = popcount(mask_a XOR mask_b)
+ * ---------------------------------------------------------------------------------- */
+static int64_t row_nnz(const int64_t *rowidx, int64_t i) { return rowidx[i + 1] - rowidx[i]; }
+static int64_t warp_load(int64_t nnz, int64_t nt) { return (nnz + nt - 1) / nt; }
+
+typedef struct {
+    int64_t *ptr;   /* [M+1] */
+    int32_t *blk;   /* [ptr[M]] */
+} blocklists;
+
+static blocklists make_blocks(int64_t M, const int64_t *rowidx, const int32_t *colidx, int32_t bw) {
+    blocklists b;
+    b.ptr = (int64_t *)calloc((size_t)M + 1, sizeof(int64_t));
+    b.blk = (int32_t *)malloc((size_t)(rowidx[M] ? rowidx[M] : 1) * sizeof(int32_t));
+    int64_t w = 0;
+    for (int64_t i = 0; i < M; ++i) {
+        b.ptr[i] = w;
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j) {
+            int32_t blk = colidx[j] / bw;
+            /* columns strictly increase within a row, so blocks are non-decreasing: unique = new value */
+            if (w == b.ptr[i] || b.blk[w - 1] != blk) b.blk[w++] = blk;
+        }
+    }
+    b.ptr[M] = w;
+    return b;
+}
+static void free_blocks(blocklists *b) { free(b->ptr); free(b->blk); }
+
+static int64_t ham(const blocklists *b, int64_t x, int64_t y) {
+    int64_t i = b->ptr[x], ie = b->ptr[x + 1], j = b->ptr[y], je = b->ptr[y + 1], common = 0;
+    while (i < ie && j < je) {
+        if (b->blk[i] == b->blk[j]) { ++common; ++i; ++j; }
+        else if (b->blk[i] < b->blk[j]) ++i;
+        else ++j;
+    }
+    return (b->ptr[x + 1] - b->ptr[x]) + (b->ptr[y + 1] - b->ptr[y]) - 2 * common;
+}
+
+/* ------------------------------------------------------------------------------------
+ * Sorts.  (key desc, row id asc): a total order, so qsort's instability is irrelevant.
+ * NNZ_SORT key = nnz_i (north star "nnz-sorted", reading A3); PLAIN_SORT key = wl_i
+ * ("We sort rows by warp load"; descending per reading A1; ties -> lowest
+ * id, "the first of these rows" P:L132, reading A2).
+ * ---------------------------------------------------------------------------------- */
+typedef struct { int64_t key; int64_t id; } keyed;
+static int cmp_desc_key_asc_id(const void *pa, const void *pb) {
+    const keyed *a = (const keyed *)pa, *b = (const keyed *)pb;
+    if (a->key != b->key) return a->key > b->key ? -1 : 1;
+    return (a->id > b->id) - (a->id < b->id);
+}
+static int cmp_asc_key_asc_id(const void *pa, const void *pb) {
+    const keyed *a = (const keyed *)pa, *b = (const keyed *)pb;
+    if (a->key != b->key) return a->key < b->key ? -1 : 1;
+    return (a->id > b->id) - (a->id < b->id);
+}
+static void sort_rows_desc(int64_t M, const int64_t *key, int32_t *out) {
+    keyed *t = (keyed *)malloc((size_t)(M ? M : 1) * sizeof(keyed));
+    for (int64_t i = 0; i < M; ++i) { t[i].key = key[i]; t[i].id = i; }
+    qsort(t, (size_t)M, sizeof(keyed), cmp_desc_key_asc_id);
+    for (int64_t i = 0; i < M; ++i) out[i] = (int32_t)t[i].id;
+    free(t);
+}
+
+/* MinHash pre-order key (reading A11 / SURVEY c2): h_i = min_{b in blocks_i} splitmix64(b XOR seed),
+ * empty rows 2^64-1.  splitmix64 is the standard finaliser (z += golden; two xor-shift-multiplies). */
+static uint64_t splitmix64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+void oracle_minhash_keys(int64_t M, const int64_t *rowidx, const int32_t *colidx, int32_t bw, uint64_t seed,
+                         uint64_t *h) {
+    for (int64_t i = 0; i < M; ++i) {
+        uint64_t m = ~(uint64_t)0;
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j) {
+            uint64_t v = splitmix64((uint64_t)(colidx[j] / bw) ^ seed);
+            if (v < m) m = v;
+        }
+        h[i] = m;
+    }
+}
+typedef struct { uint64_t key; int64_t id; } ukeyed;
+static int cmp_u_asc(const void *pa, const void *pb) {
+    const ukeyed *a = (const ukeyed *)pa, *b = (const ukeyed *)pb;
+    if (a->key != b->key) return a->key < b->key ? -1 : 1;
+    return (a->id > b->id) - (a->id < b->id);
+}
+
+/* ------------------------------------------------------------------------------------
+ * Greedy chains over one window (or segment) `om` of n rows; out receives n rows.
+ *   mode CTA   : CTA-aware Sort: first = argmin (wl, id) (reading A6); then
+ *                next = argmin over unplaced r of (ham(r, prev), id)
+ *   mode H21   : Hybrid-2.1: (ham(r,prev), |wl_r - wl_prev|, id) (readings A9, A10)
+ *   mode H22   : Hybrid-2.2: (ham(r,prev), q>=nw ? ham(r,out[q-nw]) : 0, id)
+ *   mode H1    : Hybrid-1: first = om[0] (segment's first row); then (ham(r,prev), id)
+ *   mode WARP  : Warp-aware Sort: first min(nw,n) = rows of om with smallest
+ *                (wl, id) ascending (reading A7); q>=nw: (ham(r, out[q-nw]), id)
+ *   mode H23   : Hybrid-2.3: Warp-aware with (ham(r,out[q-nw]), |wl_r - wl_out[q-1]|, id)
+ * ---------------------------------------------------------------------------------- */
+enum { M_CTA, M_H21, M_H22, M_H1, M_WARP, M_H23 };
+
+static void chain_window(int mode, const int32_t *om, int64_t n, const blocklists *bl, const int64_t *wl,
+                         int64_t nw, int32_t *out) {
+    if (n == 0) return;
+    char *placed = (char *)calloc((size_t)n, 1);
+    int64_t q0;   /* number of positions filled before the greedy loop */
+    if (mode == M_WARP || mode == M_H23) {
+        int64_t nf = n < nw ? n : nw;
+        keyed *t = (keyed *)malloc((size_t)n * sizeof(keyed));
+        for (int64_t a = 0; a < n; ++a) { t[a].key = wl[om[a]]; t[a].id = om[a]; }
+        qsort(t, (size_t)n, sizeof(keyed), cmp_asc_key_asc_id);
+        for (int64_t q = 0; q < nf; ++q) {
+            out[q] = (int32_t)t[q].id;
+            for (int64_t a = 0; a < n; ++a)
+                if (om[a] == out[q]) placed[a] = 1;
+        }
+        free(t);
+        q0 = nf;
+    } else if (mode == M_H1) {
+        out[0] = om[0];
+        placed[0] = 1;
+        q0 = 1;
+    } else {
+        int64_t best = 0;
+        for (int64_t a = 1; a < n; ++a)
+            if (wl[om[a]] < wl[om[best]] || (wl[om[a]] == wl[om[best]] && om[a] < om[best])) best = a;
+        out[0] = om[best];
+        placed[best] = 1;
+        q0 = 1;
+    }
+    for (int64_t q = q0; q < n; ++q) {
+        int64_t best = -1, bk1 = 0, bk2 = 0;
+        for (int64_t a = 0; a < n; ++a) {
+            if (placed[a]) continue;
+            int64_t r = om[a], k1, k2 = 0;
+            switch (mode) {
+                case M_CTA: case M_H1:
+                    k1 = ham(bl, r, out[q - 1]); break;
+                case M_H21:
+                    k1 = ham(bl, r, out[q - 1]); k2 = llabs(wl[r] - wl[out[q - 1]]); break;
+                case M_H22:
+                    k1 = ham(bl, r, out[q - 1]); k2 = q >= nw ? ham(bl, r, out[q - nw]) : 0; break;
+                case M_WARP:
+                    k1 = ham(bl, r, out[q - nw]); break;
+                default: /* M_H23 */
+                    k1 = ham(bl, r, out[q - nw]); k2 = llabs(wl[r] - wl[out[q - 1]]); break;
+            }
+            if (best < 0 || k1 < bk1 || (k1 == bk1 && (k2 < bk2 || (k2 == bk2 && r < om[best])))) {
+                best = a; bk1 = k1; bk2 = k2;
+            }
+        }
+        out[q] = om[best];
+        placed[best] = 1;
+    }
+    free(placed);
+}
+
+/* ------------------------------------------------------------------------------------
+ * oracle_permute: perm[p] = original row placed at position p (gather form), a bijection.
+ * window W (multiple of nw, 0 = whole matrix, reading A11); preorder 0 = original, 1 = MinHash.
+ * Returns 0 on success, 1 on invalid arguments.
+ * ---------------------------------------------------------------------------------- */
+int oracle_permute(int32_t policy, int64_t M, const int64_t *rowidx, const int32_t *colidx, int32_t nw,
+                   int32_t nt, int32_t bw, int64_t window, int32_t preorder, uint64_t seed, int32_t *perm) {
+    if (nw <= 0 || nt <= 0 || bw <= 0 || window < 0 || (window % nw) != 0) return 1;
+    int64_t *nnz = (int64_t *)malloc((size_t)(M ? M : 1) * sizeof(int64_t));
+    int64_t *wl = (int64_t *)malloc((size_t)(M ? M : 1) * sizeof(int64_t));
+    for (int64_t i = 0; i < M; ++i) { nnz[i] = row_nnz(rowidx, i); wl[i] = warp_load(nnz[i], nt); }
+    int64_t W = (window == 0 || window > M) ? M : window;
+    int rc = 0;
+
+    switch (policy) {
+    case P_IDENTITY:                      /* "original CSR" P:L217, L221 */
+        for (int64_t p = 0; p < M; ++p) perm[p] = (int32_t)p;
+        break;
+    case P_NNZ_SORT:
+        sort_rows_desc(M, nnz, perm);
+        break;
+    case P_PLAIN_SORT:
+        sort_rows_desc(M, wl, perm);
+        break;
+    case P_FLIPPED: {                     /* P:L106 "after every N_w=32 rows ... flipped" (A4) */
+        int32_t *s = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
+        sort_rows_desc(M, wl, s);
+        for (int64_t c = 0; c * nw < M; ++c) {
+            int64_t lo = c * nw, hi = (c + 1) * nw < M ? (c + 1) * nw : M;
+            for (int64_t p = lo; p < hi; ++p) perm[p] = (c & 1) ? s[lo + (hi - 1 - p)] : s[p];
+        }
+        free(s);
+        break;
+    }
+    case P_LPT: {                         /* P:L108 LPT; capacity per warp from row i -> warp i mod nw (A5) */
+        int32_t *s = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
+        sort_rows_desc(M, wl, s);
+        int64_t *load = (int64_t *)calloc((size_t)nw, sizeof(int64_t));
+        int64_t *cnt = (int64_t *)calloc((size_t)nw, sizeof(int64_t));
+        int64_t *cap = (int64_t *)calloc((size_t)nw, sizeof(int64_t));
+        int32_t *lists = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
+        for (int64_t w = 0; w < nw; ++w) cap[w] = M > w ? (M - w + nw - 1) / nw : 0;
+        for (int64_t t = 0; t < M; ++t) {
+            int64_t r = s[t], bw_ = -1;
+            for (int64_t w = 0; w < nw; ++w) {
+                if (cnt[w] >= cap[w]) continue;
+                if (bw_ < 0 || load[w] < load[bw_]) bw_ = w;
+            }
+            load[bw_] += wl[r];
+            /* list_w[k] lives at position k*nw + w */
+            lists[cnt[bw_] * nw + bw_] = (int32_t)r;
+            cnt[bw_]++;
+        }
+        for (int64_t p = 0; p < M; ++p) perm[p] = lists[p];
+        free(s); free(load); free(cnt); free(cap); free(lists);
+        break;
+    }
+    case P_DCSR: {                        /* non-empty rows (rowptr), then empty rows (bijection) */
+        int64_t q = 0;
+        for (int64_t i = 0; i < M; ++i) if (nnz[i] > 0) perm[q++] = (int32_t)i;
+        for (int64_t i = 0; i < M; ++i) if (nnz[i] == 0) perm[q++] = (int32_t)i;
+        break;
+    }
+    case P_CTA_AWARE: case P_HYBRID_2_1: case P_HYBRID_2_2: case P_WARP_AWARE: case P_HYBRID_2_3: {
+        int mode = policy == P_CTA_AWARE ? M_CTA : policy == P_HYBRID_2_1 ? M_H21 :
+                   policy == P_HYBRID_2_2 ? M_H22 : policy == P_WARP_AWARE ? M_WARP : M_H23;
+        blocklists bl = make_blocks(M, rowidx, colidx, bw);
+        int32_t *pre = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
+        if (preorder) {
+            uint64_t *h = (uint64_t *)malloc((size_t)(M ? M : 1) * sizeof(uint64_t));
+            oracle_minhash_keys(M, rowidx, colidx, bw, seed, h);
+            ukeyed *t = (ukeyed *)malloc((size_t)(M ? M : 1) * sizeof(ukeyed));
+            for (int64_t i = 0; i < M; ++i) { t[i].key = h[i]; t[i].id = i; }
+            qsort(t, (size_t)M, sizeof(ukeyed), cmp_u_asc);
+            for (int64_t i = 0; i < M; ++i) pre[i] = (int32_t)t[i].id;
+            free(t); free(h);
+        } else {
+            for (int64_t i = 0; i < M; ++i) pre[i] = (int32_t)i;
+        }
+        int64_t nwin = M ? (M + W - 1) / W : 0;
+#pragma omp parallel for schedule(dynamic, 1)
+        for (int64_t s = 0; s < nwin; ++s) {
+            int64_t lo = s * W, n = (lo + W < M ? lo + W : M) - lo;
+            chain_window(mode, pre + lo, n, &bl, wl, nw, perm + lo);
+        }
+        free(pre);
+        free_blocks(&bl);
+        break;
+    }
+    case P_HYBRID_1: {                    /* P:L132 (reading A8): Plain-Sort runs of equal wl, cut at W */
+        blocklists bl = make_blocks(M, rowidx, colidx, bw);
+        int32_t *s = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
+        sort_rows_desc(M, wl, s);
+        /* segment starts */
+        int64_t *seg = (int64_t *)malloc((size_t)(M + 1) * sizeof(int64_t));
+        int64_t ns = 0, run_start = 0;
+        for (int64_t p = 0; p < M; ++p) {
+            if (p > 0 && wl[s[p]] != wl[s[p - 1]]) run_start = p;
+            if (p == run_start || (p - run_start) % W == 0) seg[ns++] = p;
+        }
+        seg[ns] = M;
+#pragma omp parallel for schedule(dynamic, 1)
+        for (int64_t t = 0; t < ns; ++t)
+            chain_window(M_H1, s + seg[t], seg[t + 1] - seg[t], &bl, wl, nw, perm + seg[t]);
+        free(seg); free(s);
+        free_blocks(&bl);
+        break;
+    }
+    default:
+        rc = 1;
+    }
+    free(nnz); free(wl);
+    return rc;
+}
+
+/* Permuted CSR ("preserve the CSR representation", §III): rowidx'[0]=0,
+ * rowidx'[p+1] = rowidx'[p] + nnz_{perm[p]}; row segments copied in their within-row order. */
+void oracle_permuted_csr(int64_t M, const int64_t *rowidx, const int32_t *colidx, const float *value,
+                         const int32_t *perm, int64_t *rowidx2, int32_t *colidx2, float *value2) {
+    rowidx2[0] = 0;
+    for (int64_t p = 0; p < M; ++p) {
+        int64_t i = perm[p], len = row_nnz(rowidx, i);
+        rowidx2[p + 1] = rowidx2[p] + len;
+        for (int64_t t = 0; t < len; ++t) {
+            colidx2[rowidx2[p] + t] = colidx[rowidx[i] + t];
+            value2[rowidx2[p] + t] = value[rowidx[i] + t];
+        }
+    }
+}
+
+/* ------------------------------------------------------------------------------------
+ * c3. The 24 features of Table II (§V.A), in this order:
+ *  f0 n_row, f1 n_col, f2 density = nnz/(n_row*n_col)
+ *  f3-5  nnz-per-row           min/mean/max over rows
+ *  f6-8  nnz-blocks-per-row    |blocks_i| (blocks of N_w=bw consecutive columns, A14) min/mean/max
+ *  f9-11 warp load             WL_w = sum_{i mod nw = w} ceil(nnz_i/nt), min/mean/max over nw warps
+ *  f12-14 same-cache-lines     requests(b) = sum_i sum_c [b in lines(i,c)] over blocks with >=1
+ *                              request (A12); lines(i,c) = blocks of chunk c (nt consecutive nnz of
+ *                              row i, one warp instruction's coalesced B requests)
+ *  f15-17 distinct-cache-lines-per-warp  D_w = |U_{i mod nw = w} blocks_i|
+ *  f18-20 total-cache-lines-per-warp     T_w = sum_{i mod nw = w} sum_c |lines(i,c)|
+ *  f21-23 adjacent-vector-distance       ham(i, i+1), i < M-1 (A13)
+ * Means are (double)int64 sum / (double)count; an empty population gives 0.
+ * perm != NULL: features of the permuted matrix (row at position p is perm[p]).
+ * ---------------------------------------------------------------------------------- */
+static void stats(const int64_t *v, int64_t n, double *out3) {
+    if (n == 0) { out3[0] = out3[1] = out3[2] = 0.0; return; }
+    int64_t mn = v[0], mx = v[0], sum = 0;
+    for (int64_t t = 0; t < n; ++t) { if (v[t] < mn) mn = v[t]; if (v[t] > mx) mx = v[t]; sum += v[t]; }
+    out3[0] = (double)mn;
+    out3[1] = (double)sum / (double)n;
+    out3[2] = (double)mx;
+}
+
+void oracle_features(int64_t M, int64_t N, const int64_t *rowidx, const int32_t *colidx, const int32_t *perm,
+                     int32_t nw, int32_t nt, int32_t bw, double *f) {
+    int64_t nnz_total = M ? rowidx[M] : 0;
+    int64_t nblk = (N + bw - 1) / bw;
+    blocklists bl = make_blocks(M, rowidx, colidx, bw);
+    int64_t *tmp = (int64_t *)malloc((size_t)(M > nw ? M : nw) * sizeof(int64_t) + 8);
+    f[0] = (double)M;
+    f[1] = (double)N;
+    f[2] = (M && N) ? (double)nnz_total / ((double)M * (double)N) : 0.0;
+    for (int64_t p = 0; p < M; ++p) tmp[p] = row_nnz(rowidx, perm ? perm[p] : p);
+    stats(tmp, M, f + 3);
+    for (int64_t p = 0; p < M; ++p) { int64_t i = perm ? perm[p] : p; tmp[p] = bl.ptr[i + 1] - bl.ptr[i]; }
+    stats(tmp, M, f + 6);
+    for (int64_t w = 0; w < nw; ++w) tmp[w] = 0;
+    for (int64_t p = 0; p < M; ++p) tmp[p % nw] += warp_load(row_nnz(rowidx, perm ? perm[p] : p), nt);
+    stats(tmp, nw, f + 9);
+
+    /* same-cache-lines and total-cache-lines-per-warp: walk each row's nt-nnz chunks */
+    int64_t *req = (int64_t *)calloc((size_t)(nblk ? nblk : 1), sizeof(int64_t));
+    int64_t *T = (int64_t *)calloc((size_t)nw, sizeof(int64_t));
+    for (int64_t p = 0; p < M; ++p) {
+        int64_t i = perm ? perm[p] : p;
+        for (int64_t c0 = rowidx[i]; c0 < rowidx[i + 1]; c0 += nt) {
+            int64_t c1 = c0 + nt < rowidx[i + 1] ? c0 + nt : rowidx[i + 1];
+            for (int64_t j = c0; j < c1; ++j) {
+                int32_t b = colidx[j] / bw;
+                int first = 1;   /* count block b once per chunk */
+                for (int64_t jj = c0; jj < j; ++jj) if (colidx[jj] / bw == b) { first = 0; break; }
+                if (first) { req[b]++; T[p % nw]++; }
+            }
+        }
+    }
+    int64_t nreq = 0;
+    for (int64_t b = 0; b < nblk; ++b) if (req[b] > 0) req[nreq++] = req[b];
+    stats(req, nreq, f + 12);
+    free(req);
+
+    /* distinct-cache-lines-per-warp: a per-warp 0/1 array over blocks */
+    char *seen = (char *)malloc((size_t)(nblk ? nblk : 1));
+    for (int64_t w = 0; w < nw; ++w) {
+        memset(seen, 0, (size_t)(nblk ? nblk : 1));
+        int64_t d = 0;
+        for (int64_t p = w; p < M; p += nw) {
+            int64_t i = perm ? perm[p] : p;
+            for (int64_t t = bl.ptr[i]; t < bl.ptr[i + 1]; ++t)
+                if (!seen[bl.blk[t]]) { seen[bl.blk[t]] = 1; ++d; }
+        }
+        tmp[w] = d;
+    }
+    free(seen);
+    stats(tmp, nw, f + 15);
+    stats(T, nw, f + 18);
+    free(T);
+
+    int64_t na = M > 1 ? M - 1 : 0;
+    for (int64_t p = 0; p < na; ++p) tmp[p] = ham(&bl, perm ? perm[p] : p, perm ? perm[p + 1] : p + 1);
+    stats(tmp, na, f + 21);
+    free(tmp);
+    free_blocks(&bl);
+}
+
+/* c4. Partition by nnz (row-sharded mode, north star (4)):
+ * bounds[0]=0, bounds[P]=M, bounds[p] = min{ r in [0,M] : rowidx[r] >= ceil(p*nnz/P) }. */
+void oracle_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds) {
+    int64_t nnz = rowidx[M];
+    bounds[0] = 0;
+    for (int32_t p = 1; p < P; ++p) {
+        int64_t target = (p * nnz + P - 1) / P;
+        int64_t r = 0;
+        while (r < M && rowidx[r] < target) ++r;
+        bounds[p] = r;
+    }
+    bounds[P] = M;
+}
+
+/* Predictor forward (§V.B: two fully connected hidden layers of 64 and 32, one output per
+ * policy = predicted execution time, then argmin = classification).  Reading A19: inputs
+ * z = (log1p(f) - mu)/sigma, ReLU after layers 1-2.  Flat weight layout:
+ * mu[24] sigma[24] W1[64][24] b1[64] W2[32][64] b2[32] W3[P][32] b3[P].  Returns argmin (ties low). */
+int32_t oracle_mlp_forward(const double *feat, const float *w, int32_t P, double *out) {
+    const float *mu = w, *sg = w + 24, *W1 = w + 48, *b1 = W1 + 64 * 24, *W2 = b1 + 64, *b2 = W2 + 32 * 64,
+                *W3 = b2 + 32, *b3 = W3 + (int64_t)P * 32;
+    double x[24], h1[64], h2[32];
+    for (int i = 0; i < 24; ++i) x[i] = (log1p(feat[i]) - (double)mu[i]) / (double)sg[i];
+    for (int o = 0; o < 64; ++o) {
+        double s = b1[o];
+        for (int i = 0; i < 24; ++i) s += (double)W1[o * 24 + i] * x[i];
+        h1[o] = s > 0 ? s : 0;
+    }
+    for (int o = 0; o < 32; ++o) {
+        double s = b2[o];
+        for (int i = 0; i < 64; ++i) s += (double)W2[o * 64 + i] * h1[i];
+        h2[o] = s > 0 ? s : 0;
+    }
+    int32_t best = 0;
+    for (int o = 0; o < P; ++o) {
+        double s = b3[o];
+        for (int i = 0; i < 32; ++i) s += (double)W3[o * 32 + i] * h2[i];
+        out[o] = s;
+        if (s < out[best]) best = o;
+    }
+    return best;
+}
