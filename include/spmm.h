@@ -1,0 +1,150 @@
+/*
+ * spmm.h -- C ABI of the B200-native row-permuted CSR SpMM library (libspmm_b200.so).
+ *
+ * Method: Mehrabi et al., "Learning Sparse Matrix Row Permutations for Efficient SpMM on GPU
+ * Architectures", ISPASS 2021 (/root/reference/PAPER.md, cited P:L<n> + section).
+ *   C[M][K] = A[M][N] . B[N][K]                      (Alg.1 "Input: CSR A[M][N], float B[N][K]")
+ * computed on a row-PERMUTED copy of the CSR matrix (§III: "re-order rows ... yet preserve
+ * the CSR representation"), the inverse permutation being applied when C is written (C is always in
+ * ORIGINAL row order).  Policies: §III.A load balancing, §III.B cache-aware,
+ * §III.C hybrids, DCSR.  Features: Table II.  Predictor: §V.B
+ * (P:L273-277).  Exact definitions and readings: DESIGN.md §"Readings".
+ *
+ * Conventions for every entry point
+ *   - extern "C", plain pointers and sizes; nothing throws across the ABI; every call returns an
+ *     spmm_status and on failure leaves a detail message in spmm_last_error() (thread-local).
+ *   - "device" pointers are CUDA device addresses on the device that was current when the handle
+ *     was created; "host" pointers are ordinary (preferably pinned) host memory.
+ *   - cuda_stream is a cudaStream_t passed as void* (NULL = legacy default stream).  Every call that
+ *     takes a stream is stream-ordered; calls that return host data synchronise that stream.
+ *   - Layouts: CSR rowidx int64[M+1], colidx int32[nnz] (strictly increasing within a row),
+ *     value float32[nnz].  Dense B float32 row-major [N][K], C float32 row-major [M][K], both
+ *     16-byte aligned, K % 4 == 0, 4 <= K <= 1024 (B rows are read as float4 vectors along K).
+ *   - Limits: 0 <= M, N < 2^31, 0 <= nnz < 2^31 (device offsets are int32).
+ */
+#ifndef SPMM_B200_H
+#define SPMM_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct spmm_ctx *spmm_handle;
+
+typedef enum {
+    SPMM_OK = 0,
+    SPMM_ERR_INVALID_ARG = 1,  /* NULL pointer, negative size, size >= 2^31, bad window/params   */
+    SPMM_ERR_INVALID_CSR = 2,  /* rowidx[0]!=0, rowidx[M]!=nnz, decreasing offsets, column out of
+                                  range, or columns not strictly increasing within a row         */
+    SPMM_ERR_UNSUPPORTED = 3,  /* K % 4 != 0, K > 1024, misaligned B/C, W=0 chain above 32768 rows */
+    SPMM_ERR_CUDA = 4,         /* a CUDA runtime error (text in spmm_last_error)                  */
+    SPMM_ERR_OOM = 5,          /* device allocation failed                                        */
+    SPMM_ERR_STATE = 6         /* handle used on a device other than the one it was created on    */
+} spmm_status;
+
+/* Row-permutation policies.  perm[p] = ORIGINAL row placed at position p (gather form). */
+typedef enum {
+    SPMM_POLICY_IDENTITY = 0,   /* plain CSR order ("original CSR")                     */
+    SPMM_POLICY_NNZ_SORT = 1,   /* stable sort by nnz_i, descending; ties by row id (north star)       */
+    SPMM_POLICY_PLAIN_SORT = 2, /* stable sort by warp load ceil(nnz_i/nt), descending   */
+    SPMM_POLICY_CTA_AWARE = 3,  /* greedy chain: next row = min Hamming to previous row       */
+    SPMM_POLICY_HYBRID_1 = 4,   /* Plain Sort, ties (equal warp load) broken by Hamming       */
+    SPMM_POLICY_HYBRID_2_1 = 5, /* CTA-aware, Hamming ties broken by warp-load difference     */
+    SPMM_POLICY_FLIPPED = 6,    /* Plain Sort with every odd nw-row chunk reversed            */
+    SPMM_POLICY_LPT = 7,        /* LPT: rows in desc. warp load to the least-loaded warp      */
+    SPMM_POLICY_WARP_AWARE = 8, /* row at q minimises Hamming to row q-nw                 */
+    SPMM_POLICY_HYBRID_2_2 = 9, /* CTA-aware, ties broken by Hamming to row q-nw              */
+    SPMM_POLICY_HYBRID_2_3 = 10,/* Warp-aware, ties broken by warp-load difference            */
+    SPMM_POLICY_DCSR = 11,      /* non-empty rows first in original order, then empty rows     */
+    SPMM_POLICY_COUNT = 12
+} spmm_policy;
+
+typedef struct {
+    int32_t nw;             /* warps per CTA in the paper's model, default 32                */
+    int32_t nt;             /* threads per warp, default 32                                  */
+    int32_t bw;             /* columns per B cache-line block, default 32 = 128 B / 4 B */
+    int32_t split_nnz;      /* rows longer than this are cut into chunks of this many nnz whose
+                               partial sums are combined in a fixed pairwise order; default 128
+                               (bounds every fp32 accumulation chain, DESIGN.md §"Accuracy")         */
+    int64_t window;         /* greedy-chain window W (multiple of nw); 0 = whole matrix (paper-exact,
+                               supported up to 32768 rows); default 1024                               */
+    int32_t preorder;       /* chain policies: 0 = windows over the original order, 1 = MinHash key  */
+    int32_t reserved;
+    uint64_t seed;          /* MinHash seed                                                          */
+} spmm_params;
+
+/* Fill *p with the defaults (nw=nt=bw=32, split_nnz=128, window=1024, preorder=0, seed=0). */
+spmm_status spmm_default_params(spmm_params *p);
+
+/* Optional device allocator (e.g. PyTorch's caching allocator).  alloc(bytes, stream, ctx) returns a
+ * device pointer or NULL; free_(ptr, stream, ctx) releases it stream-ordered.  Pass NULLs to restore
+ * the built-in cudaMallocAsync allocator.  Process-wide; set it before creating handles. */
+spmm_status spmm_set_allocator(void *(*alloc)(size_t bytes, void *stream, void *ctx),
+                               void (*free_)(void *ptr, void *stream, void *ctx), void *ctx);
+
+/* Create a handle: copies and validates the CSR (§II.A) into handle-owned device memory
+ * (inputs_on_device = 1: the three arrays are device pointers, else host pointers; caller buffers
+ * may be freed on return).  Synchronises cuda_stream (validation result).  The current policy is
+ * IDENTITY until spmm_permute is called. */
+spmm_status spmm_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, const int64_t *rowidx,
+                        const int32_t *colidx, const float *value, int inputs_on_device, void *cuda_stream);
+
+/* Build permutation `policy` (params NULL = defaults) and the permuted CSR + long-row chunk table it
+ * implies, all on the device (offline / amortised).  Replaces the previous permutation.
+ * Needs external synchronisation against spmm_run on the same handle. */
+spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *params, void *cuda_stream);
+
+/* Copy the current permutation (M int32, HOST buffer).  Synchronises. */
+spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out);
+
+/* Copy the current permuted CSR to HOST buffers: rowidx int64[M+1], colidx int32[nnz], value f32[nnz]. */
+spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colidx, float *value);
+
+/* Counters of the current permutation: out[0]=rows with nnz==0, out[1]=rows handled whole,
+ * out[2]=split (long) rows, out[3]=chunks of the split rows, out[4]=max row nnz. */
+spmm_status spmm_get_info(spmm_handle h, int64_t out[5]);
+
+/* The 24 Table II features (definitions DESIGN.md §"Features") computed on the device,
+ * of the ORIGINAL order (use_current_order = 0) or of the current permutation (1), with nw/nt/bw from
+ * params (NULL = 32/32/32).  out: 24 doubles, HOST.  Synchronises cuda_stream. */
+spmm_status spmm_features(spmm_handle h, int use_current_order, const spmm_params *params, double out[24],
+                          void *cuda_stream);
+
+/* C = A . B on the device (beta = 0: C is fully overwritten; empty rows get zeros).
+ * B: device, float32 row-major [N][K]; C: device, float32 row-major [M][K] in ORIGINAL row order.
+ * Asynchronous on cuda_stream; reads the handle only, but shares its long-row scratch, so calls on
+ * one handle must be ordered (same stream or external synchronisation). */
+spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream);
+
+/* End-to-end variant: B_host -> device, spmm_run, C -> C_host, all on cuda_stream with handle-owned
+ * staging buffers (grown on demand).  Host buffers should be pinned for full copy bandwidth.
+ * Synchronises cuda_stream before returning. */
+spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *C_host, void *cuda_stream);
+
+/* Predictor inference (§V.B): z = (log1p(f) - mu)/sigma; h1 = relu(W1 z + b1) (64);
+ * h2 = relu(W2 h1 + b2) (32); t = W3 h2 + b3 (n_policies predicted times); policy = argmin t, ties to
+ * the lowest index.  weights: HOST float32, flat mu[24] sigma[24] W1[64][24] b1[64] W2[32][64] b2[32]
+ * W3[P][32] b3[P]; n_weights must equal 48+1536+64+2048+32+33*P.  times_out may be NULL. */
+spmm_status spmm_predict(const double features[24], const float *mlp_weights, int64_t n_weights,
+                         int32_t n_policies, int32_t *policy_out, double *times_out);
+
+/* Row-sharded mode (north star (4)): bounds[0]=0, bounds[P]=M,
+ * bounds[p] = min{ r : rowidx[r] >= ceil(p*nnz/P) }.  rowidx: HOST int64[M+1]; bounds: HOST int64[P+1]. */
+spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds);
+
+/* Release the handle and all its device memory (stream-ordered on the creation stream). */
+spmm_status spmm_destroy(spmm_handle h);
+
+const char *spmm_status_string(spmm_status s);
+const char *spmm_last_error(void);
+
+/* Number of kernel launches issued by the most recent spmm_run on this thread (bench accounting). */
+int32_t spmm_last_run_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPMM_B200_H */

@@ -1,0 +1,290 @@
+"""Thin Python binding of libspmm_b200.so (include/spmm.h) -- argument marshalling only.
+
+Every step of the hot path runs in the CUDA library; this module only converts
+numpy arrays / torch tensors to pointers, passes torch's current CUDA stream,
+and (optionally) routes the library's device allocations through PyTorch's
+caching allocator.  There is NO CPU fallback: if the extension cannot be loaded
+every entry point raises.
+
+Names follow the C ABI (``spmm_create``, ``spmm_permute``, ``spmm_run`` ...);
+``SpMM`` is a convenience object wrapping one handle.
+Paper: Mehrabi et al., ISPASS 2021; see include/spmm.h for the
+passage each entry point implements.
+"""
+from __future__ import annotations
+
+import atexit
+import ctypes
+import os
+import weakref
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libspmm_b200.so")
+
+POLICIES = {
+    "identity": 0, "nnz_sort": 1, "plain_sort": 2, "cta_aware": 3, "hybrid_1": 4, "hybrid_2_1": 5,
+    "flipped": 6, "lpt": 7, "warp_aware": 8, "hybrid_2_2": 9, "hybrid_2_3": 10, "dcsr": 11,
+}
+POLICY_NAMES = {v: k for k, v in POLICIES.items()}
+HOT_PATH_POLICIES = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1"]
+
+STATUS = {0: "SPMM_OK", 1: "SPMM_ERR_INVALID_ARG", 2: "SPMM_ERR_INVALID_CSR", 3: "SPMM_ERR_UNSUPPORTED",
+          4: "SPMM_ERR_CUDA", 5: "SPMM_ERR_OOM", 6: "SPMM_ERR_STATE"}
+
+FEATURE_NAMES = (["n_row", "n_col", "density"]
+                 + [f"{n}_{s}" for n in ("nnz_per_row", "nnz_blocks_per_row", "warp_load", "same_cache_lines",
+                                         "distinct_cache_lines_per_warp", "total_cache_lines_per_warp",
+                                         "adjacent_vector_distance") for s in ("min", "mean", "max")])
+
+
+class SpmmError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        self.status = status
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+
+
+class _Params(ctypes.Structure):
+    _fields_ = [("nw", ctypes.c_int32), ("nt", ctypes.c_int32), ("bw", ctypes.c_int32), ("split_nnz", ctypes.c_int32),
+                ("window", ctypes.c_int64), ("preorder", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("seed", ctypes.c_uint64)]
+
+
+_lib = None
+_ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+_alloc_cbs = None
+EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_predict",
+           "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
+           "spmm_last_run_launches"]
+
+
+def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load libspmm_b200.so (raises if missing -- there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    lib = ctypes.CDLL(path)
+    vp, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    st = ctypes.c_int
+    sig = {
+        "spmm_default_params": (st, [vp]),
+        "spmm_set_allocator": (st, [_ALLOC_T, _FREE_T, vp]),
+        "spmm_create": (st, [vp, i64, i64, i64, vp, vp, vp, ctypes.c_int, vp]),
+        "spmm_permute": (st, [vp, ctypes.c_int, vp, vp]),
+        "spmm_get_perm": (st, [vp, vp]),
+        "spmm_get_permuted_csr": (st, [vp, vp, vp, vp]),
+        "spmm_get_info": (st, [vp, vp]),
+        "spmm_features": (st, [vp, ctypes.c_int, vp, vp, vp]),
+        "spmm_run": (st, [vp, vp, i64, vp, vp]),
+        "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
+        "spmm_predict": (st, [vp, vp, i64, i32, vp, vp]),
+        "spmm_partition_by_nnz": (st, [vp, i64, i32, vp]),
+        "spmm_destroy": (st, [vp]),
+        "spmm_status_string": (ctypes.c_char_p, [st]),
+        "spmm_last_error": (ctypes.c_char_p, []),
+        "spmm_last_run_launches": (i32, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = lib
+    return lib
+
+
+def _check(status: int):
+    if status != 0:
+        raise SpmmError(status, load_library().spmm_last_error().decode(errors="replace"))
+
+
+def use_torch_allocator(enable: bool = True):
+    """Route the library's device allocations through torch's caching allocator (stream-ordered)."""
+    global _alloc_cbs
+    lib = load_library()
+    if not enable:
+        _check(lib.spmm_set_allocator(_ALLOC_T(), _FREE_T(), None))
+        _alloc_cbs = None
+        return
+    import torch
+
+    def _a(nbytes, stream, ctx):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), torch.cuda.current_device(), stream or 0)
+        except Exception:   # noqa: BLE001 -- report as NULL -> SPMM_ERR_OOM
+            return None
+
+    def _f(ptr, stream, ctx):
+        try:
+            torch.cuda.caching_allocator_delete(ptr)
+        except Exception:   # noqa: BLE001
+            pass
+
+    _alloc_cbs = (_ALLOC_T(_a), _FREE_T(_f))
+    _check(lib.spmm_set_allocator(_alloc_cbs[0], _alloc_cbs[1], None))
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def make_params(nw=32, nt=32, bw=32, split_nnz=128, window=1024, preorder=0, seed=0) -> _Params:
+    p = _Params()
+    _check(load_library().spmm_default_params(ctypes.byref(p)))
+    p.nw, p.nt, p.bw, p.split_nnz, p.window, p.preorder, p.seed = nw, nt, bw, split_nnz, window, preorder, seed
+    return p
+
+
+def _ptr(a):
+    """(pointer, on_device, keepalive) of a numpy array or torch tensor."""
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data, False, a
+    return a.data_ptr(), bool(a.is_cuda), a
+
+
+_live = weakref.WeakSet()
+
+
+class SpMM:
+    """One spmm_handle: create (a1) -> permute (a2-a7) -> run (a8) / features (a9)."""
+
+    def __init__(self, M, N, rowidx, colidx, value, stream=None):
+        import torch  # noqa: F401  (device / stream plumbing)
+        lib = load_library()
+        if isinstance(rowidx, np.ndarray):
+            rowidx = np.ascontiguousarray(rowidx, dtype=np.int64)
+            colidx = np.ascontiguousarray(colidx, dtype=np.int32)
+            value = np.ascontiguousarray(value, dtype=np.float32)
+        r, on_dev, _k1 = _ptr(rowidx)
+        c, _, _k2 = _ptr(colidx)
+        v, _, _k3 = _ptr(value)
+        nnz = int(rowidx[-1]) if M > 0 else 0
+        self._h = ctypes.c_void_p()
+        self.M, self.N, self.nnz = int(M), int(N), nnz
+        _check(lib.spmm_create(ctypes.byref(self._h), self.M, self.N, nnz, r, c, v, int(on_dev), _stream_ptr(stream)))
+        self.policy = "identity"
+        _live.add(self)
+
+    @classmethod
+    def from_csr(cls, csr, stream=None):
+        return cls(csr.M, csr.N, csr.rowidx, csr.colidx, csr.value, stream=stream)
+
+    def permute(self, policy, stream=None, **params):
+        pid = POLICIES[policy] if isinstance(policy, str) else int(policy)
+        p = make_params(**params)
+        _check(load_library().spmm_permute(self._h, pid, ctypes.byref(p), _stream_ptr(stream)))
+        self.policy = POLICY_NAMES[pid]
+        return self
+
+    def perm(self) -> np.ndarray:
+        out = np.empty(self.M, dtype=np.int32)
+        _check(load_library().spmm_get_perm(self._h, out.ctypes.data))
+        return out
+
+    def permuted_csr(self):
+        r = np.empty(self.M + 1, dtype=np.int64)
+        c = np.empty(self.nnz, dtype=np.int32)
+        v = np.empty(self.nnz, dtype=np.float32)
+        _check(load_library().spmm_get_permuted_csr(self._h, r.ctypes.data, c.ctypes.data, v.ctypes.data))
+        return r, c, v
+
+    def info(self) -> dict:
+        out = np.empty(5, dtype=np.int64)
+        _check(load_library().spmm_get_info(self._h, out.ctypes.data))
+        return dict(empty_rows=int(out[0]), whole_rows=int(out[1]), split_rows=int(out[2]), chunks=int(out[3]),
+                    max_row_nnz=int(out[4]))
+
+    def features(self, current_order=False, nw=32, nt=32, bw=32, stream=None) -> np.ndarray:
+        out = np.empty(24, dtype=np.float64)
+        p = make_params(nw=nw, nt=nt, bw=bw, window=0)
+        _check(load_library().spmm_features(self._h, int(bool(current_order)), ctypes.byref(p), out.ctypes.data,
+                                            _stream_ptr(stream)))
+        return out
+
+    def run(self, B, C=None, stream=None):
+        """C = A.B on the device (B: cuda float32 [N, K] row-major). Returns C (cuda float32 [M, K])."""
+        import torch
+        K = int(B.shape[1])
+        if C is None:
+            C = torch.empty((self.M, K), dtype=torch.float32, device=B.device)
+        _check(load_library().spmm_run(self._h, B.data_ptr(), K, C.data_ptr(), _stream_ptr(stream)))
+        return C
+
+    def run_host(self, B_host, C_host, stream=None):
+        """End-to-end: host B -> device, SpMM, device -> host C (host buffers, ideally pinned)."""
+        K = int(B_host.shape[1])
+        b, _, _ = _ptr(B_host)
+        c, _, _ = _ptr(C_host)
+        _check(load_library().spmm_run_host(self._h, b, K, c, _stream_ptr(stream)))
+        return C_host
+
+    @staticmethod
+    def last_run_launches() -> int:
+        return int(load_library().spmm_last_run_launches())
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            load_library().spmm_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:   # noqa: BLE001 -- interpreter shutdown
+            pass
+
+
+@atexit.register
+def _close_all():
+    for h in list(_live):
+        try:
+            h.close()
+        except Exception:   # noqa: BLE001
+            pass
+
+
+def spmm_predict(features, weights, n_policies):
+    """Predictor inference in the library: returns (policy id, predicted times)."""
+    f = np.ascontiguousarray(features, dtype=np.float64)
+    w = np.ascontiguousarray(weights, dtype=np.float32)
+    pol = ctypes.c_int32()
+    times = np.empty(n_policies, dtype=np.float64)
+    _check(load_library().spmm_predict(f.ctypes.data, w.ctypes.data, len(w), n_policies, ctypes.byref(pol),
+                                       times.ctypes.data))
+    return int(pol.value), times
+
+
+def spmm_partition_by_nnz(rowidx, P: int) -> np.ndarray:
+    r = np.ascontiguousarray(rowidx, dtype=np.int64)
+    b = np.empty(P + 1, dtype=np.int64)
+    _check(load_library().spmm_partition_by_nnz(r.ctypes.data, len(r) - 1, P, b.ctypes.data))
+    return b
+
+
+def spmm_create(M, N, rowidx, colidx, value, stream=None) -> SpMM:
+    return SpMM(M, N, rowidx, colidx, value, stream=stream)
+
+
+def spmm_permute(h: SpMM, policy, stream=None, **params) -> SpMM:
+    return h.permute(policy, stream=stream, **params)
+
+
+def spmm_run(h: SpMM, B, C=None, stream=None):
+    return h.run(B, C, stream=stream)
+
+
+def spmm_features(h: SpMM, current_order=False, **kw):
+    return h.features(current_order, **kw)
+
+
+def spmm_destroy(h: SpMM):
+    h.close()

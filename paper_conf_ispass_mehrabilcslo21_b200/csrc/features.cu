@@ -1,0 +1,226 @@
+// features.cu -- the 24 sparsity features of Table II (§V.A) on the device
+// (a9; K10 in §2.4).  All counting is integer and exact; means are formed on the host
+// as (double)int64_sum / (double)count, so the result is bit-identical to the oracle.
+//   f0-2   n_row, n_col, density
+//   f3-5   nnz-per-row                  min/mean/max over rows
+//   f6-8   nnz-blocks-per-row           |blocks_i|, blocks of bw columns (reading A14)
+//   f9-11  warp load                    WL_w = sum_{p mod nw = w} ceil(nnz_p/nt) (Tab.II)
+//   f12-14 same-cache-lines             requests per B line over lines with >= 1 request; a request =
+//                                       one nt-nnz chunk of a row touching the line (A12)
+//   f15-17 distinct-cache-lines-per-warp |union of blocks of rows p = w mod nw|
+//   f18-20 total-cache-lines-per-warp   sum over the warp's rows and chunks of distinct lines per chunk
+//   f21-23 adjacent-vector-distance     Hamming(mask_p, mask_{p+1}) (A13)
+// "row p" is original row p (use_current_order = 0) or the row at position p of the current permutation.
+#include "internal.cuh"
+#include <algorithm>
+#include <vector>
+
+namespace spmm {
+namespace {
+
+struct Stats {
+    unsigned long long mn, mx, sum, cnt;
+};
+
+__device__ __forceinline__ void stats_add(Stats *st, long long v) {
+    atomicMin(&st->mn, (unsigned long long)v);
+    atomicMax(&st->mx, (unsigned long long)v);
+    atomicAdd(&st->sum, (unsigned long long)v);
+    atomicAdd(&st->cnt, 1ULL);
+}
+
+// warp-aggregated stats of non-negative values
+__device__ __forceinline__ void warp_stats(Stats *st, long long v, bool valid) {
+    unsigned long long mn = valid ? (unsigned long long)v : ~0ULL, mx = valid ? (unsigned long long)v : 0ULL;
+    unsigned long long sm = valid ? (unsigned long long)v : 0ULL, c = valid ? 1ULL : 0ULL;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        sm += __shfl_xor_sync(0xffffffffu, sm, o);
+        c += __shfl_xor_sync(0xffffffffu, c, o);
+    }
+    if ((threadIdx.x & 31) == 0 && c) {
+        atomicMin(&st->mn, mn);
+        atomicMax(&st->mx, mx);
+        atomicAdd(&st->sum, sm);
+        atomicAdd(&st->cnt, c);
+    }
+}
+
+// access to "row p": (start, end) and column j of the chosen CSR
+struct OrigCSR {
+    const int32_t *rowidx, *colidx, *perm;   // perm == nullptr: identity
+    __device__ int32_t row(int64_t p) const { return perm ? perm[p] : (int32_t)p; }
+    __device__ int32_t begin(int64_t p) const { return rowidx[row(p)]; }
+    __device__ int32_t end(int64_t p) const { return rowidx[row(p) + 1]; }
+    __device__ int32_t col(int32_t j) const { return colidx[j]; }
+};
+
+// per row p (warp): nnz, distinct blocks, warp load into WL[p % nw], distinct lines per nt-chunk
+// (requests per line and T[p % nw]), union bitmap per warp-class (D), all exact integers.
+__global__ void k_feat_rows(OrigCSR A, int64_t M, int32_t nw, int32_t nt, int32_t bw, int64_t words, Stats *st_nnz,
+                            Stats *st_blk, unsigned long long *WL, unsigned long long *T, unsigned int *req,
+                            uint32_t *Dmap, int32_t *nblk_row) {
+    const int lane = threadIdx.x & 31;
+    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw_total = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t p0 = wid * 32; p0 < M; p0 += nw_total * 32) {
+        // 32 rows per warp iteration; per-row stats aggregated across lanes first
+        int32_t my_nnz = 0, my_blk = 0;
+        bool my_valid = false;
+        for (int r = 0; r < 32; ++r) {
+            const int64_t p = p0 + r;
+            if (p >= M) break;
+            const int32_t a = A.begin(p), b = A.end(p);
+            const int w = (int)(p % nw);
+            int32_t blocks = 0, lines = 0;
+            for (int32_t j0 = a; j0 < b; j0 += 32) {
+                const int32_t j = j0 + lane;
+                const bool in = j < b;
+                const int32_t blk = in ? A.col(j) / bw : -1;
+                const int32_t prv = (in && j > a) ? A.col(j - 1) / bw : -2;
+                const bool newblk = in && (j == a || blk != prv);
+                // chunk boundary: chunk = (j - a) / nt; first nnz of a chunk always counts as a new line
+                const bool chunk_first = in && ((j - a) % nt == 0);
+                const bool newline = in && (chunk_first || blk != prv);
+                blocks += __popc(__ballot_sync(0xffffffffu, newblk));
+                lines += __popc(__ballot_sync(0xffffffffu, newline));
+                if (newline) atomicAdd(&req[blk], 1u);
+                if (newblk) atomicOr(&Dmap[(size_t)w * words + (blk >> 5)], 1u << (blk & 31));
+            }
+            if (lane == 0) {
+                atomicAdd(&WL[w], (unsigned long long)((b - a + nt - 1) / nt));
+                atomicAdd(&T[w], (unsigned long long)lines);
+                nblk_row[p] = blocks;
+            }
+            if (lane == r) { my_nnz = b - a; my_blk = blocks; my_valid = true; }
+        }
+        warp_stats(st_nnz, my_nnz, my_valid);
+        warp_stats(st_blk, my_blk, my_valid);
+    }
+}
+
+// stats over an unsigned array (skip zeros when requested)
+__global__ void k_stats_u32(const unsigned int *v, int64_t n, int skip_zero, Stats *st) {
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x; i0 < n; i0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = i0 + threadIdx.x;
+        const bool in = i < n;
+        const unsigned int x = in ? v[i] : 0u;
+        warp_stats(st, x, in && (!skip_zero || x > 0));
+    }
+}
+
+__global__ void k_popcount_rows(const uint32_t *Dmap, int64_t words, unsigned long long *D) {
+    // one block per warp-class w
+    unsigned long long c = 0;
+    for (int64_t t = threadIdx.x; t < words; t += blockDim.x) c += __popc(Dmap[(size_t)blockIdx.x * words + t]);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(&D[blockIdx.x], c);
+}
+
+// adjacent-vector distance: Hamming(p, p+1) = |b_p| + |b_{p+1}| - 2|common|, merge of the two sorted
+// (non-decreasing, duplicated) block sequences; thread per pair
+__global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk_row, Stats *st) {
+    for (int64_t p0 = (int64_t)blockIdx.x * blockDim.x; p0 < M - 1; p0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t p = p0 + threadIdx.x;
+        long long hd = 0;
+        const bool in = p < M - 1;
+        if (in) {
+            int32_t i = A.begin(p), ie = A.end(p), j = A.begin(p + 1), je = A.end(p + 1);
+            int32_t common = 0;
+            while (i < ie && j < je) {
+                const int32_t x = A.col(i) / bw, y = A.col(j) / bw;
+                if (x == y) {
+                    ++common;
+                    while (i < ie && A.col(i) / bw == x) ++i;
+                    while (j < je && A.col(j) / bw == y) ++j;
+                } else if (x < y) {
+                    ++i;
+                } else {
+                    ++j;
+                }
+            }
+            hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * common;
+        }
+        warp_stats(st, hd, in);
+    }
+}
+
+void put3(double *out, const Stats &s, bool empty_zero = true) {
+    if (s.cnt == 0 && empty_zero) { out[0] = out[1] = out[2] = 0.0; return; }
+    out[0] = (double)(long long)s.mn;
+    out[1] = (double)(long long)s.sum / (double)(long long)s.cnt;
+    out[2] = (double)(long long)s.mx;
+}
+
+void put3_vec(double *out, const std::vector<unsigned long long> &v) {
+    if (v.empty()) { out[0] = out[1] = out[2] = 0.0; return; }
+    unsigned long long mn = v[0], mx = v[0], sm = 0;
+    for (auto x : v) { mn = std::min(mn, x); mx = std::max(mx, x); sm += x; }
+    out[0] = (double)(long long)mn;
+    out[1] = (double)(long long)sm / (double)v.size();
+    out[2] = (double)(long long)mx;
+}
+
+}  // namespace
+
+spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24], cudaStream_t s) {
+    const int64_t M = h->M, N = h->N, nnz = h->nnz;
+    const int32_t nw = p.nw, nt = p.nt, bw = p.bw;
+    out[0] = (double)M;
+    out[1] = (double)N;
+    out[2] = (M && N) ? (double)nnz / ((double)M * (double)N) : 0.0;
+    for (int i = 3; i < 24; ++i) out[i] = 0.0;
+    if (M == 0) return SPMM_OK;
+    const int64_t nblk = ceil_div(N, bw);
+    const int64_t words = std::max<int64_t>(1, ceil_div(nblk, 32));
+    DevBuf st, wl, tt, dd, req, dmap, nbr;
+    SPMM_TRY(st.alloc(4 * sizeof(Stats), s));
+    SPMM_TRY(wl.alloc(nw * sizeof(unsigned long long), s));
+    SPMM_TRY(tt.alloc(nw * sizeof(unsigned long long), s));
+    SPMM_TRY(dd.alloc(nw * sizeof(unsigned long long), s));
+    SPMM_TRY(req.alloc(std::max<int64_t>(nblk, 1) * sizeof(unsigned int), s));
+    SPMM_TRY(dmap.alloc((size_t)nw * words * sizeof(uint32_t), s));
+    SPMM_TRY(nbr.alloc(M * sizeof(int32_t), s));
+    Stats init[4];
+    for (auto &x : init) { x.mn = ~0ULL; x.mx = 0; x.sum = 0; x.cnt = 0; }
+    SPMM_CUDA(cudaMemcpyAsync(st.p, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    SPMM_CUDA(cudaMemsetAsync(wl.p, 0, wl.bytes, s));
+    SPMM_CUDA(cudaMemsetAsync(tt.p, 0, tt.bytes, s));
+    SPMM_CUDA(cudaMemsetAsync(dd.p, 0, dd.bytes, s));
+    SPMM_CUDA(cudaMemsetAsync(req.p, 0, req.bytes, s));
+    SPMM_CUDA(cudaMemsetAsync(dmap.p, 0, dmap.bytes, s));
+    OrigCSR A{h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), current_order ? h->perm.as<int32_t>() : nullptr};
+    Stats *S = st.as<Stats>();   // 0 nnz/row, 1 blocks/row, 2 requests, 3 adjacent
+    const unsigned gw = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(M, 32 * 8), 148 * 16));
+    k_feat_rows<<<gw, 256, 0, s>>>(A, M, nw, nt, bw, words, S + 0, S + 1, wl.as<unsigned long long>(),
+                                   tt.as<unsigned long long>(), req.as<unsigned int>(), dmap.as<uint32_t>(),
+                                   nbr.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    k_stats_u32<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(nblk, 256), 148 * 16)), 256, 0, s>>>(
+        req.as<unsigned int>(), nblk, 1, S + 2);
+    k_popcount_rows<<<nw, 256, 0, s>>>(dmap.as<uint32_t>(), words, dd.as<unsigned long long>());
+    if (M > 1)
+        k_adjacent<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(M, 256), 148 * 16)), 256, 0, s>>>(
+            A, M, bw, nbr.as<int32_t>(), S + 3);
+    SPMM_CUDA(cudaGetLastError());
+    Stats hs[4];
+    std::vector<unsigned long long> hwl(nw), htt(nw), hdd(nw);
+    SPMM_CUDA(cudaMemcpyAsync(hs, st.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
+    SPMM_CUDA(cudaMemcpyAsync(hwl.data(), wl.p, wl.bytes, cudaMemcpyDeviceToHost, s));
+    SPMM_CUDA(cudaMemcpyAsync(htt.data(), tt.p, tt.bytes, cudaMemcpyDeviceToHost, s));
+    SPMM_CUDA(cudaMemcpyAsync(hdd.data(), dd.p, dd.bytes, cudaMemcpyDeviceToHost, s));
+    SPMM_CUDA(cudaStreamSynchronize(s));
+    put3(out + 3, hs[0]);
+    put3(out + 6, hs[1]);
+    put3_vec(out + 9, hwl);
+    put3(out + 12, hs[2]);
+    put3_vec(out + 15, hdd);
+    put3_vec(out + 18, htt);
+    put3(out + 21, hs[3]);
+    return SPMM_OK;
+}
+
+}  // namespace spmm

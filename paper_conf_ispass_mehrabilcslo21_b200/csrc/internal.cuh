@@ -1,0 +1,120 @@
+// internal.cuh -- shared internals of libspmm_b200 (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stddef.h>
+#include <string>
+#include "../../include/spmm.h"
+
+namespace spmm {
+
+// ---- error plumbing -------------------------------------------------------------------------
+void set_error(const std::string &msg);
+spmm_status fail(spmm_status s, const std::string &msg);
+spmm_status cuda_fail(cudaError_t e, const char *what);
+
+#define SPMM_CUDA(call)                                                   \
+    do {                                                                  \
+        cudaError_t e_ = (call);                                          \
+        if (e_ != cudaSuccess) return ::spmm::cuda_fail(e_, #call);       \
+    } while (0)
+#define SPMM_TRY(call)                                                    \
+    do {                                                                  \
+        spmm_status s_ = (call);                                          \
+        if (s_ != SPMM_OK) return s_;                                     \
+    } while (0)
+
+// ---- allocation (optional user hook, else cudaMallocAsync) ------------------------------------
+void *dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void *p, cudaStream_t s);
+
+// RAII device buffer (stream-ordered free)
+struct DevBuf {
+    void *p = nullptr;
+    size_t bytes = 0;
+    cudaStream_t s = nullptr;
+    DevBuf() = default;
+    DevBuf(const DevBuf &) = delete;
+    DevBuf &operator=(const DevBuf &) = delete;
+    ~DevBuf() { release(); }
+    spmm_status alloc(size_t n, cudaStream_t st) {
+        release();
+        s = st;
+        bytes = n;
+        if (n == 0) return SPMM_OK;
+        p = dev_alloc(n, st);
+        if (!p) { bytes = 0; return fail(SPMM_ERR_OOM, "device allocation of " + std::to_string(n) + " bytes failed"); }
+        return SPMM_OK;
+    }
+    void release() {
+        if (p) dev_free(p, s);
+        p = nullptr;
+        bytes = 0;
+    }
+    template <class T> T *as() const { return reinterpret_cast<T *>(p); }
+};
+
+// ---- the handle -----------------------------------------------------------------------------
+struct LongRows {
+    int64_t n_long = 0;       // rows with nnz > split_nnz
+    int64_t n_chunks = 0;     // total chunks over those rows
+    DevBuf chunk_start;       // int32[n_chunks]  start offset into the permuted CSR
+    DevBuf chunk_len;         // int32[n_chunks]
+    DevBuf long_pos;          // int32[n_long]    position p of each long row
+    DevBuf long_chunk_ptr;    // int32[n_long+1]  chunk range of each long row
+};
+
+}  // namespace spmm
+
+struct spmm_ctx {
+    int device = 0;
+    cudaStream_t create_stream = nullptr;
+    int64_t M = 0, N = 0, nnz = 0;
+    int32_t max_row_nnz = 0;
+    int64_t n_empty = 0;
+    // original CSR on the device
+    spmm::DevBuf rowidx;   // int32[M+1]
+    spmm::DevBuf colidx;   // int32[nnz]
+    spmm::DevBuf value;    // float[nnz]
+    // current permutation and its permuted CSR (internal interleaved layout)
+    spmm_policy policy = SPMM_POLICY_IDENTITY;
+    spmm_params params{};
+    spmm::DevBuf perm;     // int32[M]
+    spmm::DevBuf rowptr_p; // int32[M+1]
+    spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
+    spmm::LongRows lr;
+    // run scratch (partials of split rows), grown on demand
+    spmm::DevBuf partials;
+    // host-run staging
+    spmm::DevBuf stage_B, stage_C;
+    int num_sms = 148;
+};
+
+namespace spmm {
+
+// kernels / device algorithms (defined in the .cu files)
+spmm_status exclusive_scan_i32(const int32_t *in, int32_t *out, int64_t n, int32_t *total_host,
+                               cudaStream_t s);   // out[n] = total when out has n+1 slots
+spmm_status exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, cudaStream_t s);
+spmm_status reduce_max_i32(const int32_t *in, int64_t n, int32_t *result_host, cudaStream_t s);
+spmm_status radix_sort_pairs(uint64_t *keys, uint32_t *vals, int64_t n, int begin_bit, int end_bit,
+                             cudaStream_t s);     // stable, ascending, in place (uses scratch)
+
+spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, cudaStream_t s);
+spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s);
+spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24],
+                             cudaStream_t s);
+spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches);
+
+// signatures of the rows (sorted unique col/bw), used by chains and features
+struct Signatures {
+    DevBuf ptr;   // int32[M+1]
+    DevBuf blk;   // int32[S]
+    int64_t S = 0;
+};
+spmm_status build_signatures(const int32_t *rowidx, const int32_t *colidx, const int32_t *order, int64_t M,
+                             int64_t nnz, int32_t bw, Signatures &sig, cudaStream_t s);
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace spmm

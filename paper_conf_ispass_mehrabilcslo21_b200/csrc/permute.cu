@@ -1,0 +1,580 @@
+// permute.cu -- device builders for the row permutations of PAPER.md §III and the
+// permuted CSR they imply ("preserve the CSR representation").
+//
+//   a2 row keys (K1)          nnz_i, warp load wl_i = ceil(nnz_i/nt)            (§II.C)
+//   a3 load-balance orders    NNZ_SORT / PLAIN_SORT: stable radix sort, desc key (reading A1-A3)
+//                             FLIPPED, LPT (reading A5), DCSR
+//   a4 signatures (K3)        blocks_i = sorted unique col/bw
+//   a5 locality orders (K4)   windowed greedy chains, one CTA per window/segment: CTA_AWARE,
+//                             HYBRID_1, HYBRID_2_1/2_2, WARP_AWARE,
+//                             HYBRID_2_3; Hamming = |a|+|b|-2|a∩b| with the reference row's
+//                             blocks held as a bitmap in shared memory ("Hamming distance (XOR)")
+//   a6 permuted CSR (K5)      rowptr' = scan(nnz[perm]), (col,val) segments gathered, interleaved int2
+//   a7 long-row chunks (K6)   rows with nnz > split_nnz cut into split_nnz chunks
+// Every argmin is over a total order ending in the original row id, so the result is deterministic
+// and bit-identical to the oracle (DESIGN.md §"Readings").
+#include "internal.cuh"
+#include <algorithm>
+#include <vector>
+
+namespace spmm {
+namespace {
+
+__global__ void k_iota(int32_t *p, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = (int32_t)i;
+}
+
+__global__ void k_row_nnz(const int32_t *rowidx, int64_t M, int32_t *nnz) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x)
+        nnz[i] = rowidx[i + 1] - rowidx[i];
+}
+
+// sort keys: ascending (maxkey - key) == descending key; value = row id (stable => ties by id)
+__global__ void k_sort_keys(const int32_t *nnz, int64_t M, int32_t nt, int use_wl, int32_t maxkey, uint64_t *keys,
+                            uint32_t *vals) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t k = use_wl ? (nnz[i] + nt - 1) / nt : nnz[i];
+        keys[i] = (uint64_t)(maxkey - k);
+        vals[i] = (uint32_t)i;
+    }
+}
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ULL;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+    return z ^ (z >> 31);
+}
+
+// MinHash pre-order key h_i = min_{b in blocks_i} splitmix64(b ^ seed); empty -> 2^64-1 (warp per row)
+__global__ void k_minhash(const int32_t *sig_ptr, const int32_t *sig, int64_t M, uint64_t seed, uint64_t *keys,
+                          uint32_t *vals) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M;
+         i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        uint64_t m = ~0ULL;
+        for (int32_t t = sig_ptr[i] + lane; t < sig_ptr[i + 1]; t += 32)
+            m = min(m, splitmix64((uint64_t)(uint32_t)sig[t] ^ seed));
+#pragma unroll
+        for (int o = 16; o; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) { keys[i] = m; vals[i] = (uint32_t)i; }
+    }
+}
+
+// ---- signatures: warp per row; distinct blocks are the positions where col/bw changes ---------
+__global__ void k_sig_count(const int32_t *rowidx, const int32_t *colidx, int64_t M, int32_t bw, int32_t *cnt) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M;
+         i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        int32_t a = rowidx[i], b = rowidx[i + 1], c = 0;
+        for (int32_t j = a + lane; j < b; j += 32)
+            c += (j == a) || (colidx[j] / bw != colidx[j - 1] / bw);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+        if (lane == 0) cnt[i] = c;
+    }
+}
+
+__global__ void k_sig_fill(const int32_t *rowidx, const int32_t *colidx, int64_t M, int32_t bw, const int32_t *ptr,
+                           int32_t *blk) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M;
+         i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        int32_t a = rowidx[i], b = rowidx[i + 1], w = ptr[i];
+        for (int32_t j0 = a; j0 < b; j0 += 32) {
+            int32_t j = j0 + lane;
+            bool f = j < b && ((j == a) || (colidx[j] / bw != colidx[j - 1] / bw));
+            unsigned m = __ballot_sync(0xffffffffu, f);
+            if (f) blk[w + __popc(m & ((1u << lane) - 1u))] = colidx[j] / bw;
+            w += __popc(m);
+        }
+    }
+}
+
+// ---- greedy chains --------------------------------------------------------------------------
+enum ChainMode { C_CTA = 0, C_H21 = 1, C_H22 = 2, C_H1 = 3, C_WARP = 4, C_H23 = 5 };
+constexpr int CHAIN_THREADS = 512;
+constexpr int CHAIN_MAX_PER_THREAD = 64;                 // placed flags in one u64 per thread
+constexpr int64_t CHAIN_MAX_N = (int64_t)CHAIN_THREADS * CHAIN_MAX_PER_THREAD;   // 32768
+
+struct Key {
+    uint32_t k1, k2, r, a;
+};
+__device__ __forceinline__ bool key_less(const Key &x, const Key &y) {
+    if (x.k1 != y.k1) return x.k1 < y.k1;
+    if (x.k2 != y.k2) return x.k2 < y.k2;
+    return x.r < y.r;
+}
+__device__ __forceinline__ Key shfl_key(const Key &k, int o) {
+    Key y;
+    y.k1 = __shfl_xor_sync(0xffffffffu, k.k1, o);
+    y.k2 = __shfl_xor_sync(0xffffffffu, k.k2, o);
+    y.r = __shfl_xor_sync(0xffffffffu, k.r, o);
+    y.a = __shfl_xor_sync(0xffffffffu, k.a, o);
+    return y;
+}
+
+// block-wide argmin; every thread returns the winner.  Uses red[] (CHAIN_THREADS/32 entries).
+__device__ __forceinline__ Key block_argmin(Key k, Key *red) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        Key y = shfl_key(k, o);
+        if (key_less(y, k)) k = y;
+    }
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = k;
+    __syncthreads();
+    Key b = red[0];
+#pragma unroll
+    for (int w = 1; w < CHAIN_THREADS / 32; ++w)
+        if (key_less(red[w], b)) b = red[w];
+    return b;
+}
+
+__device__ __forceinline__ void bitmap_set(uint32_t *bm, const int32_t *sig, int32_t s0, int32_t s1) {
+    for (int32_t t = s0 + threadIdx.x; t < s1; t += CHAIN_THREADS) {
+        uint32_t b = (uint32_t)sig[t];
+        atomicOr(&bm[b >> 5], 1u << (b & 31));
+    }
+}
+__device__ __forceinline__ void bitmap_clear(uint32_t *bm, const int32_t *sig, int32_t s0, int32_t s1) {
+    for (int32_t t = s0 + threadIdx.x; t < s1; t += CHAIN_THREADS) bm[(uint32_t)sig[t] >> 5] = 0u;
+}
+__device__ __forceinline__ uint32_t intersect(const uint32_t *bm, const int32_t *sig, int32_t s0, int32_t s1) {
+    uint32_t c = 0;
+    for (int32_t t = s0; t < s1; ++t) {
+        uint32_t b = (uint32_t)__ldg(sig + t);
+        c += (bm[b >> 5] >> (b & 31)) & 1u;
+    }
+    return c;
+}
+
+// One CTA per segment.  base: row ids in pre-order; segment s = base[seg[s] .. seg[s+1]) (or fixed
+// windows of W when seg == nullptr).  Writes perm[seg[s] + q] for q = 0..n-1.
+// Per step: (1) set the reference row's blocks in a bitmap, barrier; (2) every thread scores its
+// unplaced candidates (Hamming = |ref| + |r| - 2|ref ∩ r|), block argmin (one more barrier);
+// (3) clear the bitmap.  Bitmaps and the reduction buffer are double-buffered so two barriers per
+// step suffice: a buffer written at step q is next written at step q+2.
+template <int MODE>
+__global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const int32_t *base, const int32_t *seg, int64_t W, int64_t M,
+                                                         const int32_t *sig_ptr, const int32_t *sig,
+                                                         const int32_t *nnz, int32_t nt, int32_t nw, int64_t words,
+                                                         uint32_t *gscratch, int32_t *perm) {
+    extern __shared__ uint32_t smem_bm[];
+    __shared__ Key red[2][CHAIN_THREADS / 32];
+    constexpr int REFS = (MODE == C_H22) ? 2 : 1;   // bitmaps per step
+    uint32_t *bm = gscratch ? gscratch + (size_t)blockIdx.x * 2 * REFS * words : smem_bm;
+    const int64_t s0 = seg ? seg[blockIdx.x] : (int64_t)blockIdx.x * W;
+    const int64_t s1 = seg ? seg[blockIdx.x + 1] : min(s0 + W, M);
+    const int n = (int)(s1 - s0);
+    const int32_t *om = base + s0;
+    int32_t *out = perm + s0;
+    for (int64_t t = threadIdx.x; t < 2 * REFS * words; t += CHAIN_THREADS) bm[t] = 0u;
+    uint64_t placed = 0;   // bit k: candidate a = threadIdx.x + k*CHAIN_THREADS is placed
+    __syncthreads();
+
+    auto wl_of = [&](int32_t r) -> uint32_t { return (uint32_t)((nnz[r] + nt - 1) / nt); };
+    int32_t prev = -1;
+    int q = 0;
+    int nfirst;
+    if (MODE == C_H1) {               // Hybrid-1: the segment's first (Plain-Sort) row stays first
+        nfirst = 0;
+        if (n > 0) {
+            if (threadIdx.x == 0) { placed |= 1ULL; out[0] = om[0]; }
+            prev = om[0];
+            q = 1;
+        }
+    } else {                          // lowest (wl, id) first: 1 row (CTA-aware), nw rows (Warp-aware)
+        nfirst = (MODE == C_WARP || MODE == C_H23) ? min(n, nw) : min(n, 1);
+    }
+    for (; q < n; ++q) {
+        const int buf = q & 1;
+        const bool first = q < nfirst;
+        uint32_t *bmA = bm + (size_t)(buf * REFS) * words;
+        uint32_t *bmB = bmA + words;   // H22 only
+        int32_t refA = -1, refB = -1;
+        if (!first) {
+            if (MODE == C_WARP || MODE == C_H23) refA = nw == 1 ? prev : out[q - nw];
+            else refA = prev;
+            if (MODE == C_H22 && q >= nw) refB = nw == 1 ? prev : out[q - nw];
+        }
+        int32_t aS = 0, aE = 0, bS = 0, bE = 0;
+        if (refA >= 0) { aS = sig_ptr[refA]; aE = sig_ptr[refA + 1]; bitmap_set(bmA, sig, aS, aE); }
+        if (refB >= 0) { bS = sig_ptr[refB]; bE = sig_ptr[refB + 1]; bitmap_set(bmB, sig, bS, bE); }
+        const uint32_t cntA = (uint32_t)(aE - aS), cntB = (uint32_t)(bE - bS);
+        const uint32_t wl_prev = ((MODE == C_H21 || MODE == C_H23) && !first) ? wl_of(prev) : 0u;
+        __syncthreads();
+        Key best{0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+        for (int k = 0; k < CHAIN_MAX_PER_THREAD; ++k) {
+            const int a = threadIdx.x + k * CHAIN_THREADS;
+            if (a >= n) break;
+            if ((placed >> k) & 1ULL) continue;
+            const int32_t r = om[a];
+            Key c{0u, 0u, (uint32_t)r, (uint32_t)a};
+            if (first) {
+                c.k1 = wl_of(r);
+            } else {
+                const int32_t rs = sig_ptr[r], re = sig_ptr[r + 1];
+                const uint32_t cr = (uint32_t)(re - rs);
+                c.k1 = cntA + cr - 2u * intersect(bmA, sig, rs, re);
+                if (MODE == C_H21 || MODE == C_H23) {
+                    const uint32_t w = wl_of(r);
+                    c.k2 = w > wl_prev ? w - wl_prev : wl_prev - w;
+                } else if (MODE == C_H22) {
+                    c.k2 = refB >= 0 ? cntB + cr - 2u * intersect(bmB, sig, rs, re) : 0u;
+                }
+            }
+            if (key_less(c, best)) best = c;
+        }
+        const Key w = block_argmin(best, red[buf]);
+        if ((int)(w.a % CHAIN_THREADS) == (int)threadIdx.x) placed |= 1ULL << (w.a / CHAIN_THREADS);
+        if (threadIdx.x == 0) out[q] = (int32_t)w.r;
+        if (refA >= 0) bitmap_clear(bmA, sig, aS, aE);
+        if (refB >= 0) bitmap_clear(bmB, sig, bS, bE);
+        prev = (int32_t)w.r;
+    }
+}
+
+// HYBRID_1 segments: p starts a segment if it starts a run of equal sorted key or is W positions
+// into its run.  keys: ascending sorted (maxwl - wl).
+__global__ void k_h1_flags(const uint64_t *keys, int64_t M, int64_t W, int32_t *flag) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        // run start = lower_bound(keys, keys[p])
+        int64_t lo = 0, hi = p;
+        uint64_t k = keys[p];
+        while (lo < hi) {
+            int64_t mid = (lo + hi) >> 1;
+            if (keys[mid] < k) lo = mid + 1; else hi = mid;
+        }
+        flag[p] = ((p - lo) % W) == 0;
+    }
+}
+
+__global__ void k_compact_starts(const int32_t *flag, const int32_t *pos, int64_t M, int32_t *starts) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x)
+        if (flag[p]) starts[pos[p]] = (int32_t)p;
+}
+
+__global__ void k_set_last(int32_t *a, int64_t idx, int32_t v) { a[idx] = v; }
+
+// FLIPPED: odd nw-chunks of the Plain-Sort order reversed (a partial last chunk within its length)
+__global__ void k_flip(const uint32_t *s, int64_t M, int32_t nw, int32_t *perm) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = p / nw, lo = c * nw, hi = min(lo + nw, M);
+        perm[p] = (int32_t)((c & 1) ? s[lo + (hi - 1 - p)] : s[p]);
+    }
+}
+
+// LPT (capacity-constrained, reading A5): one warp; lane w holds warp w's load / count / capacity.
+__global__ void k_lpt(const uint32_t *s, const int32_t *nnz, int64_t M, int32_t nt, int32_t nw, int32_t *perm) {
+    const int lane = threadIdx.x;
+    int64_t load = 0, cnt = 0;
+    const int64_t cap = (lane < nw && M > lane) ? (M - lane + nw - 1) / nw : 0;
+    for (int64_t t0 = 0; t0 < M; t0 += 32) {
+        int64_t t = t0 + lane;
+        uint32_t r_mine = t < M ? s[t] : 0u;
+        int32_t wl_mine = t < M ? (nnz[r_mine] + nt - 1) / nt : 0;
+        int lim = (int)(M - t0 < 32 ? M - t0 : 32);
+        for (int u = 0; u < lim; ++u) {
+            uint32_t r = __shfl_sync(0xffffffffu, r_mine, u);
+            int32_t wl = __shfl_sync(0xffffffffu, wl_mine, u);
+            // argmin over non-full warps of (load, w)
+            int64_t key_load = (lane < nw && cnt < cap) ? load : INT64_MAX;
+            int key_w = lane;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                int64_t ol = __shfl_xor_sync(0xffffffffu, key_load, o);
+                int ow = __shfl_xor_sync(0xffffffffu, key_w, o);
+                if (ol < key_load || (ol == key_load && ow < key_w)) { key_load = ol; key_w = ow; }
+            }
+            if (lane == key_w) {
+                perm[cnt * nw + lane] = (int32_t)r;
+                load += wl;
+                ++cnt;
+            }
+        }
+    }
+}
+
+__global__ void k_dcsr_flags(const int32_t *nnz, int64_t M, int32_t *flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = nnz[i] > 0;
+}
+__global__ void k_dcsr_scatter(const int32_t *flag, const int32_t *pos, int64_t M, int32_t n_nonempty, int32_t *perm) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x)
+        perm[flag[i] ? pos[i] : n_nonempty + ((int32_t)i - pos[i])] = (int32_t)i;
+}
+
+__global__ void k_u32_to_i32(const uint32_t *a, int64_t n, int32_t *b) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        b[i] = (int32_t)a[i];
+}
+
+// ---- permuted CSR ---------------------------------------------------------------------------
+__global__ void k_perm_len(const int32_t *rowidx, const int32_t *perm, int64_t M, int32_t *len) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        int32_t i = perm[p];
+        len[p] = rowidx[i + 1] - rowidx[i];
+    }
+}
+
+// warp per position: copy the row's (col, val) pairs into the interleaved permuted array
+__global__ void k_gather(const int32_t *rowidx, const int32_t *colidx, const float *value, const int32_t *perm,
+                         const int32_t *rowptr_p, int64_t M, int2 *cv) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < M;
+         p += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        int32_t i = perm[p];
+        int32_t a = rowidx[i], len = rowidx[i + 1] - a, d = rowptr_p[p];
+        for (int32_t t = lane; t < len; t += 32)
+            cv[d + t] = make_int2(colidx[a + t], __float_as_int(value[a + t]));
+    }
+}
+
+__global__ void k_long_flags(const int32_t *rowptr_p, int64_t M, int32_t split, int32_t *flag, int32_t *nch) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        int32_t len = rowptr_p[p + 1] - rowptr_p[p];
+        bool lg = len > split;
+        flag[p] = lg;
+        nch[p] = lg ? (len + split - 1) / split : 0;
+    }
+}
+
+// per long row (warp): record its position and write its chunk table
+__global__ void k_long_fill(const int32_t *rowptr_p, const int32_t *flag, const int32_t *lpos, const int32_t *choff,
+                            int64_t M, int32_t split, int32_t *long_pos, int32_t *long_chunk_ptr, int32_t *cstart,
+                            int32_t *clen) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < M;
+         p += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        if (!flag[p]) continue;
+        int32_t l = lpos[p], c0 = choff[p], a = rowptr_p[p], len = rowptr_p[p + 1] - a;
+        int32_t nc = (len + split - 1) / split;
+        if (lane == 0) { long_pos[l] = (int32_t)p; long_chunk_ptr[l] = c0; }
+        for (int32_t c = lane; c < nc; c += 32) {
+            cstart[c0 + c] = a + c * split;
+            clen[c0 + c] = min(split, len - c * split);
+        }
+    }
+}
+
+inline unsigned grid_for(int64_t n, int threads) {
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, threads), 148 * 32));
+}
+inline unsigned grid_warps(int64_t n, int threads) {
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n * 32, threads), 148 * 64));
+}
+
+spmm_status launch_chain(int mode, const int32_t *base, const int32_t *seg, int64_t nseg, int64_t W, int64_t M,
+                         const Signatures &sig, const int32_t *nnz, const spmm_params &p, int64_t N, int32_t *perm,
+                         cudaStream_t s) {
+    if (nseg == 0) return SPMM_OK;
+    const int64_t nblk = ceil_div(N, p.bw);
+    const int64_t words = std::max<int64_t>(1, ceil_div(nblk, 32));
+    const int nbuf = mode == C_H22 ? 4 : 2;   // 2 buffers x refs
+    size_t smem = (size_t)nbuf * words * sizeof(uint32_t);
+    DevBuf gs;
+    uint32_t *gscratch = nullptr;
+    if (smem > 200 * 1024) {   // large N: per-CTA bitmaps in global memory (L2-resident)
+        SPMM_TRY(gs.alloc((size_t)nseg * nbuf * words * sizeof(uint32_t), s));
+        gscratch = gs.as<uint32_t>();
+        smem = 0;
+    }
+    auto go = [&](auto kern) -> spmm_status {
+        if (smem > 48 * 1024) SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        kern<<<(unsigned)nseg, CHAIN_THREADS, smem, s>>>(base, seg, W, M, sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(),
+                                                        nnz, p.nt, p.nw, words, gscratch, perm);
+        SPMM_CUDA(cudaGetLastError());
+        return SPMM_OK;
+    };
+    switch (mode) {
+        case C_CTA: return go(k_chain<C_CTA>);
+        case C_H21: return go(k_chain<C_H21>);
+        case C_H22: return go(k_chain<C_H22>);
+        case C_H1: return go(k_chain<C_H1>);
+        case C_WARP: return go(k_chain<C_WARP>);
+        default: return go(k_chain<C_H23>);
+    }
+}
+
+// plain sort (by nnz or by warp load), result row ids in vals (uint32[M]); keys kept for H1
+spmm_status sort_rows(const int32_t *nnz, int64_t M, int32_t nt, bool by_wl, int32_t max_nnz, DevBuf &keys, DevBuf &vals,
+                      cudaStream_t s) {
+    SPMM_TRY(keys.alloc(std::max<int64_t>(M, 1) * sizeof(uint64_t), s));
+    SPMM_TRY(vals.alloc(std::max<int64_t>(M, 1) * sizeof(uint32_t), s));
+    int32_t maxkey = by_wl ? (max_nnz + nt - 1) / nt : max_nnz;
+    if (M == 0) return SPMM_OK;
+    k_sort_keys<<<grid_for(M, 256), 256, 0, s>>>(nnz, M, nt, by_wl ? 1 : 0, maxkey, keys.as<uint64_t>(), vals.as<uint32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    int bits = 0;
+    while (bits < 32 && ((uint64_t)maxkey >> bits) != 0) ++bits;
+    return radix_sort_pairs(keys.as<uint64_t>(), vals.as<uint32_t>(), M, 0, bits, s);
+}
+
+}  // namespace
+
+spmm_status build_signatures(const int32_t *rowidx, const int32_t *colidx, const int32_t * /*order*/, int64_t M,
+                             int64_t nnz, int32_t bw, Signatures &sig, cudaStream_t s) {
+    DevBuf cnt;
+    SPMM_TRY(cnt.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
+    SPMM_TRY(sig.ptr.alloc((M + 1) * sizeof(int32_t), s));
+    if (M > 0) {
+        k_sig_count<<<grid_warps(M, 256), 256, 0, s>>>(rowidx, colidx, M, bw, cnt.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    int32_t total = 0;
+    SPMM_TRY(exclusive_scan_i32(cnt.as<int32_t>(), sig.ptr.as<int32_t>(), M, &total, s));
+    sig.S = total;
+    SPMM_TRY(sig.blk.alloc(std::max<int64_t>(total, 1) * sizeof(int32_t), s));
+    if (M > 0 && nnz > 0) {
+        k_sig_fill<<<grid_warps(M, 256), 256, 0, s>>>(rowidx, colidx, M, bw, sig.ptr.as<int32_t>(), sig.blk.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    return SPMM_OK;
+}
+
+spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, cudaStream_t s) {
+    const int64_t M = h->M;
+    SPMM_TRY(h->perm.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
+    int32_t *perm = h->perm.as<int32_t>();
+    if (M == 0) return SPMM_OK;
+    DevBuf nnzb;
+    SPMM_TRY(nnzb.alloc(M * sizeof(int32_t), s));
+    int32_t *nnz = nnzb.as<int32_t>();
+    k_row_nnz<<<grid_for(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), M, nnz);
+    SPMM_CUDA(cudaGetLastError());
+
+    switch (policy) {
+    case SPMM_POLICY_IDENTITY:
+        k_iota<<<grid_for(M, 256), 256, 0, s>>>(perm, M);
+        SPMM_CUDA(cudaGetLastError());
+        return SPMM_OK;
+    case SPMM_POLICY_NNZ_SORT:
+    case SPMM_POLICY_PLAIN_SORT:
+    case SPMM_POLICY_FLIPPED:
+    case SPMM_POLICY_LPT: {
+        DevBuf keys, vals;
+        SPMM_TRY(sort_rows(nnz, M, p.nt, policy != SPMM_POLICY_NNZ_SORT, h->max_row_nnz, keys, vals, s));
+        if (policy == SPMM_POLICY_FLIPPED) {
+            k_flip<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, p.nw, perm);
+        } else if (policy == SPMM_POLICY_LPT) {
+            if (p.nw > 32) return fail(SPMM_ERR_UNSUPPORTED, "LPT: nw > 32");
+            k_lpt<<<1, 32, 0, s>>>(vals.as<uint32_t>(), nnz, M, p.nt, p.nw, perm);
+        } else {
+            k_u32_to_i32<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, perm);
+        }
+        SPMM_CUDA(cudaGetLastError());
+        return SPMM_OK;
+    }
+    case SPMM_POLICY_DCSR: {
+        DevBuf flag, pos;
+        SPMM_TRY(flag.alloc(M * sizeof(int32_t), s));
+        SPMM_TRY(pos.alloc((M + 1) * sizeof(int32_t), s));
+        k_dcsr_flags<<<grid_for(M, 256), 256, 0, s>>>(nnz, M, flag.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        int32_t ne = 0;
+        SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), pos.as<int32_t>(), M, &ne, s));
+        k_dcsr_scatter<<<grid_for(M, 256), 256, 0, s>>>(flag.as<int32_t>(), pos.as<int32_t>(), M, ne, perm);
+        SPMM_CUDA(cudaGetLastError());
+        return SPMM_OK;
+    }
+    case SPMM_POLICY_HYBRID_1: {
+        const int64_t W = (p.window == 0 || p.window > M) ? M : p.window;
+        DevBuf keys, vals, flag, pos, starts, base;
+        SPMM_TRY(sort_rows(nnz, M, p.nt, true, h->max_row_nnz, keys, vals, s));
+        SPMM_TRY(flag.alloc(M * sizeof(int32_t), s));
+        SPMM_TRY(pos.alloc((M + 1) * sizeof(int32_t), s));
+        k_h1_flags<<<grid_for(M, 256), 256, 0, s>>>(keys.as<uint64_t>(), M, W, flag.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        int32_t nseg = 0;
+        SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), pos.as<int32_t>(), M, &nseg, s));
+        SPMM_TRY(starts.alloc((nseg + 1) * sizeof(int32_t), s));
+        k_compact_starts<<<grid_for(M, 256), 256, 0, s>>>(flag.as<int32_t>(), pos.as<int32_t>(), M, starts.as<int32_t>());
+        k_set_last<<<1, 1, 0, s>>>(starts.as<int32_t>(), nseg, (int32_t)M);
+        SPMM_CUDA(cudaGetLastError());
+        if (W > CHAIN_MAX_N) return fail(SPMM_ERR_UNSUPPORTED, "HYBRID_1: segment window above 32768 rows");
+        SPMM_TRY(base.alloc(M * sizeof(int32_t), s));
+        k_u32_to_i32<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, base.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        Signatures sig;
+        SPMM_TRY(build_signatures(h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), nullptr, M, h->nnz, p.bw, sig, s));
+        return launch_chain(C_H1, base.as<int32_t>(), starts.as<int32_t>(), nseg, 0, M, sig, nnz, p, h->N, perm, s);
+    }
+    default: {   // chain policies over windows of a pre-order
+        const int64_t W = (p.window == 0 || p.window > M) ? M : p.window;
+        if (W > CHAIN_MAX_N)
+            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows (use window > 0)");
+        int mode = policy == SPMM_POLICY_CTA_AWARE ? C_CTA : policy == SPMM_POLICY_HYBRID_2_1 ? C_H21 :
+                   policy == SPMM_POLICY_HYBRID_2_2 ? C_H22 : policy == SPMM_POLICY_WARP_AWARE ? C_WARP : C_H23;
+        Signatures sig;
+        SPMM_TRY(build_signatures(h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), nullptr, M, h->nnz, p.bw, sig, s));
+        DevBuf base;
+        SPMM_TRY(base.alloc(M * sizeof(int32_t), s));
+        if (p.preorder) {
+            DevBuf keys, vals;
+            SPMM_TRY(keys.alloc(M * sizeof(uint64_t), s));
+            SPMM_TRY(vals.alloc(M * sizeof(uint32_t), s));
+            k_minhash<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M, p.seed,
+                                                        keys.as<uint64_t>(), vals.as<uint32_t>());
+            SPMM_CUDA(cudaGetLastError());
+            SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), vals.as<uint32_t>(), M, 0, 64, s));
+            k_u32_to_i32<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, base.as<int32_t>());
+        } else {
+            k_iota<<<grid_for(M, 256), 256, 0, s>>>(base.as<int32_t>(), M);
+        }
+        SPMM_CUDA(cudaGetLastError());
+        return launch_chain(mode, base.as<int32_t>(), nullptr, ceil_div(M, W), W, M, sig, nnz, p, h->N, perm, s);
+    }
+    }
+}
+
+spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s) {
+    const int64_t M = h->M;
+    const int32_t split = h->params.split_nnz;
+    SPMM_TRY(h->rowptr_p.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(h->cv_p.alloc(std::max<int64_t>(h->nnz, 1) * sizeof(int2), s));
+    DevBuf len;
+    SPMM_TRY(len.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
+    if (M > 0) {
+        k_perm_len<<<grid_for(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), h->perm.as<int32_t>(), M, len.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    SPMM_TRY(exclusive_scan_i32(len.as<int32_t>(), h->rowptr_p.as<int32_t>(), M, nullptr, s));
+    if (M > 0 && h->nnz > 0) {
+        k_gather<<<grid_warps(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), h->value.as<float>(),
+                                                   h->perm.as<int32_t>(), h->rowptr_p.as<int32_t>(), M, h->cv_p.as<int2>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    // long rows and their chunk table
+    LongRows &lr = h->lr;
+    lr.n_long = lr.n_chunks = 0;
+    if (M == 0 || h->max_row_nnz <= split) {
+        lr.chunk_start.release(); lr.chunk_len.release(); lr.long_pos.release(); lr.long_chunk_ptr.release();
+        return SPMM_OK;
+    }
+    DevBuf flag, nch, lpos, choff;
+    SPMM_TRY(flag.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(nch.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(lpos.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(choff.alloc((M + 1) * sizeof(int32_t), s));
+    k_long_flags<<<grid_for(M, 256), 256, 0, s>>>(h->rowptr_p.as<int32_t>(), M, split, flag.as<int32_t>(), nch.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    int32_t nlong = 0, nchunks = 0;
+    SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), lpos.as<int32_t>(), M, &nlong, s));
+    SPMM_TRY(exclusive_scan_i32(nch.as<int32_t>(), choff.as<int32_t>(), M, &nchunks, s));
+    lr.n_long = nlong;
+    lr.n_chunks = nchunks;
+    SPMM_TRY(lr.long_pos.alloc(std::max(nlong, 1) * sizeof(int32_t), s));
+    SPMM_TRY(lr.long_chunk_ptr.alloc((nlong + 1) * sizeof(int32_t), s));
+    SPMM_TRY(lr.chunk_start.alloc(std::max(nchunks, 1) * sizeof(int32_t), s));
+    SPMM_TRY(lr.chunk_len.alloc(std::max(nchunks, 1) * sizeof(int32_t), s));
+    k_long_fill<<<grid_warps(M, 256), 256, 0, s>>>(h->rowptr_p.as<int32_t>(), flag.as<int32_t>(), lpos.as<int32_t>(),
+                                                  choff.as<int32_t>(), M, split, lr.long_pos.as<int32_t>(),
+                                                  lr.long_chunk_ptr.as<int32_t>(), lr.chunk_start.as<int32_t>(),
+                                                  lr.chunk_len.as<int32_t>());
+    k_set_last<<<1, 1, 0, s>>>(lr.long_chunk_ptr.as<int32_t>(), nlong, nchunks);
+    SPMM_CUDA(cudaGetLastError());
+    return SPMM_OK;
+}
+
+}  // namespace spmm

@@ -1,0 +1,83 @@
+"""C-ABI checks that need no GPU: the library loads, exports every function include/spmm.h declares, and
+its host-only entry points (partition, predictor inference, status strings) agree with the oracle."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import synthetic as syn
+import paper_conf_ispass_mehrabilcslo21_b200 as pkg
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_functions():
+    txt = open(os.path.join(ROOT, "include", "spmm.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(spmm_[a-z_0-9]+)\s*\(", txt)))
+
+
+def test_exports_every_declared_symbol():
+    lib = pkg.load_library()
+    names = header_functions()
+    assert len(names) >= 15
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(names) == set(pkg.EXPORTS)
+
+
+def test_built_for_sm100a():
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", pkg.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_status_strings():
+    lib = pkg.load_library()
+    for code, name in pkg.STATUS.items():
+        assert lib.spmm_status_string(code).decode() == name
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+def test_partition_matches_oracle(P):
+    a = syn.rmat(11, 8, 7, "natural")
+    assert np.array_equal(pkg.spmm_partition_by_nnz(a.rowidx, P), oracle.partition_by_nnz(a.rowidx, P))
+
+
+def test_partition_invalid():
+    with pytest.raises(pkg.SpmmError) as e:
+        pkg.spmm_partition_by_nnz(np.array([0, 1]), 0)
+    assert e.value.status == 1
+
+
+@pytest.mark.parametrize("P", [4, 6])
+def test_predict_matches_oracle(P):
+    rng = np.random.default_rng(P)
+    n = 48 + 64 * 24 + 64 + 32 * 64 + 32 + 33 * P
+    w = (rng.standard_normal(n) * 0.3).astype(np.float32)
+    w[24:48] = np.abs(w[24:48]) + 0.5
+    for t in range(5):
+        f = np.abs(rng.standard_normal(24)) * 10 ** rng.integers(0, 6)
+        pol, times = pkg.spmm_predict(f, w, P)
+        best, ref = oracle.mlp_forward(f, w, P)
+        assert pol == best
+        np.testing.assert_allclose(times, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_predict_rejects_bad_layout():
+    with pytest.raises(pkg.SpmmError):
+        pkg.spmm_predict(np.zeros(24), np.zeros(10, np.float32), 4)
+
+
+def test_no_cpu_fallback_in_product():
+    """The product package must not import the oracle (or any CPU fallback)."""
+    pdir = os.path.join(ROOT, "paper_conf_ispass_mehrabilcslo21_b200")
+    for dp, _, fs in os.walk(pdir):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                src = open(os.path.join(dp, f)).read()
+                for bad in ("import oracle", "from oracle", "liboracle", '#include "../../oracle', "oracle/"):
+                    assert bad not in src, (f, bad)

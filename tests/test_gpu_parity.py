@@ -1,0 +1,275 @@
+"""GPU parity: the CUDA path through the C-ABI vs the CPU oracle on the same seeded inputs (-m gpu).
+
+Bars (BASELINE.json north star): permutation arrays, permuted CSR and the 24 features bit-exact;
+C within |C_gpu - C_ref| <= 1e-5 * sum_j |a_ij||b_jk| + 1e-6; integer-valued inputs exact; C
+bit-identical across all permutation policies (C depends only on each row's nnz order).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synthetic as syn
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
+
+ALL_POLICIES = list(pkg.POLICIES)
+
+
+def within_tol(C_gpu, C_ref, bound):
+    err = np.abs(C_gpu.astype(np.float64) - C_ref)
+    ok = err <= 1e-5 * bound + 1e-6
+    return bool(ok.all()), float((err / (1e-5 * bound + 1e-6)).max()) if err.size else 0.0
+
+
+def run_c(h, B, K=None):
+    Bd = torch.from_numpy(np.ascontiguousarray(B)).cuda()
+    C = h.run(Bd)
+    torch.cuda.synchronize()
+    return C.cpu().numpy()
+
+
+GENS = {
+    "rmat12_natural": lambda: syn.rmat(12, 12, 1000, "natural"),
+    "rmat12_randlabel": lambda: syn.rmat(12, 12, 1001, "random-label"),
+    "rmat13_local": lambda: syn.rmat(13, 10, 1002, "local"),
+    "stencil16": lambda: syn.stencil27(16, 1003),
+    "uniform": lambda: syn.uniform(5000, 7000, 9, 1004, poisson=True),
+    "block": lambda: syn.blockcluster(4099, 9000, 32, 4, 20, 1005),
+}
+
+
+@pytest.fixture(scope="module")
+def mats():
+    return {k: g() for k, g in GENS.items()}
+
+
+@pytest.mark.parametrize("gen", list(GENS))
+@pytest.mark.parametrize("policy", ALL_POLICIES)
+def test_perm_and_permuted_csr_bit_exact(mats, gen, policy):
+    a = mats[gen]
+    for window in (0, 64, 1024):
+        h = pkg.SpMM.from_csr(a)
+        h.permute(policy, window=window)
+        perm = h.perm()
+        ref = oracle.permute(a, policy, window=window)
+        assert np.array_equal(perm, ref), (gen, policy, window, int(np.argmax(perm != ref)))
+        r2, c2, v2 = h.permuted_csr()
+        rr, cr, vr = oracle.permuted_csr(a, ref)
+        assert np.array_equal(r2, rr) and np.array_equal(c2, cr) and np.array_equal(v2.view(np.int32), vr.view(np.int32))
+        h.close()
+
+
+@pytest.mark.parametrize("params", [dict(nw=8, nt=8, bw=8, window=64), dict(nw=4, nt=16, bw=64, window=0),
+                                    dict(nw=32, nt=32, bw=16, window=96)])
+@pytest.mark.parametrize("policy", ALL_POLICIES)
+def test_perm_params(mats, params, policy):
+    a = mats["rmat12_natural"]
+    h = pkg.SpMM.from_csr(a)
+    h.permute(policy, **params)
+    assert np.array_equal(h.perm(), oracle.permute(a, policy, **params)), (policy, params)
+    h.close()
+
+
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_2_2", "warp_aware", "hybrid_2_3"])
+def test_minhash_preorder(mats, policy):
+    a = mats["block"]
+    h = pkg.SpMM.from_csr(a)
+    h.permute(policy, window=256, preorder=1, seed=12345)
+    assert np.array_equal(h.perm(), oracle.permute(a, policy, window=256, preorder=1, seed=12345))
+    h.close()
+
+
+@pytest.mark.parametrize("gen", list(GENS))
+@pytest.mark.parametrize("K", [32, 64, 128])
+def test_spmm_tolerance_all_policies(mats, gen, K):
+    a = mats[gen]
+    B = syn.dense(a.N, K, 77)
+    C_ref, bound = oracle.spmm(a, B)
+    h = pkg.SpMM.from_csr(a)
+    first = None
+    for pol in ALL_POLICIES:
+        h.permute(pol, window=1024 if pol != "hybrid_1" else 256)
+        C = run_c(h, B)
+        ok, worst = within_tol(C, C_ref, bound)
+        assert ok, (gen, K, pol, worst)
+        if first is None:
+            first = C
+        else:   # permutation invariance: bit-identical C
+            assert np.array_equal(C.view(np.int32), first.view(np.int32)), (gen, K, pol)
+    h.close()
+
+
+@pytest.mark.parametrize("K", [4, 8, 12, 16, 20, 36, 48, 96, 192, 256, 260, 512, 516, 1024])
+def test_spmm_K_sweep_integer_exact(K):
+    a = syn.rmat(11, 10, 31, "random-label", int_values=True)
+    B = syn.dense(a.N, K, 32, int_values=True)
+    C_ref, _ = oracle.spmm(a, B)
+    h = pkg.SpMM.from_csr(a)
+    for pol in ("identity", "nnz_sort", "cta_aware"):
+        h.permute(pol)
+        assert np.array_equal(run_c(h, B).astype(np.float64), C_ref), (K, pol)
+    h.close()
+
+
+@pytest.mark.parametrize("split", [1, 7, 32, 128, 1000])
+def test_split_rows_exact_and_tolerance(split):
+    # one huge row (> 1e6 nnz) plus a power-law body: the split path + pairwise combine
+    body = syn.rmat(12, 8, 41, "natural", int_values=True)
+    N = 1 << 21
+    big = list(range(0, N, 2))[:1_048_600]
+    rows = [body.colidx[body.rowidx[i]:body.rowidx[i + 1]].tolist() for i in range(body.M)]
+    rows.insert(17, big)
+    vals = [np.asarray(body.value[body.rowidx[i]:body.rowidx[i + 1]]).tolist() for i in range(body.M)]
+    vals.insert(17, [1.0 if (t % 3) else -2.0 for t in range(len(big))])
+    a = syn.from_lists(body.M + 1, N, rows, vals)
+    B = syn.dense(N, 16, 42, int_values=True)
+    C_ref, _ = oracle.spmm(a, B)
+    h = pkg.SpMM.from_csr(a)
+    for pol in ("identity", "nnz_sort", "hybrid_2_1"):
+        h.permute(pol, split_nnz=split)
+        info = h.info()
+        assert info["split_rows"] >= 1 and info["max_row_nnz"] == len(big)
+        assert np.array_equal(run_c(h, B).astype(np.float64), C_ref), (split, pol)
+    # real-valued: tolerance
+    Bf = syn.dense(N, 16, 43)
+    af = syn.CSR(a.M, a.N, a.rowidx, a.colidx, syn.dense(1, a.nnz, 44)[0])
+    C_ref, bound = oracle.spmm(af, Bf)
+    hf = pkg.SpMM.from_csr(af)
+    hf.permute("nnz_sort", split_nnz=split)
+    ok, worst = within_tol(run_c(hf, Bf), C_ref, bound)
+    assert ok, (split, worst)
+    h.close()
+    hf.close()
+
+
+@pytest.mark.parametrize("gen", list(GENS))
+@pytest.mark.parametrize("params", [dict(), dict(nw=8, nt=4, bw=8), dict(nw=3, nt=32, bw=64)])
+def test_features_bit_exact(mats, gen, params):
+    a = mats[gen]
+    h = pkg.SpMM.from_csr(a)
+    np.testing.assert_array_equal(h.features(**params), oracle.features(a, **params))
+    for pol in ("nnz_sort", "cta_aware"):
+        h.permute(pol)
+        np.testing.assert_array_equal(h.features(current_order=True, **params),
+                                      oracle.features(a, oracle.permute(a, pol), **params))
+    h.close()
+
+
+def test_e1_worked_example(e1):
+    a = syn.from_lists(e1["M"], e1["N"], e1["rows"])
+    h = pkg.SpMM.from_csr(a)
+    np.testing.assert_array_equal(h.features(nw=2, nt=2, bw=2), np.array(e1["features_identity"]))
+    for name, spec in e1["perm"].items():
+        h.permute(spec.get("policy", name), nw=2, nt=2, bw=2, window=spec["window"])
+        assert h.perm().tolist() == spec["perm"], name
+    K = e1["spmm"]["K"]
+    B = np.array([[j + 1 + 10 * k for k in range(K)] for j in range(e1["N"])], dtype=np.float32)
+    B4 = np.zeros((e1["N"], 4), np.float32)
+    B4[:, :K] = B
+    assert run_c(h, B4)[:, :K].tolist() == e1["spmm"]["C"]
+    h.close()
+
+
+def test_edge_cases():
+    # M = 0
+    z = syn.from_lists(0, 10, [])
+    h = pkg.SpMM.from_csr(z)
+    h.permute("cta_aware")
+    assert run_c(h, syn.dense(10, 8, 1)).shape == (0, 8)
+    h.close()
+    # nnz = 0: C zero-filled
+    e = syn.from_lists(5, 10, [[]] * 5)
+    h = pkg.SpMM.from_csr(e)
+    Bd = torch.from_numpy(syn.dense(10, 8, 1)).cuda()
+    C = torch.full((5, 8), 7.0, device="cuda")
+    h.run(Bd, C)
+    torch.cuda.synchronize()
+    assert torch.all(C == 0)
+    np.testing.assert_array_equal(h.features(), oracle.features(e))
+    h.close()
+    # empty rows interleaved, M not a multiple of nw, N not a multiple of bw
+    a = syn.from_lists(37, 45, [[] if i % 3 == 0 else [i % 45, (i * 7 + 1) % 45][: 1 + i % 2] for i in range(37)])
+    a.colidx = np.concatenate([np.sort(a.colidx[a.rowidx[i]:a.rowidx[i + 1]]) for i in range(37)]).astype(np.int32)
+    B = syn.dense(45, 12, 3, int_values=True)
+    C_ref, _ = oracle.spmm(a, B)
+    h = pkg.SpMM.from_csr(a)
+    for pol in ALL_POLICIES:
+        h.permute(pol, window=0)
+        assert np.array_equal(h.perm(), oracle.permute(a, pol, window=0)), pol
+        assert np.array_equal(run_c(h, B).astype(np.float64), C_ref), pol
+    h.close()
+
+
+def test_errors():
+    a = syn.rmat(8, 4, 5)
+    h = pkg.SpMM.from_csr(a)
+    Bd = torch.from_numpy(syn.dense(a.N, 10, 1)).cuda()
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.run(Bd)                                   # K % 4 != 0
+    assert ex.value.status == 3
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.run(torch.zeros(a.N, 1028, device="cuda"))   # K > 1024
+    assert ex.value.status == 3
+    Bm = torch.zeros(a.N * 8 + 1, device="cuda")[1:].view(a.N, 8)
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.run(Bm)                                   # not 16-byte aligned
+    assert ex.value.status == 3
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.permute("cta_aware", window=48)          # not a multiple of nw
+    assert ex.value.status == 1
+    big = syn.rmat(16, 2, 5)
+    hb = pkg.SpMM.from_csr(big)
+    with pytest.raises(pkg.SpmmError) as ex:
+        hb.permute("cta_aware", window=0)          # W=0 above 32768 rows
+    assert ex.value.status == 3
+    hb.close()
+    h.close()
+    # invalid CSR
+    bad = [(np.array([0, 2, 1, 3]), np.array([0, 1, 2], np.int32)),      # decreasing offsets
+           (np.array([0, 2, 3, 3]), np.array([1, 0, 2], np.int32)),      # unsorted row
+           (np.array([0, 1, 2, 3]), np.array([0, 9, 2], np.int32)),      # out of range
+           (np.array([1, 2, 3, 3]), np.array([0, 1, 2], np.int32))]      # rowidx[0] != 0
+    for r, c in bad:
+        with pytest.raises(pkg.SpmmError) as ex:
+            pkg.SpMM(3, 4, r, c, np.ones(3, np.float32))
+        assert ex.value.status == 2
+
+
+def test_device_inputs_and_host_run():
+    a = syn.rmat(11, 8, 51, "local")
+    K = 64
+    B = syn.dense(a.N, K, 52)
+    C_ref, bound = oracle.spmm(a, B)
+    h = pkg.SpMM(a.M, a.N, torch.from_numpy(a.rowidx).cuda(), torch.from_numpy(a.colidx).cuda(),
+                 torch.from_numpy(a.value).cuda())
+    h.permute("hybrid_2_1")
+    Bh = torch.from_numpy(B).pin_memory()
+    Ch = torch.empty((a.M, K), dtype=torch.float32).pin_memory()
+    h.run_host(Bh, Ch)
+    ok, worst = within_tol(Ch.numpy(), C_ref, bound)
+    assert ok, worst
+    h.close()
+
+
+def test_torch_allocator_and_streams():
+    pkg.use_torch_allocator(True)
+    try:
+        a = syn.rmat(12, 8, 61, "natural")
+        B = syn.dense(a.N, 128, 62)
+        C_ref, bound = oracle.spmm(a, B)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            h = pkg.SpMM.from_csr(a, stream=s)
+            h.permute("cta_aware", stream=s)
+            Bd = torch.from_numpy(B).cuda()
+            C = h.run(Bd, stream=s)
+        s.synchronize()
+        ok, worst = within_tol(C.cpu().numpy(), C_ref, bound)
+        assert ok, worst
+        assert pkg.SpMM.last_run_launches() >= 1
+        h.close()
+    finally:
+        pkg.use_torch_allocator(False)
