@@ -92,8 +92,10 @@ spmm_status spmm_set_allocator(void *(*alloc)(size_t bytes, void *stream, void *
 spmm_status spmm_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, const int64_t *rowidx,
                         const int32_t *colidx, const float *value, int inputs_on_device, void *cuda_stream);
 
-/* Build permutation `policy` (params NULL = defaults) and the permuted CSR + long-row chunk table it
- * implies, all on the device (offline / amortised).  Replaces the previous permutation.
+/* Build permutation `policy` (params NULL = defaults), the permuted CSR it implies and its row-class
+ * counts, all on the device (offline / amortised).  Replaces the previous permutation.  The
+ * K-dependent run schedule (a7: empty / whole / split rows packed into warp tasks) is built by the next
+ * spmm_run (once per permutation and lanes-per-row geometry; that call synchronises its stream).
  * Needs external synchronisation against spmm_run on the same handle. */
 spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *params, void *cuda_stream);
 
@@ -103,8 +105,9 @@ spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out);
 /* Copy the current permuted CSR to HOST buffers: rowidx int64[M+1], colidx int32[nnz], value f32[nnz]. */
 spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colidx, float *value);
 
-/* Counters of the current permutation: out[0]=rows with nnz==0, out[1]=rows handled whole,
- * out[2]=split (long) rows, out[3]=chunks of the split rows, out[4]=max row nnz. */
+/* Row classes of the current permutation (a7): out[0]=empty rows (nnz==0, zero-filled), out[1]=non-empty
+ * rows handled whole (nnz <= split_nnz), out[2]=split (long) rows, out[3]=split_nnz-chunks of the split
+ * rows, out[4]=max row nnz. */
 spmm_status spmm_get_info(spmm_handle h, int64_t out[5]);
 
 /* The 24 Table II features (definitions DESIGN.md §"Features") computed on the device,

@@ -253,9 +253,9 @@ spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colid
 spmm_status spmm_get_info(spmm_handle h, int64_t out[5]) {
     if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     out[0] = h->n_empty;
-    out[1] = h->M - h->lr.n_long;
-    out[2] = h->lr.n_long;
-    out[3] = h->lr.n_chunks;
+    out[1] = h->M - h->n_empty - h->rc.n_long;
+    out[2] = h->rc.n_long;
+    out[3] = h->rc.n_chunks;
     out[4] = h->max_row_nnz;
     return SPMM_OK;
 }

@@ -55,13 +55,27 @@ struct DevBuf {
 };
 
 // ---- the handle -----------------------------------------------------------------------------
-struct LongRows {
+// a7 row classes (counts, K-independent; computed by spmm_permute)
+struct RowClasses {
     int64_t n_long = 0;       // rows with nnz > split_nnz
-    int64_t n_chunks = 0;     // total chunks over those rows
-    DevBuf chunk_start;       // int32[n_chunks]  start offset into the permuted CSR
-    DevBuf chunk_len;         // int32[n_chunks]
-    DevBuf long_pos;          // int32[n_long]    position p of each long row
-    DevBuf long_chunk_ptr;    // int32[n_long+1]  chunk range of each long row
+    int64_t n_chunks = 0;     // split_nnz-chunks over those rows
+};
+
+// a7 run schedule for one lanes-per-row geometry (rows per warp RPW), built on the first spmm_run after
+// a permute with that RPW.  Warp task t owns units [t*RPW, (t+1)*RPW): either up to RPW consecutive
+// non-empty short rows of the permuted order, or RPW consecutive chunks of one long row (a chunk group,
+// reduced across the warp into one partial).  Units: int4 (start, len, dst, 0); dst >= 0: C row,
+// dst == INT_MIN: padding, dst < 0: chunk group -> partial slot -(dst+1).
+struct Schedule {
+    int32_t rpw = 0;          // 0 = not built
+    int64_t n_tasks = 0;
+    DevBuf units;             // int4[n_tasks * rpw]
+    int64_t n_long = 0;
+    DevBuf long_dst;          // int32[n_long]      C row of each long row
+    DevBuf pslot_ptr;         // int32[n_long + 1]  partial-slot range of each long row
+    int64_t n_pslots = 0;
+    int64_t n_empty = 0;
+    DevBuf empty_dst;         // int32[n_empty]     C rows of empty rows (zero-filled)
 };
 
 }  // namespace spmm
@@ -82,7 +96,8 @@ struct spmm_ctx {
     spmm::DevBuf perm;     // int32[M]
     spmm::DevBuf rowptr_p; // int32[M+1]
     spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
-    spmm::LongRows lr;
+    spmm::RowClasses rc;
+    spmm::Schedule sched;
     // run scratch (partials of split rows), grown on demand
     spmm::DevBuf partials;
     // host-run staging

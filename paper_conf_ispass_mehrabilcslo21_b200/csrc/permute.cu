@@ -340,24 +340,6 @@ __global__ void k_long_flags(const int32_t *rowptr_p, int64_t M, int32_t split, 
     }
 }
 
-// per long row (warp): record its position and write its chunk table
-__global__ void k_long_fill(const int32_t *rowptr_p, const int32_t *flag, const int32_t *lpos, const int32_t *choff,
-                            int64_t M, int32_t split, int32_t *long_pos, int32_t *long_chunk_ptr, int32_t *cstart,
-                            int32_t *clen) {
-    const int lane = threadIdx.x & 31;
-    for (int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < M;
-         p += ((int64_t)gridDim.x * blockDim.x) >> 5) {
-        if (!flag[p]) continue;
-        int32_t l = lpos[p], c0 = choff[p], a = rowptr_p[p], len = rowptr_p[p + 1] - a;
-        int32_t nc = (len + split - 1) / split;
-        if (lane == 0) { long_pos[l] = (int32_t)p; long_chunk_ptr[l] = c0; }
-        for (int32_t c = lane; c < nc; c += 32) {
-            cstart[c0 + c] = a + c * split;
-            clen[c0 + c] = min(split, len - c * split);
-        }
-    }
-}
-
 inline unsigned grid_for(int64_t n, int threads) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, threads), 148 * 32));
 }
@@ -545,35 +527,21 @@ spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s) {
                                                    h->perm.as<int32_t>(), h->rowptr_p.as<int32_t>(), M, h->cv_p.as<int2>());
         SPMM_CUDA(cudaGetLastError());
     }
-    // long rows and their chunk table
-    LongRows &lr = h->lr;
-    lr.n_long = lr.n_chunks = 0;
-    if (M == 0 || h->max_row_nnz <= split) {
-        lr.chunk_start.release(); lr.chunk_len.release(); lr.long_pos.release(); lr.long_chunk_ptr.release();
-        return SPMM_OK;
-    }
-    DevBuf flag, nch, lpos, choff;
+    // a7 row-class counts (the K-dependent run schedule is built by the first spmm_run)
+    h->sched.rpw = 0;
+    h->rc.n_long = h->rc.n_chunks = 0;
+    if (M == 0 || h->max_row_nnz <= split) return SPMM_OK;
+    DevBuf flag, nch, tmp;
     SPMM_TRY(flag.alloc(M * sizeof(int32_t), s));
     SPMM_TRY(nch.alloc(M * sizeof(int32_t), s));
-    SPMM_TRY(lpos.alloc((M + 1) * sizeof(int32_t), s));
-    SPMM_TRY(choff.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(tmp.alloc((M + 1) * sizeof(int32_t), s));
     k_long_flags<<<grid_for(M, 256), 256, 0, s>>>(h->rowptr_p.as<int32_t>(), M, split, flag.as<int32_t>(), nch.as<int32_t>());
     SPMM_CUDA(cudaGetLastError());
     int32_t nlong = 0, nchunks = 0;
-    SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), lpos.as<int32_t>(), M, &nlong, s));
-    SPMM_TRY(exclusive_scan_i32(nch.as<int32_t>(), choff.as<int32_t>(), M, &nchunks, s));
-    lr.n_long = nlong;
-    lr.n_chunks = nchunks;
-    SPMM_TRY(lr.long_pos.alloc(std::max(nlong, 1) * sizeof(int32_t), s));
-    SPMM_TRY(lr.long_chunk_ptr.alloc((nlong + 1) * sizeof(int32_t), s));
-    SPMM_TRY(lr.chunk_start.alloc(std::max(nchunks, 1) * sizeof(int32_t), s));
-    SPMM_TRY(lr.chunk_len.alloc(std::max(nchunks, 1) * sizeof(int32_t), s));
-    k_long_fill<<<grid_warps(M, 256), 256, 0, s>>>(h->rowptr_p.as<int32_t>(), flag.as<int32_t>(), lpos.as<int32_t>(),
-                                                  choff.as<int32_t>(), M, split, lr.long_pos.as<int32_t>(),
-                                                  lr.long_chunk_ptr.as<int32_t>(), lr.chunk_start.as<int32_t>(),
-                                                  lr.chunk_len.as<int32_t>());
-    k_set_last<<<1, 1, 0, s>>>(lr.long_chunk_ptr.as<int32_t>(), nlong, nchunks);
-    SPMM_CUDA(cudaGetLastError());
+    SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), tmp.as<int32_t>(), M, &nlong, s));
+    SPMM_TRY(exclusive_scan_i32(nch.as<int32_t>(), tmp.as<int32_t>(), M, &nchunks, s));
+    h->rc.n_long = nlong;
+    h->rc.n_chunks = nchunks;
     return SPMM_OK;
 }
 

@@ -1,28 +1,35 @@
 // spmm_kernels.cu -- the timed SpMM of the hot path (a8):
 //   C[perm[p]][k] = sum_{j in row' p} value'[j] * B[colidx'[j]][k]      (Alg.1)
-// on the row-permuted CSR, with the inverse permutation fused into the C store.
+// on the row-permuted CSR, with the inverse permutation fused into the C store, plus the a7 run
+// schedule (row classes: empty / whole / split rows) it executes.
 //
 // B200 design (DESIGN.md §"SpMM kernel"), not the paper's warp-per-row Volta kernel:
-//   * a row is owned by a lane GROUP of G lanes; each lane owns V float4 column vectors of the C
-//     row (4*V*G columns per tile), so a warp works on 32/G consecutive permuted rows at once and
-//     the sorted/clustered orders decide how balanced those rows are (the paper's "warp load",
-//     P:L84-88, re-expressed for this mapping);
+//   * a work unit is owned by a lane GROUP of G lanes; each lane owns V float4 column vectors of the
+//     C row (4*V*G columns per tile), so a warp works on RPW = 32/G units at once, and the sorted /
+//     clustered orders decide how balanced those units are (the paper's "warp load", P:L84-88,
+//     re-expressed for this mapping);
 //   * per nnz, the G lanes of a group broadcast-load the interleaved (col, val) pair (8 B) and issue
 //     V coalesced 16-byte loads of the B row (G*16 B contiguous per vector), then 4*V FP32 FMAs as
 //     packed FFMA2 (sm_100 fma.rn.f32x2) -- every accumulator is a sequential chain in ascending j,
 //     the order of the oracle's definition (oracle.c c1);
-//   * rows longer than split_nnz are cut into split_nnz-nnz chunks processed like rows; their
-//     partial sums are combined in a fixed pairwise order by k_combine (deterministic, bounded
-//     rounding, DESIGN.md §"Accuracy");
+//   * warp tasks follow the permuted order: runs of non-empty short rows are packed RPW per task;
+//     a row longer than split_nnz is cut into split_nnz-nnz chunks, RPW consecutive chunks form one
+//     warp task whose group sums are reduced across the warp in a fixed butterfly tree, and the
+//     per-task partials are combined in a fixed pairwise order by k_combine (deterministic, bounded
+//     rounding, DESIGN.md §"Accuracy"); all chunking is relative to the row start, so C is
+//     bit-identical for every permutation;
+//   * empty rows are a class of their own (zero-filled, the B200 form of DCSR's skip);
 //   * C is written once with streaming stores at C[perm[p]] (original order, beta = 0).
 // Bound: HBM bandwidth (algorithmic bytes 4(M+1) + 8 nnz + 4K|cols(A)| + 4MK, BASELINE.json north star).
 #include "internal.cuh"
 #include <algorithm>
+#include <climits>
 
 namespace spmm {
 namespace {
 
 constexpr int SPMM_THREADS = 256;
+constexpr int32_t NOSTORE = INT_MIN;
 
 __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
     float2 lo = __ffma2_rn(make_float2(a, a), make_float2(b.x, b.y), make_float2(acc.x, acc.y));
@@ -30,46 +37,25 @@ __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
     acc.x = lo.x; acc.y = lo.y; acc.z = hi.x; acc.w = hi.y;
 }
 
-// U nnz per iteration, V float4 per lane, G lanes per row, MASK: column tail present.
+// V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
 template <int V, int G, bool MASK>
-__global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int32_t *__restrict__ rowptr, const int2 *__restrict__ cv,
-                                                       const int32_t *__restrict__ perm, const float4 *__restrict__ B4,
-                                                       float4 *__restrict__ C4, int64_t M, int32_t K4, int32_t split,
-                                                       const int32_t *__restrict__ cstart,
-                                                       const int32_t *__restrict__ clen, int64_t n_chunks,
-                                                       float4 *__restrict__ P4) {
+__global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
+                                                       const int2 *__restrict__ cv, const float4 *__restrict__ B4,
+                                                       float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4) {
     constexpr int RPW = 32 / G;
     constexpr int CT4 = V * G;
     constexpr int U = 2;
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
     const int col0 = blockIdx.y * CT4 + gl;      // this lane's first float4 column; then + v*G
-    const int64_t row_tasks = (M + RPW - 1) / RPW;
-    const int64_t total = row_tasks + (n_chunks + RPW - 1) / RPW;
     const int64_t nwarps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
     bool colok[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < K4);
 
-    for (int64_t t = (int64_t)blockIdx.x * (SPMM_THREADS / 32) + (threadIdx.x >> 5); t < total; t += nwarps) {
-        int32_t start = 0, end = 0;
-        float4 *dst = nullptr;
-        if (t < row_tasks) {
-            const int64_t p = t * RPW + g;
-            if (p < M) {
-                start = __ldg(rowptr + p);
-                end = __ldg(rowptr + p + 1);
-                if (end - start <= split) dst = C4 + (size_t)__ldg(perm + p) * K4;
-            }
-        } else {
-            const int64_t c = (t - row_tasks) * RPW + g;
-            if (c < n_chunks) {
-                start = __ldg(cstart + c);
-                end = start + __ldg(clen + c);
-                dst = P4 + (size_t)c * K4;
-            }
-        }
-        if (dst == nullptr) continue;   // long row (its chunks do the work) or past the end
+    for (int64_t t = (int64_t)blockIdx.x * (SPMM_THREADS / 32) + (threadIdx.x >> 5); t < n_tasks; t += nwarps) {
+        const int4 u = __ldg(units + t * RPW + g);
+        const int32_t start = u.x, end = u.x + u.y, dst = u.z;
         float4 acc[V];
 #pragma unroll
         for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -77,19 +63,19 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int32_t *__restrict
         for (; j + U <= end; j += U) {
             int2 e[U];
 #pragma unroll
-            for (int u = 0; u < U; ++u) e[u] = __ldg(cv + j + u);
+            for (int q = 0; q < U; ++q) e[q] = __ldg(cv + j + q);
             float4 x[U][V];
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const float4 *b = B4 + (size_t)e[u].x * K4 + col0;
+            for (int q = 0; q < U; ++q) {
+                const float4 *b = B4 + (size_t)e[q].x * K4 + col0;
 #pragma unroll
-                for (int v = 0; v < V; ++v) x[u][v] = colok[v] ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int v = 0; v < V; ++v) x[q][v] = colok[v] ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
             }
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const float a = __int_as_float(e[u].y);
+            for (int q = 0; q < U; ++q) {
+                const float a = __int_as_float(e[q].y);
 #pragma unroll
-                for (int v = 0; v < V; ++v) fma4(a, x[u][v], acc[v]);
+                for (int v = 0; v < V; ++v) fma4(a, x[q][v], acc[v]);
             }
         }
         if (j < end) {
@@ -100,21 +86,39 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int32_t *__restrict
             for (int v = 0; v < V; ++v)
                 if (colok[v]) fma4(a, __ldg(b + v * G), acc[v]);
         }
+        if (dst >= 0) {                                    // a whole row: C[perm[p]]
 #pragma unroll
-        for (int v = 0; v < V; ++v)
-            if (colok[v]) __stcs(dst + col0 + v * G, acc[v]);
+            for (int v = 0; v < V; ++v)
+                if (colok[v]) __stcs(C4 + (size_t)dst * K4 + col0 + v * G, acc[v]);
+        } else if (dst != NOSTORE) {                       // chunk group of a long row (warp-uniform)
+#pragma unroll
+            for (int off = G; off < 32; off <<= 1) {       // fixed butterfly: ((c0+c1)+(c2+c3))...
+#pragma unroll
+                for (int v = 0; v < V; ++v) {
+                    acc[v].x += __shfl_xor_sync(0xffffffffu, acc[v].x, off);
+                    acc[v].y += __shfl_xor_sync(0xffffffffu, acc[v].y, off);
+                    acc[v].z += __shfl_xor_sync(0xffffffffu, acc[v].z, off);
+                    acc[v].w += __shfl_xor_sync(0xffffffffu, acc[v].w, off);
+                }
+            }
+            if (g == 0) {
+                const int64_t slot = -(int64_t)dst - 1;
+#pragma unroll
+                for (int v = 0; v < V; ++v)
+                    if (colok[v]) P4[slot * K4 + col0 + v * G] = acc[v];
+            }
+        }
     }
 }
 
-// Pairwise (binary-counter) combine of a long row's chunk partials, fixed order -> deterministic;
-// rounding grows with log2(#chunks) instead of #chunks.  One CTA per long row, thread per float4.
-__global__ void __launch_bounds__(128) k_combine(const float4 *__restrict__ P4, const int32_t *__restrict__ long_pos,
-                                                 const int32_t *__restrict__ long_chunk_ptr,
-                                                 const int32_t *__restrict__ perm, float4 *__restrict__ C4,
+// Pairwise (binary-counter) combine of a long row's chunk-group partials, fixed order -> deterministic;
+// rounding grows with log2(#groups).  One CTA per long row, thread per float4 column.
+__global__ void __launch_bounds__(128) k_combine(const float4 *__restrict__ P4, const int32_t *__restrict__ pslot_ptr,
+                                                 const int32_t *__restrict__ long_dst, float4 *__restrict__ C4,
                                                  int32_t K4) {
     const int32_t l = blockIdx.x;
-    const int32_t c0 = long_chunk_ptr[l], c1 = long_chunk_ptr[l + 1];
-    float4 *dst = C4 + (size_t)perm[long_pos[l]] * K4;
+    const int32_t c0 = pslot_ptr[l], c1 = pslot_ptr[l + 1];
+    float4 *dst = C4 + (size_t)long_dst[l] * K4;
     for (int32_t col = threadIdx.x; col < K4; col += blockDim.x) {
         float4 stk[32];
         int sp = 0;
@@ -135,13 +139,150 @@ __global__ void __launch_bounds__(128) k_combine(const float4 *__restrict__ P4, 
     }
 }
 
-__global__ void k_zero_rows(float4 *C4, int64_t n4) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
-        C4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+// empty rows: zero-fill their C rows (thread per float4)
+__global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, float4 *__restrict__ C4) {
+    const int64_t total = n * K4;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
+        __stcs(C4 + (size_t)rows[i / K4] * K4 + (i % K4), make_float4(0.f, 0.f, 0.f, 0.f));
 }
 
-using SpmmKernel = void (*)(const int32_t *, const int2 *, const int32_t *, const float4 *, float4 *, int64_t, int32_t,
-                            int32_t, const int32_t *, const int32_t *, int64_t, float4 *);
+// ---- a7 schedule construction ------------------------------------------------------------------
+// class flags per position: 0 empty, 1 short (0 < len <= split), 2 long
+__global__ void k_class_flags(const int32_t *rowptr, int64_t M, int32_t split, int32_t *is_empty, int32_t *is_short,
+                              int32_t *is_long) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t len = rowptr[p + 1] - rowptr[p];
+        is_empty[p] = len == 0;
+        is_short[p] = len > 0 && len <= split;
+        is_long[p] = len > split;
+    }
+}
+
+__global__ void k_scatter_flagged(const int32_t *flag, const int32_t *pos, const int32_t *val, int64_t M, int32_t *out) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x)
+        if (flag[p]) out[pos[p]] = val ? val[p] : (int32_t)p;
+}
+
+// per "segment" k = 0..n_long: the run of short rows before long row k (k = n_long: trailing run) and
+// long row k itself.  tasks_k = ceil(s_k / RPW) + ceil(nch_k / RPW); groups_k = ceil(nch_k / RPW).
+__global__ void k_segment_counts(const int32_t *lpos, int64_t n_long, const int32_t *sp, int32_t n_short,
+                                 const int32_t *rowptr, int32_t split, int32_t rpw, int32_t *tasks, int32_t *groups) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k <= n_long; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t before = k > 0 ? sp[lpos[k - 1]] : 0;
+        const int32_t upto = k < n_long ? sp[lpos[k]] : n_short;
+        const int32_t s_k = upto - before;
+        int32_t nch = 0;
+        if (k < n_long) {
+            const int32_t len = rowptr[lpos[k] + 1] - rowptr[lpos[k]];
+            nch = (len + split - 1) / split;
+        }
+        const int32_t gk = (nch + rpw - 1) / rpw;
+        tasks[k] = (s_k + rpw - 1) / rpw + gk;
+        groups[k] = gk;
+    }
+}
+
+__global__ void k_fill_short(const int32_t *is_short, const int32_t *sp, const int32_t *lidx, const int32_t *lpos,
+                             const int32_t *taskbase, const int32_t *rowptr, const int32_t *perm, int64_t M,
+                             int32_t rpw, int4 *units) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        if (!is_short[p]) continue;
+        const int32_t k = lidx[p];                         // long rows before p = this run's segment
+        const int32_t idx = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
+        const int64_t task = (int64_t)taskbase[k] + idx / rpw;
+        units[task * rpw + idx % rpw] = make_int4(rowptr[p], rowptr[p + 1] - rowptr[p], perm[p], 0);
+    }
+}
+
+// warp per long row: its chunk groups follow the run of short rows of its segment
+__global__ void k_fill_long(const int32_t *lpos, int64_t n_long, const int32_t *sp, const int32_t *taskbase,
+                            const int32_t *pslot_ptr, const int32_t *rowptr, const int32_t *perm, int32_t split,
+                            int32_t rpw, int4 *units, int32_t *long_dst) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t k = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n_long;
+         k += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int32_t p = lpos[k];
+        const int32_t s_k = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
+        const int64_t t0 = (int64_t)taskbase[k] + (s_k + rpw - 1) / rpw;
+        const int32_t a = rowptr[p], len = rowptr[p + 1] - a, nch = (len + split - 1) / split;
+        const int32_t ng = pslot_ptr[k + 1] - pslot_ptr[k];
+        for (int32_t c = lane; c < ng * rpw; c += 32) {
+            const int32_t dst = -(pslot_ptr[k] + c / rpw) - 1;
+            units[(t0 + c / rpw) * rpw + c % rpw] =
+                c < nch ? make_int4(a + c * split, min(split, len - c * split), dst, 0) : make_int4(0, 0, dst, 0);
+        }
+        if (lane == 0) long_dst[k] = perm[p];
+    }
+}
+
+__global__ void k_fill_int4(int4 *a, int64_t n, int4 v) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) a[i] = v;
+}
+
+inline unsigned g1(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 32)); }
+
+spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
+    Schedule &S = h->sched;
+    S.rpw = 0;
+    const int64_t M = h->M;
+    const int32_t split = h->params.split_nnz;
+    const int32_t *rowptr = h->rowptr_p.as<int32_t>();
+    DevBuf fe, fs, fl, pe, ps, pl, lpos, tasks, groups, taskbase;
+    SPMM_TRY(fe.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(fs.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(fl.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(pe.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(ps.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(pl.alloc((M + 1) * sizeof(int32_t), s));
+    k_class_flags<<<g1(M), 256, 0, s>>>(rowptr, M, split, fe.as<int32_t>(), fs.as<int32_t>(), fl.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    int32_t n_empty = 0, n_short = 0, n_long = 0;
+    SPMM_TRY(exclusive_scan_i32(fe.as<int32_t>(), pe.as<int32_t>(), M, &n_empty, s));
+    SPMM_TRY(exclusive_scan_i32(fs.as<int32_t>(), ps.as<int32_t>(), M, &n_short, s));
+    SPMM_TRY(exclusive_scan_i32(fl.as<int32_t>(), pl.as<int32_t>(), M, &n_long, s));
+    // empty rows -> their C rows
+    S.n_empty = n_empty;
+    SPMM_TRY(S.empty_dst.alloc(std::max(n_empty, 1) * sizeof(int32_t), s));
+    k_scatter_flagged<<<g1(M), 256, 0, s>>>(fe.as<int32_t>(), pe.as<int32_t>(), h->perm.as<int32_t>(), M,
+                                            S.empty_dst.as<int32_t>());
+    // long rows in order
+    SPMM_TRY(lpos.alloc(std::max(n_long, 1) * sizeof(int32_t), s));
+    k_scatter_flagged<<<g1(M), 256, 0, s>>>(fl.as<int32_t>(), pl.as<int32_t>(), nullptr, M, lpos.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    // segments: tasks and chunk groups
+    SPMM_TRY(tasks.alloc((n_long + 1) * sizeof(int32_t), s));
+    SPMM_TRY(groups.alloc((n_long + 1) * sizeof(int32_t), s));
+    SPMM_TRY(taskbase.alloc((n_long + 2) * sizeof(int32_t), s));
+    SPMM_TRY(S.pslot_ptr.alloc((n_long + 2) * sizeof(int32_t), s));
+    k_segment_counts<<<g1(n_long + 1), 256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), n_short, rowptr,
+                                                    split, rpw, tasks.as<int32_t>(), groups.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    int32_t n_tasks = 0, n_groups = 0;
+    SPMM_TRY(exclusive_scan_i32(tasks.as<int32_t>(), taskbase.as<int32_t>(), n_long + 1, &n_tasks, s));
+    SPMM_TRY(exclusive_scan_i32(groups.as<int32_t>(), S.pslot_ptr.as<int32_t>(), n_long + 1, &n_groups, s));
+    S.n_tasks = n_tasks;
+    S.n_pslots = n_groups;
+    S.n_long = n_long;
+    SPMM_TRY(S.units.alloc(std::max<int64_t>((int64_t)n_tasks * rpw, 1) * sizeof(int4), s));
+    SPMM_TRY(S.long_dst.alloc(std::max(n_long, 1) * sizeof(int32_t), s));
+    if (n_tasks > 0) {
+        k_fill_int4<<<g1((int64_t)n_tasks * rpw), 256, 0, s>>>(S.units.as<int4>(), (int64_t)n_tasks * rpw,
+                                                                make_int4(0, 0, NOSTORE, 0));
+        k_fill_short<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), pl.as<int32_t>(), lpos.as<int32_t>(),
+                                           taskbase.as<int32_t>(), rowptr, h->perm.as<int32_t>(), M, rpw,
+                                           S.units.as<int4>());
+        if (n_long > 0)
+            k_fill_long<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)n_long * 32, 256), 148 * 32)),
+                          256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), taskbase.as<int32_t>(),
+                                       S.pslot_ptr.as<int32_t>(), rowptr, h->perm.as<int32_t>(), split, rpw,
+                                       S.units.as<int4>(), S.long_dst.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    S.rpw = rpw;
+    return SPMM_OK;
+}
+
+using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *);
 
 template <int V, bool MASK>
 SpmmKernel pick_g(int G) {
@@ -184,40 +325,38 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
-    if (h->nnz == 0) {
-        k_zero_rows<<<(unsigned)std::min<int64_t>(ceil_div(M * K4, 256), 148 * 16), 256, 0, s>>>(
-            reinterpret_cast<float4 *>(C), M * K4);
-        SPMM_CUDA(cudaGetLastError());
-        *launches = 1;
-        return SPMM_OK;
-    }
-    const LongRows &lr = h->lr;
+    const Config cfg = choose(K4);
+    const int32_t rpw = 32 / cfg.G;
+    if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
+    const Schedule &S = h->sched;
+    float4 *C4 = reinterpret_cast<float4 *>(C);
     float4 *P4 = nullptr;
-    if (lr.n_chunks > 0) {
-        size_t need = (size_t)lr.n_chunks * K * sizeof(float);
+    if (S.n_pslots > 0) {
+        const size_t need = (size_t)S.n_pslots * K * sizeof(float);
         if (h->partials.bytes < need) SPMM_TRY(h->partials.alloc(need, s));
         P4 = h->partials.as<float4>();
     }
-    Config cfg = choose(K4);
-    const int rpw = 32 / cfg.G;
-    const int64_t tasks = ceil_div(M, rpw) + ceil_div(lr.n_chunks, rpw);
-    int occ = 0;
-    SPMM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, cfg.kern, SPMM_THREADS, 0));
-    occ = std::max(occ, 1);
-    const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(tasks, SPMM_THREADS / 32),
-                                                                  (int64_t)h->num_sms * occ));
-    dim3 grid((unsigned)blocks, (unsigned)cfg.tiles);
-    cfg.kern<<<grid, SPMM_THREADS, 0, s>>>(h->rowptr_p.as<int32_t>(), h->cv_p.as<int2>(), h->perm.as<int32_t>(),
-                                           reinterpret_cast<const float4 *>(B), reinterpret_cast<float4 *>(C), M, K4,
-                                           h->params.split_nnz, lr.chunk_start.as<int32_t>(), lr.chunk_len.as<int32_t>(),
-                                           lr.n_chunks, P4);
-    SPMM_CUDA(cudaGetLastError());
-    *launches = 1;
-    if (lr.n_long > 0) {
-        k_combine<<<(unsigned)lr.n_long, 128, 0, s>>>(P4, lr.long_pos.as<int32_t>(), lr.long_chunk_ptr.as<int32_t>(),
-                                                     h->perm.as<int32_t>(), reinterpret_cast<float4 *>(C), K4);
+    if (S.n_empty > 0) {
+        k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4);
         SPMM_CUDA(cudaGetLastError());
-        *launches = 2;
+        ++*launches;
+    }
+    if (S.n_tasks > 0) {
+        int occ = 0;
+        SPMM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, cfg.kern, SPMM_THREADS, 0));
+        occ = std::max(occ, 1);
+        const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(S.n_tasks, SPMM_THREADS / 32),
+                                                                      (int64_t)h->num_sms * occ));
+        const dim3 grid((unsigned)blocks, (unsigned)cfg.tiles);
+        cfg.kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
+                                               reinterpret_cast<const float4 *>(B), C4, K4, P4);
+        SPMM_CUDA(cudaGetLastError());
+        ++*launches;
+    }
+    if (S.n_long > 0) {
+        k_combine<<<(unsigned)S.n_long, 128, 0, s>>>(P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), C4, K4);
+        SPMM_CUDA(cudaGetLastError());
+        ++*launches;
     }
     return SPMM_OK;
 }
