@@ -197,6 +197,7 @@ def main():
     ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cusparse", action="store_true")
+    ap.add_argument("--no-ceiling", action="store_true", help="skip the host LRU model of L2 reuse")
     ap.add_argument("--out", default=None, help="also write the JSON line to this file")
     args = ap.parse_args()
     assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
@@ -269,6 +270,14 @@ def main():
         ms = statistics.median(ts)
         pol_res[pol] = {"ms": ms, "gflops": flops / ms / 1e6, "build_ms": build_ms, "launches": h.last_run_launches(),
                         "info": h.info()}
+        if not args.no_ceiling and rank == 0:
+            # L2-capacity ceiling: B-row misses of an LRU of L2-size in this order
+            import tools
+            cap = int(torch.cuda.get_device_properties(dev).L2_cache_size // (4 * K))
+            miss = tools.lru_misses(a, h.perm(), cap)
+            traffic = alg_bytes - 4 * K * ncols + 4 * K * miss
+            pol_res[pol]["lru_model"] = {"l2_rows": cap, "b_row_misses": miss, "model_bytes": traffic,
+                                         "ceiling_frac": alg_bytes / traffic}
     # choose the fastest (max over ranks of each policy's time)
     names = list(pol_res)
     tvec = torch.tensor([pol_res[n]["ms"] for n in names], dtype=torch.float64, device=dev)

@@ -100,6 +100,7 @@ struct spmm_ctx {
     spmm::Schedule sched;
     // run scratch (partials of split rows), grown on demand
     spmm::DevBuf partials;
+    spmm::DevBuf counters;  // dynamic warp-task counters, one per column tile
     // host-run staging
     spmm::DevBuf stage_B, stage_C;
     int num_sms = 148;

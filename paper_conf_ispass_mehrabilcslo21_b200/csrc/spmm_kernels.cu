@@ -38,22 +38,28 @@ __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
 }
 
 // V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
+// Warp tasks are claimed dynamically (one atomicAdd per task on a per-column-tile counter), so the set
+// of tasks in flight stays a narrow window of the permuted order whatever the task costs: the order's
+// B-row locality survives into L2 and no warp is left with a long static tail.
 template <int V, int G, bool MASK>
 __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
-                                                       float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4) {
+                                                       float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
+                                                       unsigned int *__restrict__ counter) {
     constexpr int RPW = 32 / G;
     constexpr int CT4 = V * G;
     constexpr int U = 2;
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
     const int col0 = blockIdx.y * CT4 + gl;      // this lane's first float4 column; then + v*G
-    const int64_t nwarps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
     bool colok[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < K4);
 
-    for (int64_t t = (int64_t)blockIdx.x * (SPMM_THREADS / 32) + (threadIdx.x >> 5); t < n_tasks; t += nwarps) {
+    unsigned int tk = 0;
+    if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+    tk = __shfl_sync(0xffffffffu, tk, 0);
+    for (int64_t t = tk; t < n_tasks;) {
         const int4 u = __ldg(units + t * RPW + g);
         const int32_t start = u.x, end = u.x + u.y, dst = u.z;
         float4 acc[V];
@@ -108,6 +114,8 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ 
                     if (colok[v]) P4[slot * K4 + col0 + v * G] = acc[v];
             }
         }
+        if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+        t = __shfl_sync(0xffffffffu, tk, 0);
     }
 }
 
@@ -282,7 +290,8 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
     return SPMM_OK;
 }
 
-using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *);
+using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
+                            unsigned int *);
 
 template <int V, bool MASK>
 SpmmKernel pick_g(int G) {
@@ -348,8 +357,12 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(S.n_tasks, SPMM_THREADS / 32),
                                                                       (int64_t)h->num_sms * occ));
         const dim3 grid((unsigned)blocks, (unsigned)cfg.tiles);
+        if (h->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int))
+            SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
+        SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
         cfg.kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
-                                               reinterpret_cast<const float4 *>(B), C4, K4, P4);
+                                               reinterpret_cast<const float4 *>(B), C4, K4, P4,
+                                               h->counters.as<unsigned int>());
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
