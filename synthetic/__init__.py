@@ -48,6 +48,8 @@ def _load():
         lib.synth_uniform.argtypes = [i64, i64, f64, i32, u64, i32]
         lib.synth_blockcluster.restype = vp
         lib.synth_blockcluster.argtypes = [i64, i64, i64, i64, i64, i32, i32, u64, i32]
+        lib.synth_banded.restype = vp
+        lib.synth_banded.argtypes = [i64, i64, i64, i64, u64, i32]
         lib.synth_from_degrees.restype = vp
         lib.synth_from_degrees.argtypes = [i64, i64, vp, u64, i32]
         lib.synth_sizes.restype = None
@@ -113,6 +115,11 @@ def blockcluster(M: int, N: int, g: int, c: int, d: int, seed: int, planted: boo
     """Groups of g rows share c column blocks of bw columns; d columns per row; rows shuffled."""
     return _take(_load().synth_blockcluster(M, N, g, c, d, bw, int(planted), seed, int(int_values)),
                  f"blockcluster-{M}-g{g}-c{c}-d{d}{'-planted' if planted else ''}-s{seed}")
+
+
+def banded(M: int, d: int, halfwidth: int, seed: int, int_values: bool = False) -> CSR:
+    """Banded random (FEM-like bandwidth): d distinct uniform columns within [i - w, i + w]."""
+    return _take(_load().synth_banded(M, M, d, halfwidth, seed, int(int_values)), f"banded-{M}-d{d}-w{halfwidth}-s{seed}")
 
 
 def from_degrees(M: int, N: int, degrees: np.ndarray, seed: int, int_values: bool = False) -> CSR:

@@ -343,6 +343,39 @@ void *synth_from_degrees(int64_t M, int64_t N, const int64_t *deg_in, uint64_t s
     return s;
 }
 
+/* Banded random: row i draws min(d, band) distinct columns uniformly in [i-w, i+w] (clipped to [0,N)). */
+void *synth_banded(int64_t M, int64_t N, int64_t d, int64_t w, uint64_t seed, int32_t value_mode) {
+    int64_t *off = (int64_t *)malloc((size_t)(M + 1) * sizeof(int64_t));
+    off[0] = 0;
+    for (int64_t i = 0; i < M; ++i) {
+        int64_t lo = i - w < 0 ? 0 : i - w, hi = i + w + 1 > N ? N : i + w + 1;
+        int64_t band = hi > lo ? hi - lo : 0;
+        off[i + 1] = off[i] + (d < band ? d : band);
+    }
+    const int64_t E = off[M];
+    int32_t *er = (int32_t *)malloc((size_t)(E ? E : 1) * sizeof(int32_t));
+    int32_t *ec = (int32_t *)malloc((size_t)(E ? E : 1) * sizeof(int32_t));
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t i = 0; i < M; ++i) {
+        int64_t lo = i - w < 0 ? 0 : i - w, hi = i + w + 1 > N ? N : i + w + 1;
+        int64_t band = hi - lo, k = off[i + 1] - off[i], base = off[i], got = 0;
+        for (int64_t t = band - k; t < band; ++t) {   /* Floyd over [0, band) */
+            int64_t v = (int64_t)(((unsigned __int128)rnd(seed, STREAM_UNIF + 11, (uint64_t)(base + got)) *
+                                   (unsigned __int128)(t + 1)) >> 64);
+            int dup = 0;
+            for (int64_t q = 0; q < got; ++q)
+                if (ec[base + q] == (int32_t)(lo + v)) { dup = 1; break; }
+            ec[base + got] = (int32_t)(lo + (dup ? t : v));
+            er[base + got] = (int32_t)i;
+            ++got;
+        }
+    }
+    free(off);
+    staged_csr *s = edges_to_csr(M, N, E, er, ec, seed, value_mode);
+    free(er); free(ec);
+    return s;
+}
+
 void synth_sizes(const void *h, int64_t *M, int64_t *N, int64_t *nnz) {
     const staged_csr *s = (const staged_csr *)h;
     *M = s->M; *N = s->N; *nnz = s->nnz;
