@@ -24,6 +24,7 @@
 #include "internal.cuh"
 #include <algorithm>
 #include <climits>
+#include <cstdlib>
 
 namespace spmm {
 namespace {
@@ -41,14 +42,59 @@ __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
 // Warp tasks are claimed dynamically (one atomicAdd per task on a per-column-tile counter), so the set
 // of tasks in flight stays a narrow window of the permuted order whatever the task costs: the order's
 // B-row locality survives into L2 and no warp is left with a long static tail.
-template <int V, int G, bool MASK>
+// CTA-contiguous task claiming (SCHED = 1): the CTA takes chunks of CTA_CHUNK consecutive warp tasks
+// from the global counter, so the consecutive rows of a chunk run concurrently on one SM (the paper's
+// "clusters of N_w consecutive rows ... processed in parallel" by a CTA) and their shared B rows
+// can hit in L1.  Warps draw tickets from a shared-memory counter; ticket k belongs to local chunk
+// k / CTA_CHUNK, whose global id is published in a ring slot by the warp holding its first ticket.  A
+// slot is republished only after all readers of its previous chunk have read it (no ABA, no barrier).
+constexpr int CTA_CHUNK = SPMM_THREADS / 32;
+constexpr int RING = 4;
+
+struct TaskQueue {
+    unsigned int ticket;
+    unsigned int gid[RING];
+    int tag[RING];
+    int pending[RING];
+};
+
+__device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *gcounter, int lane) {
+    unsigned int task = 0;
+    if (lane == 0) {
+        const unsigned int k = atomicAdd(&q->ticket, 1u);
+        const int c = (int)(k / CTA_CHUNK), w = (int)(k % CTA_CHUNK), s = c % RING;
+        volatile int *vtag = q->tag;
+        volatile int *vpend = q->pending;
+        volatile unsigned int *vgid = q->gid;
+        unsigned int g;
+        if (w == 0) {
+            while (vpend[s] != 0) { }
+            g = atomicAdd(gcounter, 1u);
+            vgid[s] = g;
+            vpend[s] = CTA_CHUNK - 1;
+            __threadfence_block();
+            vtag[s] = c;
+        } else {
+            while (vtag[s] != c) { }
+            __threadfence_block();
+            g = vgid[s];
+            atomicSub(&q->pending[s], 1);
+        }
+        task = g * CTA_CHUNK + (unsigned int)w;
+    }
+    return __shfl_sync(0xffffffffu, task, 0);
+}
+
+template <int V, int G, bool MASK, int SCHED>
 __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter) {
     constexpr int RPW = 32 / G;
     constexpr int CT4 = V * G;
-    constexpr int U = 2;
+    constexpr int U = V >= 3 ? 2 : 4;            // nnz per inner step (B loads in flight per lane: U*V)
+    constexpr int BATCH = G >= 8 ? G : 8;        // (col, val) pairs prefetched per group per batch
+    constexpr int PL = BATCH / G;                // pairs held per lane
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
     const int col0 = blockIdx.y * CT4 + gl;      // this lane's first float4 column; then + v*G
@@ -56,41 +102,82 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ 
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < K4);
 
+    __shared__ TaskQueue q;
     unsigned int tk = 0;
-    if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
-    tk = __shfl_sync(0xffffffffu, tk, 0);
-    for (int64_t t = tk; t < n_tasks;) {
-        const int4 u = __ldg(units + t * RPW + g);
-        const int32_t start = u.x, end = u.x + u.y, dst = u.z;
+    if (SCHED == 1) {
+        if (threadIdx.x == 0) {
+            q.ticket = 0;
+            for (int r = 0; r < RING; ++r) { q.tag[r] = -1; q.pending[r] = 0; q.gid[r] = 0; }
+        }
+        __syncthreads();
+        tk = claim_task(&q, counter + blockIdx.y, lane);
+    } else {
+        if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+        tk = __shfl_sync(0xffffffffu, tk, 0);
+    }
+    int64_t t = tk;
+    int4 u = t < n_tasks ? __ldg(units + t * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+    while (t < n_tasks) {
+        // claim and fetch the next task first, so its latency hides behind this one
+        int64_t t_next;
+        if (SCHED == 1) {
+            t_next = claim_task(&q, counter + blockIdx.y, lane);
+        } else {
+            if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+            t_next = __shfl_sync(0xffffffffu, tk, 0);
+        }
+        const int4 u_next = t_next < n_tasks ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+        const int32_t start = u.x, len = u.y, dst = u.z;
+        // warp-uniform trip count (groups past their own length are predicated off, not diverged, so
+        // the (col, val) shuffles below stay warp-wide)
+        const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
         float4 acc[V];
 #pragma unroll
         for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
-        int32_t j = start;
-        for (; j + U <= end; j += U) {
-            int2 e[U];
+        // (col, val) pairs: each lane loads PL of the group's next BATCH pairs (coalesced), one batch
+        // ahead of use; every nnz is then broadcast inside the group with two shuffles
+        int2 cur[PL];
 #pragma unroll
-            for (int q = 0; q < U; ++q) e[q] = __ldg(cv + j + q);
-            float4 x[U][V];
-#pragma unroll
-            for (int q = 0; q < U; ++q) {
-                const float4 *b = B4 + (size_t)e[q].x * K4 + col0;
-#pragma unroll
-                for (int v = 0; v < V; ++v) x[q][v] = colok[v] ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
-            }
-#pragma unroll
-            for (int q = 0; q < U; ++q) {
-                const float a = __int_as_float(e[q].y);
-#pragma unroll
-                for (int v = 0; v < V; ++v) fma4(a, x[q][v], acc[v]);
-            }
+        for (int p = 0; p < PL; ++p) {
+            const int32_t o = p * G + gl;
+            cur[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
         }
-        if (j < end) {
-            const int2 e = __ldg(cv + j);
-            const float4 *b = B4 + (size_t)e.x * K4 + col0;
-            const float a = __int_as_float(e.y);
+        for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
+            int2 nxt[PL];
 #pragma unroll
-            for (int v = 0; v < V; ++v)
-                if (colok[v]) fma4(a, __ldg(b + v * G), acc[v]);
+            for (int p = 0; p < PL; ++p) {
+                const int32_t o = b0 + BATCH + p * G + gl;
+                nxt[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
+            }
+#pragma unroll
+            for (int q0 = 0; q0 < BATCH; q0 += U) {
+                int32_t col[U];
+                float a[U];
+                bool ok[U];
+#pragma unroll
+                for (int w = 0; w < U; ++w) {
+                    const int qq = q0 + w;
+                    const int src = g * G + (qq % G);
+                    col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
+                    a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
+                    ok[w] = b0 + qq < len;
+                }
+                float4 x[U][V];
+#pragma unroll
+                for (int w = 0; w < U; ++w) {
+                    const float4 *b = B4 + (size_t)col[w] * K4 + col0;
+#pragma unroll
+                    for (int v = 0; v < V; ++v)
+                        x[w][v] = (ok[w] && colok[v]) ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+#pragma unroll
+                for (int w = 0; w < U; ++w)
+#pragma unroll
+                    for (int v = 0; v < V; ++v)
+                        if (ok[w]) fma4(a[w], x[w][v], acc[v]);
+            }
+#pragma unroll
+            for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
         }
         if (dst >= 0) {                                    // a whole row: C[perm[p]]
 #pragma unroll
@@ -114,8 +201,8 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ 
                     if (colok[v]) P4[slot * K4 + col0 + v * G] = acc[v];
             }
         }
-        if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
-        t = __shfl_sync(0xffffffffu, tk, 0);
+        t = t_next;
+        u = u_next;
     }
 }
 
@@ -293,17 +380,19 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
 using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
                             unsigned int *);
 
-template <int V, bool MASK>
+template <int V, bool MASK, int SCHED>
 SpmmKernel pick_g(int G) {
     switch (G) {
-        case 1: return k_spmm<V, 1, MASK>;
-        case 2: return k_spmm<V, 2, MASK>;
-        case 4: return k_spmm<V, 4, MASK>;
-        case 8: return k_spmm<V, 8, MASK>;
-        case 16: return k_spmm<V, 16, MASK>;
-        default: return k_spmm<V, 32, MASK>;
+        case 1: return k_spmm<V, 1, MASK, SCHED>;
+        case 2: return k_spmm<V, 2, MASK, SCHED>;
+        case 4: return k_spmm<V, 4, MASK, SCHED>;
+        case 8: return k_spmm<V, 8, MASK, SCHED>;
+        case 16: return k_spmm<V, 16, MASK, SCHED>;
+        default: return k_spmm<V, 32, MASK, SCHED>;
     }
 }
+template <int V, bool MASK>
+SpmmKernel pick_gs(int G, int sched) { return sched ? pick_g<V, MASK, 1>(G) : pick_g<V, MASK, 0>(G); }
 
 struct Config {
     SpmmKernel kern;
@@ -311,20 +400,20 @@ struct Config {
 };
 
 // exact fit 4*V*G == K with V in {4,3,2,1}, G a power of two <= 32; else V=4 with a masked tail
-Config choose(int32_t K4) {
+Config choose(int32_t K4, int sched) {
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
         int G = K4 / V;
         if (G >= 1 && G <= 32 && (G & (G - 1)) == 0) {
-            SpmmKernel k = V == 4 ? pick_g<4, false>(G) : V == 3 ? pick_g<3, false>(G) : V == 2 ? pick_g<2, false>(G)
-                                                                                            : pick_g<1, false>(G);
+            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched) : V == 3 ? pick_gs<3, false>(G, sched)
+                         : V == 2 ? pick_gs<2, false>(G, sched) : pick_gs<1, false>(G, sched);
             return {k, V, G, 1};
         }
     }
     int G = 1;
     while (G < 32 && 4 * G < K4) G <<= 1;
     int tiles = (int)ceil_div(K4, 4 * G);
-    return {pick_g<4, true>(G), 4, G, tiles};
+    return {pick_gs<4, true>(G, sched), 4, G, tiles};
 }
 
 }  // namespace
@@ -334,7 +423,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
-    const Config cfg = choose(K4);
+    static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 1; }();
+    const Config cfg = choose(K4, sched);
     const int32_t rpw = 32 / cfg.G;
     if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
     const Schedule &S = h->sched;

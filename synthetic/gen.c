@@ -12,11 +12,9 @@
  * count or scheduling.  Output CSR: rowidx int64[M+1], colidx int32[nnz] strictly
  * increasing per row, value float32[nnz].
  *
- * Memory protocol: every generator is called twice through the Python wrapper --
- * a "plan" call fills the sizes, then the caller allocates and a "fill" call
- * writes.  To avoid running the (expensive) draw twice, generators build the
- * CSR in a malloc'd staging buffer kept in a small registry keyed by a handle;
- * synth_take() copies it out and frees it.
+ * Memory protocol: a generator builds the CSR in malloc'd staging buffers and
+ * returns an opaque pointer; synth_sizes() reports M, N, nnz so the caller can
+ * allocate, and synth_take() copies the arrays out and frees the staging.
  */
 #include <stdint.h>
 #include <stdlib.h>
