@@ -184,16 +184,49 @@ def run_reference(args):
     }))
 
 
+def shard_inputs(torch, dist, a_full, world, rank, dev, pkg):
+    """Rank 0 holds the generated matrix; every rank gets its nnz-balanced row shard as CUDA tensors
+    (NCCL send/recv for N>1).  Returns (M_r, lo, rowidx, colidx, value) with rowidx rebased to 0."""
+    if rank == 0:
+        bounds = pkg.spmm_partition_by_nnz(a_full.rowidx, world)
+        meta = torch.tensor([[int(bounds[r + 1] - bounds[r]), int(a_full.rowidx[bounds[r + 1]] - a_full.rowidx[bounds[r]]),
+                              int(bounds[r])] for r in range(world)], dtype=torch.int64, device=dev)
+    else:
+        meta = torch.empty((world, 3), dtype=torch.int64, device=dev)
+    if world > 1:
+        dist.broadcast(meta, src=0)
+    parts = None
+    if rank == 0:
+        parts = []
+        for r in range(world):
+            lo, hi = int(bounds[r]), int(bounds[r + 1])
+            r0, r1 = int(a_full.rowidx[lo]), int(a_full.rowidx[hi])
+            parts.append((torch.from_numpy(a_full.rowidx[lo:hi + 1] - r0), torch.from_numpy(a_full.colidx[r0:r1]),
+                          torch.from_numpy(a_full.value[r0:r1])))
+        for r in range(1, world):
+            for t in parts[r]:
+                dist.send(t.to(dev), dst=r)
+        mine = tuple(t.to(dev) for t in parts[0])
+    else:
+        Mr, nnzr = int(meta[rank, 0]), int(meta[rank, 1])
+        mine = (torch.empty(Mr + 1, dtype=torch.int64, device=dev), torch.empty(nnzr, dtype=torch.int32, device=dev),
+                torch.empty(nnzr, dtype=torch.float32, device=dev))
+        for t in mine:
+            dist.recv(t, src=0)
+    return int(meta[rank, 0]), int(meta[rank, 2]), mine, meta
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="c5", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--policies", default=",".join(HOT))
     ap.add_argument("--window", type=int, default=1024)
-    ap.add_argument("--policy-steps", type=int, default=10, help="timed steps per policy for the exhaustive selection")
+    ap.add_argument("--policy-steps", type=int, default=5, help="timed steps per policy for the exhaustive selection")
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cusparse", action="store_true")
@@ -221,41 +254,45 @@ def main():
     bseed = (cfg["gen"][3] if cfg["gen"][0] == "rmat" else cfg["gen"][2]) + 1
 
     t0 = time.perf_counter()
-    a_full = make_matrix(cfg)
+    a_full = make_matrix(cfg) if rank == 0 else None
     gen_s = time.perf_counter() - t0
-    # row shard (rank r owns original rows [lo, hi) with about nnz/P non-zeros)
-    bounds = pkg.spmm_partition_by_nnz(a_full.rowidx, world)
-    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
-    r0 = a_full.rowidx[lo]
-    a = syn.CSR(hi - lo, a_full.N, a_full.rowidx[lo:hi + 1] - r0, a_full.colidx[r0:a_full.rowidx[hi]],
-                a_full.value[r0:a_full.rowidx[hi]], a_full.name)
-    alg_bytes, ncols = algorithmic_bytes(a, K)
-    flops = 2.0 * a.nnz * K
-    total_flops = 2.0 * a_full.nnz * K
+    Mr, lo, (rowidx_d, colidx_d, value_d), meta = shard_inputs(torch, dist, a_full, world, rank, dev, pkg)
+    N = a_full.N if rank == 0 else None
+    nN = torch.tensor([N or 0], dtype=torch.int64, device=dev)
+    if world > 1:
+        dist.broadcast(nN, src=0)
+    N = int(nN.item())
+    nnz_r = int(colidx_d.numel())
+    nnz_total = int(meta[:, 1].sum().item())
+    seen = torch.zeros(N, dtype=torch.bool, device=dev)
+    seen[colidx_d.long()] = True
+    ncols = int(seen.sum().item())
+    del seen
+    alg_bytes = 4 * (Mr + 1) + 8 * nnz_r + 4 * K * ncols + 4 * Mr * K   # north star, this rank's shard
+    flops = 2.0 * nnz_r * K
+    total_flops = 2.0 * nnz_total * K
 
     # B: drawn on rank 0 (host), broadcast over NCCL to the other ranks (outside the timed region)
-    if rank == 0:
-        B_host = torch.from_numpy(syn.dense(a.N, K, bseed))
-        Bd = B_host.to(dev)
-    else:
-        B_host = None
-        Bd = torch.empty((a.N, K), dtype=torch.float32, device=dev)
+    B_host = torch.from_numpy(syn.dense(N, K, bseed)) if rank == 0 else None
+    Bd = B_host.to(dev) if rank == 0 else torch.empty((N, K), dtype=torch.float32, device=dev)
     if world > 1:
         dist.broadcast(Bd, src=0)
-        if B_host is None:
-            B_host = Bd.cpu()
-    Cd = torch.empty((a.M, K), dtype=torch.float32, device=dev)
+    Cd = torch.empty((Mr, K), dtype=torch.float32, device=dev)
     flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
 
     def flush():
         flush_buf.fill_(1.0)
 
     pkg.use_torch_allocator(True)
-    h = pkg.SpMM.from_csr(a)
+    h = pkg.SpMM(Mr, N, rowidx_d, colidx_d, value_d)
     torch.cuda.synchronize()
     feat_t0 = time.perf_counter()
     feats = h.features()
     features_ms = 1e3 * (time.perf_counter() - feat_t0)
+    a_host = None
+    if rank == 0 and not args.no_ceiling:
+        r0, r1 = int(a_full.rowidx[0]), int(a_full.rowidx[Mr])
+        a_host = syn.CSR(Mr, N, a_full.rowidx[:Mr + 1] - r0, a_full.colidx[r0:r1], a_full.value[r0:r1])
 
     # ---- exhaustive per-policy timing (a10) ----
     pol_res = {}
@@ -270,11 +307,11 @@ def main():
         ms = statistics.median(ts)
         pol_res[pol] = {"ms": ms, "gflops": flops / ms / 1e6, "build_ms": build_ms, "launches": h.last_run_launches(),
                         "info": h.info()}
-        if not args.no_ceiling and rank == 0:
-            # L2-capacity ceiling: B-row misses of an LRU of L2-size in this order
+        if a_host is not None:
+            # L2-capacity ceiling: B-row misses of an LRU of L2 size in this order
             import tools
             cap = int(torch.cuda.get_device_properties(dev).L2_cache_size // (4 * K))
-            miss = tools.lru_misses(a, h.perm(), cap)
+            miss = tools.lru_misses(a_host, h.perm(), cap)
             traffic = alg_bytes - 4 * K * ncols + 4 * K * miss
             pol_res[pol]["lru_model"] = {"l2_rows": cap, "b_row_misses": miss, "model_bytes": traffic,
                                          "ceiling_frac": alg_bytes / traffic}
@@ -286,7 +323,7 @@ def main():
     best = names[int(torch.argmin(tvec))]
     h.permute(best, window=args.window)
 
-    # ---- the timed region: K steps of the selected policy ----
+    # ---- the timed region: `steps` steps of the selected policy ----
     for _ in range(args.warmup):
         h.run(Bd, Cd)
     torch.cuda.synchronize()
@@ -309,15 +346,30 @@ def main():
     peak, peak_src = peaks()
     achieved = alg_bytes / (statistics.mean(ts) * 1e-3) / 1e9
 
-    # ---- e2e through the public API with host buffers (H2D of B, SpMM, D2H of C per step) ----
-    Bp = B_host.pin_memory()
-    Cp = torch.empty((a.M, K), dtype=torch.float32).pin_memory()
-    h.run_host(Bp, Cp)
+    # ---- e2e through the public API with host buffers ----
+    # N=1: spmm_run_host (H2D of B, SpMM, D2H of C).  N>1: rank 0 H2D of B, NCCL broadcast, SpMM on every
+    # shard, D2H of every C shard; max over ranks.
+    Cp = torch.empty((Mr, K), dtype=torch.float32).pin_memory()
+    Bp = B_host.pin_memory() if rank == 0 else None
+
+    def e2e_step():
+        if world == 1:
+            h.run_host(Bp, Cp)
+        else:
+            if rank == 0:
+                Bd.copy_(Bp, non_blocking=True)
+            dist.broadcast(Bd, src=0)
+            h.run(Bd, Cd)
+            Cp.copy_(Cd, non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+    e2e_step()
     e2e_ts = []
-    for _ in range(max(3, min(args.steps, 10))):
+    for _ in range(max(3, args.e2e_steps)):
+        if world > 1:
+            dist.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        h.run_host(Bp, Cp)
+        e2e_step()
         e1.record(stream)
         e1.synchronize()
         e2e_ts.append(e0.elapsed_time(e1))
@@ -325,21 +377,22 @@ def main():
     if world > 1:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e = {"value": total_flops / float(e2e_t.item()) / 1e6, "unit": "GFLOP/s",
-           "h2d_bytes_per_step": int(Bp.numel() * 4), "d2h_bytes_per_step": int(Cp.numel() * 4),
-           "ms_per_step": float(e2e_t.item())}
+           "h2d_bytes_per_step": int(N * K * 4), "d2h_bytes_per_step": int(int(meta[:, 0].sum().item()) * K * 4),
+           "ms_per_step": float(e2e_t.item()),
+           "path": "spmm_run_host" if world == 1 else "H2D(B) on rank 0 + NCCL broadcast + spmm_run + D2H(C shards)"}
 
     # ---- cuSPARSE comparator (torch.sparse CSR @ dense -> cusparseSpMM), same inputs, same flush ----
     cus = None
-    if not args.no_cusparse:
+    if not args.no_cusparse and rank == 0:
         try:
-            A_t = torch.sparse_csr_tensor(torch.from_numpy(a.rowidx), torch.from_numpy(a.colidx.astype(np.int64)),
-                                          torch.from_numpy(a.value), size=(a.M, a.N)).to(dev)
+            A_t = torch.sparse_csr_tensor(rowidx_d, colidx_d.long(), value_d, size=(Mr, N))
             for _ in range(3):
                 A_t @ Bd
             cts = time_runs(torch, lambda: A_t @ Bd, max(3, args.policy_steps), flush, stream)
             cms = statistics.median(cts)
             cus = {"ms": cms, "gflops": flops / cms / 1e6, "speedup_best_vs_cusparse": cms / pol_res[best]["ms"],
-                   "via": "torch.sparse_csr @ dense (cusparseSpMM, default algorithm)"}
+                   "speedup_identity_vs_cusparse": cms / pol_res["identity"]["ms"] if "identity" in pol_res else None,
+                   "via": "torch.sparse_csr @ dense (cusparseSpMM, default algorithm), rank 0 shard"}
             del A_t
         except Exception as e:  # noqa: BLE001
             cus = {"error": str(e)[:200]}
@@ -366,13 +419,14 @@ def main():
         "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": cfg["desc"], "M": a_full.M, "N": a_full.N, "nnz": a_full.nnz, "K": K,
+        "config": {"workload": cfg["desc"], "M": int(meta[:, 0].sum().item()), "N": N, "nnz": nnz_total, "K": K,
                    "policy": best, "window": args.window, "parallelism": f"rows sharded by nnz over {world} GPU(s)",
                    "l2": "256 MiB scratch written between timed steps (L2 flush); B, C also > L2",
                    "selection": "exhaustive timing over " + ",".join(pol_res)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "algorithmic_bytes_per_launch": alg_bytes, "distinct_columns": ncols,
-                     "peak_source": peak_src, "kernel": "k_spmm (+k_combine for split rows), per spmm_run"},
+                     "peak_source": peak_src,
+                     "kernel": "one spmm_run = k_zero_rows + k_spmm + k_combine (rank 0 shard), CUDA events"},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,

@@ -86,7 +86,7 @@ __device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *g
 }
 
 template <int V, int G, bool MASK, int SCHED>
-__global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
+__global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter) {
@@ -153,28 +153,38 @@ __global__ void __launch_bounds__(SPMM_THREADS) k_spmm(const int4 *__restrict__ 
             for (int q0 = 0; q0 < BATCH; q0 += U) {
                 int32_t col[U];
                 float a[U];
-                bool ok[U];
 #pragma unroll
                 for (int w = 0; w < U; ++w) {
                     const int qq = q0 + w;
                     const int src = g * G + (qq % G);
                     col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
                     a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
-                    ok[w] = b0 + qq < len;
                 }
-                float4 x[U][V];
+                const int32_t rem = len - (b0 + q0);    // nnz left for this group
+                if (rem >= U) {                          // full step: U*V independent B loads in flight
+                    float4 x[U][V];
 #pragma unroll
-                for (int w = 0; w < U; ++w) {
-                    const float4 *b = B4 + (size_t)col[w] * K4 + col0;
+                    for (int w = 0; w < U; ++w) {
+                        const float4 *b = B4 + (size_t)col[w] * K4 + col0;
 #pragma unroll
-                    for (int v = 0; v < V; ++v)
-                        x[w][v] = (ok[w] && colok[v]) ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
+                        for (int v = 0; v < V; ++v)
+                            x[w][v] = colok[v] ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    }
+#pragma unroll
+                    for (int w = 0; w < U; ++w)
+#pragma unroll
+                        for (int v = 0; v < V; ++v) fma4(a[w], x[w][v], acc[v]);
+                } else if (rem > 0) {                    // the group's tail
+#pragma unroll
+                    for (int w = 0; w < U - 1; ++w) {
+                        if (w < rem) {
+                            const float4 *b = B4 + (size_t)col[w] * K4 + col0;
+#pragma unroll
+                            for (int v = 0; v < V; ++v)
+                                if (colok[v]) fma4(a[w], __ldg(b + v * G), acc[v]);
+                        }
+                    }
                 }
-#pragma unroll
-                for (int w = 0; w < U; ++w)
-#pragma unroll
-                    for (int v = 0; v < V; ++v)
-                        if (ok[w]) fma4(a[w], x[w][v], acc[v]);
             }
 #pragma unroll
             for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
