@@ -345,6 +345,17 @@ def main():
     value = total_flops / ms_step / 1e6   # GFLOP/s, whole job
     peak, peak_src = peaks()
     achieved = alg_bytes / (statistics.mean(ts) * 1e-3) / 1e9
+    l2 = None
+    if rank == 0:
+        try:   # second ceiling: every nnz pulls a 4K-byte B row through L2 unless it hits in L1
+            import tools
+            l2_bw = tools.l2_read_bandwidth() / 1e9
+            l2_bytes = 4.0 * K * nnz_r
+            l2 = {"read_peak_gbs": l2_bw, "b_row_bytes_per_launch": l2_bytes,
+                  "ceiling_frac_without_l1_reuse": (alg_bytes / peak) / (l2_bytes / l2_bw),
+                  "how": "tools/l2probe.cu: float4 __ldcg over a 64 MiB L2-resident buffer, CUDA events"}
+        except Exception as e:  # noqa: BLE001
+            l2 = {"error": str(e)[:200]}
 
     # ---- e2e through the public API with host buffers ----
     # N=1: spmm_run_host (H2D of B, SpMM, D2H of C).  N>1: rank 0 H2D of B, NCCL broadcast, SpMM on every
@@ -425,7 +436,7 @@ def main():
                    "selection": "exhaustive timing over " + ",".join(pol_res)},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "algorithmic_bytes_per_launch": alg_bytes, "distinct_columns": ncols,
-                     "peak_source": peak_src,
+                     "peak_source": peak_src, "l2": l2,
                      "kernel": "one spmm_run = k_zero_rows + k_spmm + k_combine (rank 0 shard), CUDA events"},
         "cpu_baseline": cpu,
         "e2e": e2e,

@@ -409,8 +409,19 @@ struct Config {
     int V, G, tiles;
 };
 
-// exact fit 4*V*G == K with V in {4,3,2,1}, G a power of two <= 32; else V=4 with a masked tail
+// Exact fit 4*V*G == K with V in {4,3,2,1} and G a power of two <= 32, preferring G >= 8 so that one
+// vector load of a group covers whole 128-byte lines (G*16 B >= 128 B: an L1 wavefront per line, measured
+// to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
 Config choose(int32_t K4, int sched) {
+    for (int V = 4; V >= 1; --V) {
+        if (K4 % V) continue;
+        int G = K4 / V;
+        if (G >= 8 && G <= 32 && (G & (G - 1)) == 0) {
+            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched) : V == 3 ? pick_gs<3, false>(G, sched)
+                         : V == 2 ? pick_gs<2, false>(G, sched) : pick_gs<1, false>(G, sched);
+            return {k, V, G, 1};
+        }
+    }
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
         int G = K4 / V;
@@ -433,7 +444,7 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
-    static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 1; }();
+    static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 0; }();
     const Config cfg = choose(K4, sched);
     const int32_t rpw = 32 / cfg.G;
     if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));

@@ -15,3 +15,6 @@ for cp in $PROFILES; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm -s 1 -c 1 -f -o gpurun_out/prof_${c}_$pol \
      python scripts/profile_spmm.py --config $c --policy $pol --runs 2 > gpurun_out/prof_${c}_$pol.log 2>&1; echo "prof $c $pol rc=$?"
 done
+if [ -n "$CORPUS" ]; then
+  timeout 3000 python scripts/corpus.py $CORPUS --out gpurun_out/corpus.jsonl > gpurun_out/corpus.log 2>&1; echo "corpus rc=$?"; tail -3 gpurun_out/corpus.log
+fi

@@ -10,11 +10,27 @@ _LIB = os.path.join(_HERE, "liblru.so")
 _lib = None
 
 
+_PROBE = os.path.join(_HERE, "libl2probe.so")
+
+
 def build():
     src = os.path.join(_HERE, "lru_model.c")
     if not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(src):
         subprocess.check_call(["gcc", "-O3", "-shared", "-fPIC", src, "-o", _LIB])
+    psrc = os.path.join(_HERE, "l2probe.cu")
+    if not os.path.exists(_PROBE) or os.path.getmtime(_PROBE) < os.path.getmtime(psrc):
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
+                               "-shared", "-Xcompiler", "-fPIC", psrc, "-o", _PROBE])
     return _LIB
+
+
+def l2_read_bandwidth(bytes_=64 << 20, reps=50):
+    """Achievable L2->SM read bandwidth (bytes/s) measured on the current GPU (buffer < L2)."""
+    build()
+    lib = ctypes.CDLL(_PROBE)
+    lib.l2probe_read_bw.restype = ctypes.c_double
+    lib.l2probe_read_bw.argtypes = [ctypes.c_int64, ctypes.c_int]
+    return float(lib.l2probe_read_bw(int(bytes_), int(reps)))
 
 
 def lru_misses(csr, order, cap_rows):

@@ -1,0 +1,46 @@
+// tools/l2probe.cu -- measurement helper (not the method): achievable L2->SM read bandwidth on this GPU.
+// Every warp streams float4 loads over an L2-resident buffer (size < L2) `reps` times; the sum is
+// written out so the loads are not dead.  Returns bytes/second via CUDA events.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+__global__ void __launch_bounds__(256) k_l2read(const float4 *__restrict__ buf, int64_t n4, int reps, float *out) {
+    float acc = 0.f;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int r = 0; r < reps; ++r) {
+        for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride * 4) {
+            float4 a = __ldcg(buf + i);
+            float4 b = i + stride < n4 ? __ldcg(buf + i + stride) : make_float4(0, 0, 0, 0);
+            float4 c = i + 2 * stride < n4 ? __ldcg(buf + i + 2 * stride) : make_float4(0, 0, 0, 0);
+            float4 d = i + 3 * stride < n4 ? __ldcg(buf + i + 3 * stride) : make_float4(0, 0, 0, 0);
+            acc += a.x + a.y + a.z + a.w + b.x + b.y + b.z + b.w + c.x + c.y + c.z + c.w + d.x + d.y + d.z + d.w;
+        }
+    }
+    out[(int64_t)blockIdx.x * blockDim.x + threadIdx.x] = acc;
+}
+
+extern "C" double l2probe_read_bw(int64_t bytes, int reps) {
+    int sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    float4 *buf = nullptr;
+    float *out = nullptr;
+    const int blocks = sms * 8, threads = 256;
+    if (cudaMalloc(&buf, bytes) != cudaSuccess) return -1.0;
+    cudaMalloc(&out, (size_t)blocks * threads * sizeof(float));
+    cudaMemset(buf, 0, bytes);
+    const int64_t n4 = bytes / 16;
+    k_l2read<<<blocks, threads>>>(buf, n4, 2, out);   // warm L2
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    cudaEventRecord(e0);
+    k_l2read<<<blocks, threads>>>(buf, n4, reps, out);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    cudaFree(buf);
+    cudaFree(out);
+    return (double)bytes * reps / (ms * 1e-3);
+}
