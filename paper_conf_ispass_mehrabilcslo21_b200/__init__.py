@@ -263,6 +263,26 @@ def spmm_predict(features, weights, n_policies):
     return int(pol.value), times
 
 
+PREDICTOR_POLICIES = HOT_PATH_POLICIES          # classes of the bundled predictor (reading A20)
+PAPER4_POLICIES = ["identity", "dcsr", "lpt", "warp_aware"]   # the paper's four classes
+
+
+def predictor_weights(K: int, paper_classes: bool = False) -> np.ndarray:
+    """Bundled MLP weights (spmm_predict layout) trained on the C4 corpus for the nearest trained K."""
+    d = os.path.join(_HERE, "predictor4" if paper_classes else "predictor")
+    ks = sorted(int(f[5:-4]) for f in os.listdir(d) if f.startswith("mlp_K") and f.endswith(".npy"))
+    k = min(ks, key=lambda x: (abs(np.log2(x) - np.log2(K)), x))
+    return np.load(os.path.join(d, f"mlp_K{k}.npy"))
+
+
+def select_policy(h: "SpMM", K: int, paper_classes: bool = False) -> str:
+    """a10 predicted selection: features of the original order on the GPU (spmm_features), MLP inference
+    in the library (spmm_predict), argmin of the predicted times."""
+    classes = PAPER4_POLICIES if paper_classes else PREDICTOR_POLICIES
+    pol, _ = spmm_predict(h.features(current_order=False), predictor_weights(K, paper_classes), len(classes))
+    return classes[pol]
+
+
 def spmm_partition_by_nnz(rowidx, P: int) -> np.ndarray:
     r = np.ascontiguousarray(rowidx, dtype=np.int64)
     b = np.empty(P + 1, dtype=np.int64)

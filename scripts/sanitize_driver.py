@@ -1,0 +1,27 @@
+"""Small pass over every entry point and policy (for compute-sanitizer)."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synthetic as syn  # noqa: E402
+import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
+
+a = syn.rmat(12, 12, 1000, "natural")
+h = pkg.SpMM.from_csr(a)
+h.features()
+for pol in pkg.POLICIES:
+    for K in (32, 64, 128, 36):
+        h.permute(pol, window=0 if pol not in ("hybrid_1",) else 256, split_nnz=64)
+        B = torch.from_numpy(syn.dense(a.N, K, 1)).cuda()
+        C = h.run(B)
+    h.features(current_order=True)
+torch.cuda.synchronize()
+h2 = pkg.SpMM.from_csr(syn.blockcluster(3000, 5000, 32, 4, 12, 3))
+h2.permute("hybrid_2_2", window=512, preorder=1, seed=3)
+h2.run(torch.zeros((5000, 64), device="cuda"))
+torch.cuda.synchronize()
+print("sanitize driver done")

@@ -81,3 +81,21 @@ def test_no_cpu_fallback_in_product():
                 src = open(os.path.join(dp, f)).read()
                 for bad in ("import oracle", "from oracle", "liboracle", '#include "../../oracle', "oracle/"):
                     assert bad not in src, (f, bad)
+
+
+def test_bundled_predictor_matches_oracle_forward():
+    """The bundled weights run through the library's C inference (spmm_predict) give the same argmin and
+    times as the oracle's float64 forward, on the committed corpus features (profiles/corpus_r1.jsonl)."""
+    import json
+    recs = [json.loads(l) for l in open(os.path.join(ROOT, "profiles", "corpus_r1.jsonl"))][:60]
+    for paper in (False, True):
+        P = len(pkg.PAPER4_POLICIES if paper else pkg.PREDICTOR_POLICIES)
+        for K in (32, 64, 128, 256):
+            w = pkg.predictor_weights(K, paper)
+            assert len(w) == 48 + 64 * 24 + 64 + 32 * 64 + 32 + 33 * P
+            for r in recs:
+                f = np.array(r["features"])
+                pol, t = pkg.spmm_predict(f, w, P)
+                best, ref = oracle.mlp_forward(f, w, P)
+                assert pol == best
+                np.testing.assert_allclose(t, ref, rtol=1e-9, atol=1e-9)
