@@ -10,12 +10,12 @@ import torch  # noqa: E402
 import synthetic as syn  # noqa: E402
 import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
 
-a = syn.rmat(12, 12, 1000, "natural")
+a = syn.rmat(11, 10, 1000, "natural")
 h = pkg.SpMM.from_csr(a)
 h.features()
 for pol in pkg.POLICIES:
-    for K in (32, 64, 128, 36):
-        h.permute(pol, window=0 if pol not in ("hybrid_1",) else 256, split_nnz=64)
+    h.permute(pol, window=256, split_nnz=64)
+    for K in (32, 128, 36):
         B = torch.from_numpy(syn.dense(a.N, K, 1)).cuda()
         C = h.run(B)
     h.features(current_order=True)
