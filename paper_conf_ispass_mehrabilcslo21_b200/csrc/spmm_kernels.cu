@@ -38,7 +38,36 @@ __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
     acc.x = lo.x; acc.y = lo.y; acc.z = hi.x; acc.w = hi.y;
 }
 
+// L2 cache-policy loads (VAR & 1): B rows are the reused operand -> L2::evict_last; the streamed
+// (col, val) pairs -> L2::evict_first and no L1 allocation.
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+template <bool HINT>
+__device__ __forceinline__ float4 ld_b(const float4 *ptr, uint64_t pol) {
+    if (!HINT) return __ldg(ptr);
+    float4 r;
+    asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(ptr), "l"(pol));
+    return r;
+}
+template <bool HINT>
+__device__ __forceinline__ int2 ld_cv(const int2 *ptr, uint64_t pol) {
+    if (!HINT) return __ldg(ptr);
+    int2 r;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(ptr), "l"(pol));
+    return r;
+}
+
 // V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
+// VAR bit 0: L2 cache-policy hints; bit 1: U = 4 nnz per step for V = 4.
 // Warp tasks are claimed dynamically (one atomicAdd per task on a per-column-tile counter), so the set
 // of tasks in flight stays a narrow window of the permuted order whatever the task costs: the order's
 // B-row locality survives into L2 and no warp is left with a long static tail.
@@ -85,14 +114,15 @@ __device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *g
     return __shfl_sync(0xffffffffu, task, 0);
 }
 
-template <int V, int G, bool MASK, int SCHED>
+template <int V, int G, bool MASK, int SCHED, int VAR>
 __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter) {
     constexpr int RPW = 32 / G;
     constexpr int CT4 = V * G;
-    constexpr int U = V >= 3 ? 2 : 4;            // nnz per inner step (B loads in flight per lane: U*V)
+    constexpr bool HINT = (VAR & 1) != 0;
+    constexpr int U = (V >= 3 && !(VAR & 2)) ? 2 : 4;   // nnz per inner step (B loads in flight per lane: U*V)
     constexpr int BATCH = G >= 8 ? G : 8;        // (col, val) pairs prefetched per group per batch
     constexpr int PL = BATCH / G;                // pairs held per lane
     const int lane = threadIdx.x & 31;
@@ -101,6 +131,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
     bool colok[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < K4);
+    const uint64_t pol_b = HINT ? policy_evict_last() : 0, pol_a = HINT ? policy_evict_first() : 0;
 
     __shared__ TaskQueue q;
     unsigned int tk = 0;
@@ -140,14 +171,14 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
 #pragma unroll
         for (int p = 0; p < PL; ++p) {
             const int32_t o = p * G + gl;
-            cur[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
+            cur[p] = o < len ? ld_cv<HINT>(cv + start + o, pol_a) : make_int2(0, 0);
         }
         for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
             int2 nxt[PL];
 #pragma unroll
             for (int p = 0; p < PL; ++p) {
                 const int32_t o = b0 + BATCH + p * G + gl;
-                nxt[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
+                nxt[p] = o < len ? ld_cv<HINT>(cv + start + o, pol_a) : make_int2(0, 0);
             }
 #pragma unroll
             for (int q0 = 0; q0 < BATCH; q0 += U) {
@@ -168,7 +199,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
                         const float4 *b = B4 + (size_t)col[w] * K4 + col0;
 #pragma unroll
                         for (int v = 0; v < V; ++v)
-                            x[w][v] = colok[v] ? __ldg(b + v * G) : make_float4(0.f, 0.f, 0.f, 0.f);
+                            x[w][v] = colok[v] ? ld_b<HINT>(b + v * G, pol_b) : make_float4(0.f, 0.f, 0.f, 0.f);
                     }
 #pragma unroll
                     for (int w = 0; w < U; ++w)
@@ -181,7 +212,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
                             const float4 *b = B4 + (size_t)col[w] * K4 + col0;
 #pragma unroll
                             for (int v = 0; v < V; ++v)
-                                if (colok[v]) fma4(a[w], __ldg(b + v * G), acc[v]);
+                                if (colok[v]) fma4(a[w], ld_b<HINT>(b + v * G, pol_b), acc[v]);
                         }
                     }
                 }
@@ -390,19 +421,29 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
 using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
                             unsigned int *);
 
-template <int V, bool MASK, int SCHED>
+template <int V, bool MASK, int SCHED, int VAR>
 SpmmKernel pick_g(int G) {
     switch (G) {
-        case 1: return k_spmm<V, 1, MASK, SCHED>;
-        case 2: return k_spmm<V, 2, MASK, SCHED>;
-        case 4: return k_spmm<V, 4, MASK, SCHED>;
-        case 8: return k_spmm<V, 8, MASK, SCHED>;
-        case 16: return k_spmm<V, 16, MASK, SCHED>;
-        default: return k_spmm<V, 32, MASK, SCHED>;
+        case 1: return k_spmm<V, 1, MASK, SCHED, VAR>;
+        case 2: return k_spmm<V, 2, MASK, SCHED, VAR>;
+        case 4: return k_spmm<V, 4, MASK, SCHED, VAR>;
+        case 8: return k_spmm<V, 8, MASK, SCHED, VAR>;
+        case 16: return k_spmm<V, 16, MASK, SCHED, VAR>;
+        default: return k_spmm<V, 32, MASK, SCHED, VAR>;
     }
 }
+// run-time knobs (tuning experiments; defaults are the measured best): SPMM_SCHED (0 per-warp claiming,
+// 1 CTA-contiguous queue), SPMM_VARIANT (bit 0 L2 cache hints, bit 1 U=4)
 template <int V, bool MASK>
-SpmmKernel pick_gs(int G, int sched) { return sched ? pick_g<V, MASK, 1>(G) : pick_g<V, MASK, 0>(G); }
+SpmmKernel pick_gs(int G, int sched, int var) {
+    if (sched) return pick_g<V, MASK, 1, 0>(G);
+    switch (var) {
+        case 1: return pick_g<V, MASK, 0, 1>(G);
+        case 2: return pick_g<V, MASK, 0, 2>(G);
+        case 3: return pick_g<V, MASK, 0, 3>(G);
+        default: return pick_g<V, MASK, 0, 0>(G);
+    }
+}
 
 struct Config {
     SpmmKernel kern;
@@ -412,13 +453,13 @@ struct Config {
 // Exact fit 4*V*G == K with V in {4,3,2,1} and G a power of two <= 32, preferring G >= 8 so that one
 // vector load of a group covers whole 128-byte lines (G*16 B >= 128 B: an L1 wavefront per line, measured
 // to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
-Config choose(int32_t K4, int sched) {
+Config choose(int32_t K4, int sched, int var) {
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
         int G = K4 / V;
         if (G >= 8 && G <= 32 && (G & (G - 1)) == 0) {
-            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched) : V == 3 ? pick_gs<3, false>(G, sched)
-                         : V == 2 ? pick_gs<2, false>(G, sched) : pick_gs<1, false>(G, sched);
+            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
+                         : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
             return {k, V, G, 1};
         }
     }
@@ -426,15 +467,15 @@ Config choose(int32_t K4, int sched) {
         if (K4 % V) continue;
         int G = K4 / V;
         if (G >= 1 && G <= 32 && (G & (G - 1)) == 0) {
-            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched) : V == 3 ? pick_gs<3, false>(G, sched)
-                         : V == 2 ? pick_gs<2, false>(G, sched) : pick_gs<1, false>(G, sched);
+            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
+                         : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
             return {k, V, G, 1};
         }
     }
     int G = 1;
     while (G < 32 && 4 * G < K4) G <<= 1;
     int tiles = (int)ceil_div(K4, 4 * G);
-    return {pick_gs<4, true>(G, sched), 4, G, tiles};
+    return {pick_gs<4, true>(G, sched, var), 4, G, tiles};
 }
 
 }  // namespace
@@ -445,7 +486,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
     static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 0; }();
-    const Config cfg = choose(K4, sched);
+    static const int var = [] { const char *e = getenv("SPMM_VARIANT"); return e ? atoi(e) : 0; }();
+    const Config cfg = choose(K4, sched, var);
     const int32_t rpw = 32 / cfg.G;
     if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
     const Schedule &S = h->sched;
