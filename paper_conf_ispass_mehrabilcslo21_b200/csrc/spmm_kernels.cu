@@ -247,6 +247,125 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
     }
 }
 
+// ---- kernel mode 2: panel-staged SpMM (schedule: panel.cu) --------------------------------------
+// One CTA (16 warps) per SM claims panels of consecutive permuted rows.  Per panel it first copies the
+// panel's staged B rows into shared memory with cp.async, then its warps claim the panel's work units
+// RPW at a time (shared-memory counter); a nnz whose column was staged (col < 0 in the rewritten cv)
+// reads its B row from shared memory, the others from global memory, through one generic load.  Same
+// per-row FMA order as the row-group kernel; chunks of long rows write partials (combined pairwise).
+constexpr int PS_THREADS = 512;
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+}
+
+template <int V, int G>
+__global__ void __launch_bounds__(PS_THREADS, 1) k_spmm_ps(const int4 *__restrict__ units,
+                                                           const int32_t *__restrict__ panel_unit_ptr,
+                                                           const int32_t *__restrict__ stage_ptr,
+                                                           const int32_t *__restrict__ staged_cols, int64_t n_panels,
+                                                           const int2 *__restrict__ cv, const float4 *__restrict__ B4,
+                                                           float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
+                                                           unsigned int *__restrict__ counter) {
+    extern __shared__ float4 sB[];
+    __shared__ unsigned int s_panel, s_next;
+    constexpr int RPW = 32 / G;
+    constexpr int U = V >= 3 ? 2 : 4;
+    constexpr int BATCH = G >= 8 ? G : 8;
+    constexpr int PL = BATCH / G;
+    const int lane = threadIdx.x & 31;
+    const int g = lane / G, gl = lane % G;
+    for (;;) {
+        if (threadIdx.x == 0) { s_panel = atomicAdd(counter, 1u); s_next = 0u; }
+        __syncthreads();
+        const unsigned int P = s_panel;
+        if (P >= n_panels) break;
+        const int32_t s0 = stage_ptr[P], ns = stage_ptr[P + 1] - s0;
+        for (int32_t i = threadIdx.x; i < ns * K4; i += PS_THREADS) {
+            const int32_t r = i / K4, c = i - r * K4;
+            cp_async16(sB + (size_t)r * K4 + c, B4 + (size_t)staged_cols[s0 + r] * K4 + c);
+        }
+        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+        __syncthreads();
+        const int32_t u0 = panel_unit_ptr[P], nu = panel_unit_ptr[P + 1] - u0;
+        for (;;) {
+            unsigned int kk = 0;
+            if (lane == 0) kk = atomicAdd(&s_next, (unsigned)RPW);
+            kk = __shfl_sync(0xffffffffu, kk, 0);
+            if ((int32_t)kk >= nu) break;
+            const int4 u = (int32_t)kk + g < nu ? __ldg(units + u0 + kk + g) : make_int4(0, 0, NOSTORE, 0);
+            const int32_t start = u.x, len = u.y, dst = u.z;
+            const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
+            float4 acc[V];
+#pragma unroll
+            for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+            int2 cur[PL];
+#pragma unroll
+            for (int p = 0; p < PL; ++p) {
+                const int32_t o = p * G + gl;
+                cur[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
+            }
+            for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
+                int2 nxt[PL];
+#pragma unroll
+                for (int p = 0; p < PL; ++p) {
+                    const int32_t o = b0 + BATCH + p * G + gl;
+                    nxt[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
+                }
+#pragma unroll
+                for (int q0 = 0; q0 < BATCH; q0 += U) {
+                    int32_t col[U];
+                    float a[U];
+#pragma unroll
+                    for (int w = 0; w < U; ++w) {
+                        const int qq = q0 + w;
+                        const int src = g * G + (qq % G);
+                        col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
+                        a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
+                    }
+                    const int32_t rem = len - (b0 + q0);
+                    if (rem >= U) {
+                        float4 x[U][V];
+#pragma unroll
+                        for (int w = 0; w < U; ++w) {
+                            const float4 *b = col[w] < 0 ? sB + (size_t)(col[w] & 0x7fffffff) * K4 + gl
+                                                         : B4 + (size_t)col[w] * K4 + gl;
+#pragma unroll
+                            for (int v = 0; v < V; ++v) x[w][v] = b[v * G];
+                        }
+#pragma unroll
+                        for (int w = 0; w < U; ++w)
+#pragma unroll
+                            for (int v = 0; v < V; ++v) fma4(a[w], x[w][v], acc[v]);
+                    } else if (rem > 0) {
+#pragma unroll
+                        for (int w = 0; w < U - 1; ++w) {
+                            if (w < rem) {
+                                const float4 *b = col[w] < 0 ? sB + (size_t)(col[w] & 0x7fffffff) * K4 + gl
+                                                             : B4 + (size_t)col[w] * K4 + gl;
+#pragma unroll
+                                for (int v = 0; v < V; ++v) fma4(a[w], b[v * G], acc[v]);
+                            }
+                        }
+                    }
+                }
+#pragma unroll
+                for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
+            }
+            if (dst >= 0) {
+#pragma unroll
+                for (int v = 0; v < V; ++v) __stcs(C4 + (size_t)dst * K4 + gl + v * G, acc[v]);
+            } else if (dst != NOSTORE) {
+                const int64_t slot = -(int64_t)dst - 1;
+#pragma unroll
+                for (int v = 0; v < V; ++v) P4[slot * K4 + gl + v * G] = acc[v];
+            }
+        }
+        __syncthreads();   // every warp is done with this panel before the next one is staged
+    }
+}
+
 // Pairwise (binary-counter) combine of a long row's chunk-group partials, fixed order -> deterministic;
 // rounding grows with log2(#groups).  One CTA per long row, thread per float4 column.
 __global__ void __launch_bounds__(128) k_combine(const float4 *__restrict__ P4, const int32_t *__restrict__ pslot_ptr,
@@ -445,6 +564,15 @@ SpmmKernel pick_gs(int G, int sched, int var) {
     }
 }
 
+using PsKernel = void (*)(const int4 *, const int32_t *, const int32_t *, const int32_t *, int64_t, const int2 *,
+                          const float4 *, float4 *, int32_t, float4 *, unsigned int *);
+PsKernel pick_ps(int V, int G) {
+    if (G == 8) return V == 4 ? k_spmm_ps<4, 8> : V == 3 ? k_spmm_ps<3, 8> : V == 2 ? k_spmm_ps<2, 8> : k_spmm_ps<1, 8>;
+    if (G == 16) return V == 4 ? k_spmm_ps<4, 16> : V == 3 ? k_spmm_ps<3, 16> : V == 2 ? k_spmm_ps<2, 16> : k_spmm_ps<1, 16>;
+    if (G == 32) return V == 4 ? k_spmm_ps<4, 32> : V == 3 ? k_spmm_ps<3, 32> : V == 2 ? k_spmm_ps<2, 32> : k_spmm_ps<1, 32>;
+    return nullptr;
+}
+
 struct Config {
     SpmmKernel kern;
     int V, G, tiles;
@@ -480,6 +608,47 @@ Config choose(int32_t K4, int sched, int var) {
 
 }  // namespace
 
+static spmm_status launch_ps(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int V, int G,
+                             int32_t *launches) {
+    const int32_t K4 = (int32_t)(K / 4);
+    static const int pr = [] { const char *e = getenv("SPMM_PANEL_ROWS"); return e ? atoi(e) : 256; }();
+    static const int smem_kb = [] { const char *e = getenv("SPMM_PS_SMEM_KB"); return e ? atoi(e) : 200; }();
+    const int32_t cap = (int32_t)std::max<int64_t>(1, ((int64_t)smem_kb * 1024) / (K * 4));
+    if (h->psched.K != K) SPMM_TRY(build_panel_schedule(h, K, pr, cap, s));
+    const PanelSchedule &S = h->psched;
+    float4 *C4 = reinterpret_cast<float4 *>(C);
+    float4 *P4 = nullptr;
+    if (S.n_pslots > 0) {
+        const size_t need = (size_t)S.n_pslots * K * sizeof(float);
+        if (h->partials.bytes < need) SPMM_TRY(h->partials.alloc(need, s));
+        P4 = h->partials.as<float4>();
+    }
+    if (S.n_empty > 0) {
+        k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4);
+        SPMM_CUDA(cudaGetLastError());
+        ++*launches;
+    }
+    if (S.n_units > 0) {
+        PsKernel kern = pick_ps(V, G);
+        const size_t smem = (size_t)cap * K * sizeof(float);
+        SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if (h->counters.bytes < sizeof(unsigned int)) SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
+        SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, sizeof(unsigned int), s));
+        kern<<<(unsigned)std::min<int64_t>(h->num_sms, S.n_panels), PS_THREADS, smem, s>>>(
+            S.units.as<int4>(), S.panel_unit_ptr.as<int32_t>(), S.stage_ptr.as<int32_t>(), S.staged_cols.as<int32_t>(),
+            S.n_panels, S.cv_ps.as<int2>(), reinterpret_cast<const float4 *>(B), C4, K4, P4,
+            h->counters.as<unsigned int>());
+        SPMM_CUDA(cudaGetLastError());
+        ++*launches;
+    }
+    if (S.n_long > 0) {
+        k_combine<<<(unsigned)S.n_long, 128, 0, s>>>(P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), C4, K4);
+        SPMM_CUDA(cudaGetLastError());
+        ++*launches;
+    }
+    return SPMM_OK;
+}
+
 spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches) {
     *launches = 0;
     const int64_t M = h->M;
@@ -488,6 +657,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 0; }();
     static const int var = [] { const char *e = getenv("SPMM_VARIANT"); return e ? atoi(e) : 0; }();
     const Config cfg = choose(K4, sched, var);
+    static const int kmode = [] { const char *e = getenv("SPMM_KERNEL"); return e ? atoi(e) : 1; }();
+    if (kmode == 2 && cfg.tiles == 1 && pick_ps(cfg.V, cfg.G) != nullptr) return launch_ps(h, B, K, C, s, cfg.V, cfg.G, launches);
     const int32_t rpw = 32 / cfg.G;
     if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
     const Schedule &S = h->sched;

@@ -273,3 +273,61 @@ def test_torch_allocator_and_streams():
         h.close()
     finally:
         pkg.use_torch_allocator(False)
+
+
+_SUBPROC = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import oracle, synthetic as syn, paper_conf_ispass_mehrabilcslo21_b200 as pkg
+a = syn.rmat(12, 10, 3, "natural", int_values=True)
+B = syn.dense(a.N, 128, 4, int_values=True)
+ref, _ = oracle.spmm(a, B)
+h = pkg.SpMM.from_csr(a)
+for K in (128, 64, 32, 256):
+    BK = np.ascontiguousarray(B[:, :K]) if K <= 128 else np.ascontiguousarray(np.tile(B, (1, 2)))
+    refK, _ = oracle.spmm(a, BK)
+    for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_1"):
+        h.permute(pol, split_nnz=32)
+        C = h.run(torch.from_numpy(BK).cuda()).cpu().numpy()
+        assert np.array_equal(C.astype(np.float64), refK), (K, pol)
+# real-valued tolerance + permutation invariance
+Bf = syn.dense(a.N, 128, 9)
+af = syn.rmat(12, 10, 3, "local")
+ref, bound = oracle.spmm(af, Bf)
+hf = pkg.SpMM.from_csr(af)
+first = None
+for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_2_1"):
+    hf.permute(pol)
+    C = hf.run(torch.from_numpy(Bf).cuda()).cpu().numpy()
+    assert np.all(np.abs(C - ref) <= 1e-5 * bound + 1e-6), pol
+    if first is None: first = C
+    assert np.array_equal(C.view(np.int32), first.view(np.int32)), pol
+print("OK")
+"""
+
+
+@pytest.mark.parametrize("env", [{"SPMM_SCHED": "1"}, {"SPMM_VARIANT": "1"}, {"SPMM_VARIANT": "2"},
+                                 {"SPMM_VARIANT": "3"}, {"SPMM_KERNEL": "2"},
+                                 {"SPMM_KERNEL": "2", "SPMM_PANEL_ROWS": "64", "SPMM_PS_SMEM_KB": "8"}])
+def test_kernel_variants_exact(env):
+    """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4) are exact on integer inputs."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _SUBPROC.format(root=root)], env={**os.environ, **env},
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "OK" in r.stdout, r.stderr[-2000:]
+
+
+def test_select_policy_runs():
+    a = syn.rmat(12, 8, 7, "local")
+    h = pkg.SpMM.from_csr(a)
+    for K in (32, 128):
+        pol = pkg.select_policy(h, K)
+        assert pol in pkg.PREDICTOR_POLICIES
+        pol4 = pkg.select_policy(h, K, paper_classes=True)
+        assert pol4 in pkg.PAPER4_POLICIES
+        h.permute(pol)
+        assert np.array_equal(h.perm(), oracle.permute(a, pol, window=1024))
+    h.close()
