@@ -10,7 +10,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libspmm_b200.so")
-SOURCES = ["api.cu", "primitives.cu", "permute.cu", "spmm_kernels.cu", "features.cu", "panel.cu"]
+SOURCES = ["api.cu", "primitives.cu", "permute.cu", "spmm_kernels.cu", "features.cu"]
 HEADERS = ["internal.cuh", os.path.join("..", "..", "include", "spmm.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",

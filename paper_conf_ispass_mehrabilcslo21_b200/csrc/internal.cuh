@@ -78,22 +78,6 @@ struct Schedule {
     DevBuf empty_dst;         // int32[n_empty]     C rows of empty rows (zero-filled)
 };
 
-// a7 panel-staged schedule (kernel mode 2) for one K: positions are cut into panels of `pr` consecutive
-// rows; the B rows of the columns a panel references most often (>= 2 times, up to `cap` rows that fit in
-// shared memory) are staged once per panel and read from shared memory by all of the panel's rows.
-struct PanelSchedule {
-    int64_t K = 0;            // 0 = not built
-    int32_t pr = 0, cap = 0;
-    int64_t n_panels = 0, n_units = 0, n_staged = 0, staged_nnz = 0;
-    DevBuf units;             // int4[n_units]: (start, len, dst, 0), dst >= 0 C row, < 0 partial slot
-    DevBuf panel_unit_ptr;    // int32[n_panels + 1]
-    DevBuf stage_ptr;         // int32[n_panels + 1]
-    DevBuf staged_cols;       // int32[n_staged]
-    DevBuf cv_ps;             // int2[nnz]: cv' with staged columns replaced by (slot | 0x80000000)
-    int64_t n_long = 0, n_pslots = 0, n_empty = 0;
-    DevBuf long_dst, pslot_ptr, empty_dst;
-};
-
 }  // namespace spmm
 
 struct spmm_ctx {
@@ -114,7 +98,6 @@ struct spmm_ctx {
     spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
     spmm::RowClasses rc;
     spmm::Schedule sched;
-    spmm::PanelSchedule psched;
     // run scratch (partials of split rows), grown on demand
     spmm::DevBuf partials;
     spmm::DevBuf counters;  // dynamic warp-task counters, one per column tile
@@ -138,7 +121,6 @@ spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s);
 spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24],
                              cudaStream_t s);
 spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches);
-spmm_status build_panel_schedule(spmm_ctx *h, int64_t K, int32_t pr, int32_t cap, cudaStream_t s);
 
 // signatures of the rows (sorted unique col/bw), used by chains and features
 struct Signatures {

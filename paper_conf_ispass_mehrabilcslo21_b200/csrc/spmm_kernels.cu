@@ -32,14 +32,49 @@ namespace {
 constexpr int SPMM_THREADS = 256;
 constexpr int32_t NOSTORE = INT_MIN;
 
+// ---- per-lane vectors: W = 4 floats (LDG.128) or W = 8 floats (sm_100 LDG.E.ENL2.256) ---------------
+struct float8 {
+    float4 lo, hi;
+};
+template <int W> struct VecT;
+template <> struct VecT<4> { using T = float4; };
+template <> struct VecT<8> { using T = float8; };
+
 __device__ __forceinline__ void fma4(float a, const float4 &b, float4 &acc) {
     float2 lo = __ffma2_rn(make_float2(a, a), make_float2(b.x, b.y), make_float2(acc.x, acc.y));
     float2 hi = __ffma2_rn(make_float2(a, a), make_float2(b.z, b.w), make_float2(acc.z, acc.w));
     acc.x = lo.x; acc.y = lo.y; acc.z = hi.x; acc.w = hi.y;
 }
+__device__ __forceinline__ void vfma(float a, const float4 &b, float4 &acc) { fma4(a, b, acc); }
+__device__ __forceinline__ void vfma(float a, const float8 &b, float8 &acc) {
+    fma4(a, b.lo, acc.lo);
+    fma4(a, b.hi, acc.hi);
+}
+__device__ __forceinline__ void vzero(float4 &a) { a = make_float4(0.f, 0.f, 0.f, 0.f); }
+__device__ __forceinline__ void vzero(float8 &a) { vzero(a.lo); vzero(a.hi); }
+__device__ __forceinline__ void xadd(float4 &a, int off) {
+    a.x += __shfl_xor_sync(0xffffffffu, a.x, off);
+    a.y += __shfl_xor_sync(0xffffffffu, a.y, off);
+    a.z += __shfl_xor_sync(0xffffffffu, a.z, off);
+    a.w += __shfl_xor_sync(0xffffffffu, a.w, off);
+}
+__device__ __forceinline__ void xadd(float8 &a, int off) { xadd(a.lo, off); xadd(a.hi, off); }
+__device__ __forceinline__ void vstore_cs(float4 *p, const float4 &v) { __stcs(p, v); }
+__device__ __forceinline__ void vstore_cs(float8 *p, const float8 &v) {
+    asm volatile("st.global.cs.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v.lo.x), "f"(v.lo.y),
+                 "f"(v.lo.z), "f"(v.lo.w), "f"(v.hi.x), "f"(v.hi.y), "f"(v.hi.z), "f"(v.hi.w) : "memory");
+}
+__device__ __forceinline__ void vstore(float4 *p, const float4 &v) { *p = v; }
+__device__ __forceinline__ void vstore(float8 *p, const float8 &v) {
+    asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v.lo.x), "f"(v.lo.y),
+                 "f"(v.lo.z), "f"(v.lo.w), "f"(v.hi.x), "f"(v.hi.y), "f"(v.hi.z), "f"(v.hi.w) : "memory");
+}
 
-// L2 cache-policy loads (VAR & 1): B rows are the reused operand -> L2::evict_last; the streamed
-// (col, val) pairs -> L2::evict_first and no L1 allocation.
+// Load flavours of the inner loop (LD template parameter; defaults are the measured best):
+//   LD 0: plain read-only loads (ld.global.nc) of (col, val) and of B rows;
+//   LD 1: L2 cache-policy hints: B rows, the reused operand -> L2::evict_last; the streamed (col, val)
+//         pairs -> L2::evict_first and no L1 allocation;
+//   LD 2: (col, val) pairs bypass L1 (L1::no_allocate), B rows plain (L1 keeps only B).
 __device__ __forceinline__ uint64_t policy_evict_last() {
     uint64_t p;
     asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
@@ -50,24 +85,142 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-template <bool HINT>
+#define SPMM_V4_OUT "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+#define SPMM_V8_OUT "=f"(r.lo.x), "=f"(r.lo.y), "=f"(r.lo.z), "=f"(r.lo.w), "=f"(r.hi.x), "=f"(r.hi.y), "=f"(r.hi.z), "=f"(r.hi.w)
+template <int LD>
 __device__ __forceinline__ float4 ld_b(const float4 *ptr, uint64_t pol) {
-    if (!HINT) return __ldg(ptr);
     float4 r;
-    asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-        : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(ptr), "l"(pol));
+    if (LD == 1) {
+        asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;" : SPMM_V4_OUT : "l"(ptr), "l"(pol));
+    } else {
+        r = __ldg(ptr);
+    }
     return r;
 }
-template <bool HINT>
+template <int LD>
+__device__ __forceinline__ float8 ld_b(const float8 *ptr, uint64_t pol) {
+    float8 r;
+    if (LD == 1) {
+        asm("ld.global.nc.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;" : SPMM_V8_OUT : "l"(ptr), "l"(pol));
+    } else {
+        asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];" : SPMM_V8_OUT : "l"(ptr));
+    }
+    return r;
+}
+#undef SPMM_V4_OUT
+#undef SPMM_V8_OUT
+template <int LD>
 __device__ __forceinline__ int2 ld_cv(const int2 *ptr, uint64_t pol) {
-    if (!HINT) return __ldg(ptr);
     int2 r;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(ptr), "l"(pol));
+    if (LD == 1) {
+        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(ptr), "l"(pol));
+    } else if (LD >= 2) {
+        asm("ld.global.nc.L1::no_allocate.v2.s32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(ptr));
+    } else {
+        r = __ldg(ptr);
+    }
     return r;
 }
 
+// One work unit per lane group: the G lanes of group g own the unit u = (start, len, dst) and the V vectors
+// (VT = W floats each) col0 + v*G of its C row (colok: inside K; indices in VT units, KV = K / W per row).
+// Per nnz the group broadcasts the (col, val) pair with two shuffles from a register batch prefetched one
+// batch ahead (coalesced 8-byte loads of the interleaved permuted CSR), issues V coalesced W*4-byte loads of
+// the B row (G*W*4 contiguous bytes per group and vector: whole 128-byte lines), then W*V/2 packed FFMA2
+// -- each accumulator is a sequential chain in ascending j, the order of the oracle's definition
+// (oracle.c c1).  U nnz per inner step: U*V independent B loads are issued before the first FMA.  The trip
+// count is warp-uniform (groups past their own length are predicated off), so the shuffles stay warp-wide.
+// Store: a whole row -> C[perm[p]] (streaming store); a chunk group of a long row -> the warp's groups
+// are reduced by a fixed xor butterfly and group 0 writes the partial.
+template <int V, int G, int U, int LD, class VT>
+__device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int gl, const int col0, const bool (&colok)[V],
+                                          const int2 *__restrict__ cv, const VT *__restrict__ BV,
+                                          VT *__restrict__ CV, const int32_t KV, VT *__restrict__ PV,
+                                          const uint64_t pol_b, const uint64_t pol_a) {
+    constexpr int BATCH = (G >= 8 ? G : 8) >= U ? (G >= 8 ? G : 8) : U;   // (col, val) pairs per group per batch
+    constexpr int PL = BATCH / G;                // pairs held per lane
+    const int32_t start = u.x, len = u.y, dst = u.z;
+    const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
+    VT acc[V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) vzero(acc[v]);
+    int2 cur[PL];
+#pragma unroll
+    for (int p = 0; p < PL; ++p) {
+        const int32_t o = p * G + gl;
+        cur[p] = o < len ? ld_cv<LD>(cv + start + o, pol_a) : make_int2(0, 0);
+    }
+    for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
+        int2 nxt[PL];
+#pragma unroll
+        for (int p = 0; p < PL; ++p) {
+            const int32_t o = b0 + BATCH + p * G + gl;
+            nxt[p] = o < len ? ld_cv<LD>(cv + start + o, pol_a) : make_int2(0, 0);
+        }
+#pragma unroll
+        for (int q0 = 0; q0 < BATCH; q0 += U) {
+            int32_t col[U];
+            float a[U];
+#pragma unroll
+            for (int w = 0; w < U; ++w) {
+                const int qq = q0 + w;
+                const int src = g * G + (qq % G);
+                col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
+                a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
+            }
+            const int32_t rem = len - (b0 + q0);    // nnz left for this group
+            if (rem >= U) {                          // full step: U*V independent B loads in flight
+                VT x[U][V];
+#pragma unroll
+                for (int w = 0; w < U; ++w) {
+                    const VT *b = BV + (size_t)col[w] * KV + col0;
+#pragma unroll
+                    for (int v = 0; v < V; ++v) {
+                        if (colok[v]) x[w][v] = ld_b<LD>(b + v * G, pol_b);
+                        else vzero(x[w][v]);
+                    }
+                }
+#pragma unroll
+                for (int w = 0; w < U; ++w)
+#pragma unroll
+                    for (int v = 0; v < V; ++v) vfma(a[w], x[w][v], acc[v]);
+            } else if (rem > 0) {                    // the group's tail
+#pragma unroll
+                for (int w = 0; w < U - 1; ++w) {
+                    if (w < rem) {
+                        const VT *b = BV + (size_t)col[w] * KV + col0;
+#pragma unroll
+                        for (int v = 0; v < V; ++v)
+                            if (colok[v]) vfma(a[w], ld_b<LD>(b + v * G, pol_b), acc[v]);
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
+    }
+    if (dst >= 0) {                                    // a whole row: C[perm[p]]
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+            if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[v]);
+    } else if (dst != NOSTORE) {                       // chunk group of a long row (warp-uniform)
+#pragma unroll
+        for (int off = G; off < 32; off <<= 1) {       // fixed butterfly: ((c0+c1)+(c2+c3))...
+#pragma unroll
+            for (int v = 0; v < V; ++v) xadd(acc[v], off);
+        }
+        if (g == 0) {
+            const int64_t slot = -(int64_t)dst - 1;
+#pragma unroll
+            for (int v = 0; v < V; ++v)
+                if (colok[v]) vstore(PV + slot * KV + col0 + v * G, acc[v]);
+        }
+    }
+}
+
+// Kernel mode 1 (default): row-group SpMM over the a7 warp-task list.
 // V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
-// VAR bit 0: L2 cache-policy hints; bit 1: U = 4 nnz per step for V = 4.
+// VAR bit 0: L2 cache-policy hints (LD 1); bit 1: U = 4 nnz per step for V = 4.
 // Warp tasks are claimed dynamically (one atomicAdd per task on a per-column-tile counter), so the set
 // of tasks in flight stays a narrow window of the permuted order whatever the task costs: the order's
 // B-row locality survives into L2 and no warp is left with a long static tail.
@@ -114,24 +267,24 @@ __device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *g
     return __shfl_sync(0xffffffffu, task, 0);
 }
 
-template <int V, int G, bool MASK, int SCHED, int VAR>
+template <int V, int G, bool MASK, int SCHED, int VAR, int W>
 __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter) {
+    using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
-    constexpr int CT4 = V * G;
-    constexpr bool HINT = (VAR & 1) != 0;
-    constexpr int U = (V >= 3 && !(VAR & 2)) ? 2 : 4;   // nnz per inner step (B loads in flight per lane: U*V)
-    constexpr int BATCH = G >= 8 ? G : 8;        // (col, val) pairs prefetched per group per batch
-    constexpr int PL = BATCH / G;                // pairs held per lane
+    constexpr int CTV = V * G;
+    constexpr int LD = (VAR & 1) ? 1 : 0;
+    constexpr int U = (V * W >= 12 && !(VAR & 2)) ? 2 : 4;   // nnz per inner step (B loads in flight per lane: U*V)
+    const int32_t KV = K4 * 4 / W;
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
-    const int col0 = blockIdx.y * CT4 + gl;      // this lane's first float4 column; then + v*G
+    const int col0 = blockIdx.y * CTV + gl;      // this lane's first vector column; then + v*G
     bool colok[V];
 #pragma unroll
-    for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < K4);
-    const uint64_t pol_b = HINT ? policy_evict_last() : 0, pol_a = HINT ? policy_evict_first() : 0;
+    for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < KV);
+    const uint64_t pol_b = LD == 1 ? policy_evict_last() : 0, pol_a = LD == 1 ? policy_evict_first() : 0;
 
     __shared__ TaskQueue q;
     unsigned int tk = 0;
@@ -158,211 +311,91 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
             t_next = __shfl_sync(0xffffffffu, tk, 0);
         }
         const int4 u_next = t_next < n_tasks ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
-        const int32_t start = u.x, len = u.y, dst = u.z;
-        // warp-uniform trip count (groups past their own length are predicated off, not diverged, so
-        // the (col, val) shuffles below stay warp-wide)
-        const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
-        float4 acc[V];
-#pragma unroll
-        for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
-        // (col, val) pairs: each lane loads PL of the group's next BATCH pairs (coalesced), one batch
-        // ahead of use; every nnz is then broadcast inside the group with two shuffles
-        int2 cur[PL];
-#pragma unroll
-        for (int p = 0; p < PL; ++p) {
-            const int32_t o = p * G + gl;
-            cur[p] = o < len ? ld_cv<HINT>(cv + start + o, pol_a) : make_int2(0, 0);
-        }
-        for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
-            int2 nxt[PL];
-#pragma unroll
-            for (int p = 0; p < PL; ++p) {
-                const int32_t o = b0 + BATCH + p * G + gl;
-                nxt[p] = o < len ? ld_cv<HINT>(cv + start + o, pol_a) : make_int2(0, 0);
-            }
-#pragma unroll
-            for (int q0 = 0; q0 < BATCH; q0 += U) {
-                int32_t col[U];
-                float a[U];
-#pragma unroll
-                for (int w = 0; w < U; ++w) {
-                    const int qq = q0 + w;
-                    const int src = g * G + (qq % G);
-                    col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
-                    a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
-                }
-                const int32_t rem = len - (b0 + q0);    // nnz left for this group
-                if (rem >= U) {                          // full step: U*V independent B loads in flight
-                    float4 x[U][V];
-#pragma unroll
-                    for (int w = 0; w < U; ++w) {
-                        const float4 *b = B4 + (size_t)col[w] * K4 + col0;
-#pragma unroll
-                        for (int v = 0; v < V; ++v)
-                            x[w][v] = colok[v] ? ld_b<HINT>(b + v * G, pol_b) : make_float4(0.f, 0.f, 0.f, 0.f);
-                    }
-#pragma unroll
-                    for (int w = 0; w < U; ++w)
-#pragma unroll
-                        for (int v = 0; v < V; ++v) fma4(a[w], x[w][v], acc[v]);
-                } else if (rem > 0) {                    // the group's tail
-#pragma unroll
-                    for (int w = 0; w < U - 1; ++w) {
-                        if (w < rem) {
-                            const float4 *b = B4 + (size_t)col[w] * K4 + col0;
-#pragma unroll
-                            for (int v = 0; v < V; ++v)
-                                if (colok[v]) fma4(a[w], ld_b<HINT>(b + v * G, pol_b), acc[v]);
-                        }
-                    }
-                }
-            }
-#pragma unroll
-            for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
-        }
-        if (dst >= 0) {                                    // a whole row: C[perm[p]]
-#pragma unroll
-            for (int v = 0; v < V; ++v)
-                if (colok[v]) __stcs(C4 + (size_t)dst * K4 + col0 + v * G, acc[v]);
-        } else if (dst != NOSTORE) {                       // chunk group of a long row (warp-uniform)
-#pragma unroll
-            for (int off = G; off < 32; off <<= 1) {       // fixed butterfly: ((c0+c1)+(c2+c3))...
-#pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    acc[v].x += __shfl_xor_sync(0xffffffffu, acc[v].x, off);
-                    acc[v].y += __shfl_xor_sync(0xffffffffu, acc[v].y, off);
-                    acc[v].z += __shfl_xor_sync(0xffffffffu, acc[v].z, off);
-                    acc[v].w += __shfl_xor_sync(0xffffffffu, acc[v].w, off);
-                }
-            }
-            if (g == 0) {
-                const int64_t slot = -(int64_t)dst - 1;
-#pragma unroll
-                for (int v = 0; v < V; ++v)
-                    if (colok[v]) P4[slot * K4 + col0 + v * G] = acc[v];
-            }
-        }
+        spmm_unit<V, G, U, LD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4),
+                               KV, reinterpret_cast<VT *>(P4), pol_b, pol_a);
         t = t_next;
         u = u_next;
     }
 }
 
-// ---- kernel mode 2: panel-staged SpMM (schedule: panel.cu) --------------------------------------
-// One CTA (16 warps) per SM claims panels of consecutive permuted rows.  Per panel it first copies the
-// panel's staged B rows into shared memory with cp.async, then its warps claim the panel's work units
-// RPW at a time (shared-memory counter); a nnz whose column was staged (col < 0 in the rewritten cv)
-// reads its B row from shared memory, the others from global memory, through one generic load.  Same
-// per-row FMA order as the row-group kernel; chunks of long rows write partials (combined pairwise).
-constexpr int PS_THREADS = 512;
+// ---- kernel mode 3: SM-affine column-tiled SpMM ---------------------------------------------------
+// One persistent CTA per SM.  Work items are (panel, column tile) pairs, panel = `ppt` consecutive warp
+// tasks of the a7 schedule (so a panel is a run of consecutive rows of the permuted order), column tile =
+// 4*V*G columns of C.  A CTA owns one item at a time and its warps claim the item's tasks from a
+// shared-memory counter, so every B row the panel's rows share is requested by ONE SM within a short time
+// and can be served by that SM's L1 (the B-row reuse the paper's CTA-aware order aims at, made
+// SM-local; the column tile keeps a panel's working set L1-sized).  The T tiles of a panel are consecutive
+// items, claimed by different SMs at about the same time, so the panel's (col, val) stream is read from
+// HBM once and from L2 by the other tiles.
+// Item hand-over without a barrier: state = (item << 32) | next task offset, advanced by atomicAdd; the
+// one warp that draws offset == #tasks claims the next item from the global counter and publishes it with
+// atomicExch; warps that overshoot spin until the item changes and retry.
+constexpr int AFF_THREADS = 768;
 
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
+// claim the next (item, task) of this CTA; returns false when the work is exhausted
+__device__ __forceinline__ bool aff_claim(unsigned long long *state, unsigned int *counter, int64_t n_tasks,
+                                          int32_t ppt, int32_t T, int64_t n_items, int lane, int64_t &task,
+                                          int32_t &tile) {
+    for (;;) {
+        unsigned long long old = 0;
+        if (lane == 0) old = atomicAdd(state, 1ull);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        const int64_t item = (int64_t)(old >> 32);
+        if (item >= n_items) return false;
+        const int64_t off = (int64_t)(old & 0xffffffffull);
+        const int64_t panel = item / T;
+        const int64_t t0 = panel * ppt;
+        const int64_t nt = n_tasks - t0 < ppt ? n_tasks - t0 : ppt;
+        if (off < nt) {
+            task = t0 + off;
+            tile = (int32_t)(item - panel * T);
+            return true;
+        }
+        if (off == nt) {
+            if (lane == 0) atomicExch(state, (unsigned long long)atomicAdd(counter, 1u) << 32);
+        } else if (lane == 0) {
+            volatile unsigned long long *vs = state;
+            while ((int64_t)(*vs >> 32) == item) { }
+        }
+        __syncwarp();
+    }
 }
 
-template <int V, int G>
-__global__ void __launch_bounds__(PS_THREADS, 1) k_spmm_ps(const int4 *__restrict__ units,
-                                                           const int32_t *__restrict__ panel_unit_ptr,
-                                                           const int32_t *__restrict__ stage_ptr,
-                                                           const int32_t *__restrict__ staged_cols, int64_t n_panels,
-                                                           const int2 *__restrict__ cv, const float4 *__restrict__ B4,
-                                                           float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
-                                                           unsigned int *__restrict__ counter) {
-    extern __shared__ float4 sB[];
-    __shared__ unsigned int s_panel, s_next;
+template <int V, int G, int LD, int W>
+__global__ void __launch_bounds__(AFF_THREADS, 1) k_spmm_aff(const int4 *__restrict__ units, int64_t n_tasks,
+                                                          int32_t ppt, int32_t T, int64_t n_items,
+                                                          const int2 *__restrict__ cv, const float4 *__restrict__ B4,
+                                                          float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
+                                                          unsigned int *__restrict__ counter) {
+    using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
-    constexpr int U = V >= 3 ? 2 : 4;
-    constexpr int BATCH = G >= 8 ? G : 8;
-    constexpr int PL = BATCH / G;
+    constexpr int CTV = V * G;
+    constexpr int U = V * W == 4 ? 8 : V * W == 8 ? 4 : 2;
+    const int32_t KV = K4 * 4 / W;
+    __shared__ unsigned long long state;
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
-    for (;;) {
-        if (threadIdx.x == 0) { s_panel = atomicAdd(counter, 1u); s_next = 0u; }
-        __syncthreads();
-        const unsigned int P = s_panel;
-        if (P >= n_panels) break;
-        const int32_t s0 = stage_ptr[P], ns = stage_ptr[P + 1] - s0;
-        for (int32_t i = threadIdx.x; i < ns * K4; i += PS_THREADS) {
-            const int32_t r = i / K4, c = i - r * K4;
-            cp_async16(sB + (size_t)r * K4 + c, B4 + (size_t)staged_cols[s0 + r] * K4 + c);
-        }
-        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-        __syncthreads();
-        const int32_t u0 = panel_unit_ptr[P], nu = panel_unit_ptr[P + 1] - u0;
-        for (;;) {
-            unsigned int kk = 0;
-            if (lane == 0) kk = atomicAdd(&s_next, (unsigned)RPW);
-            kk = __shfl_sync(0xffffffffu, kk, 0);
-            if ((int32_t)kk >= nu) break;
-            const int4 u = (int32_t)kk + g < nu ? __ldg(units + u0 + kk + g) : make_int4(0, 0, NOSTORE, 0);
-            const int32_t start = u.x, len = u.y, dst = u.z;
-            const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
-            float4 acc[V];
+    bool colok[V];
 #pragma unroll
-            for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
-            int2 cur[PL];
-#pragma unroll
-            for (int p = 0; p < PL; ++p) {
-                const int32_t o = p * G + gl;
-                cur[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
-            }
-            for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
-                int2 nxt[PL];
-#pragma unroll
-                for (int p = 0; p < PL; ++p) {
-                    const int32_t o = b0 + BATCH + p * G + gl;
-                    nxt[p] = o < len ? __ldg(cv + start + o) : make_int2(0, 0);
-                }
-#pragma unroll
-                for (int q0 = 0; q0 < BATCH; q0 += U) {
-                    int32_t col[U];
-                    float a[U];
-#pragma unroll
-                    for (int w = 0; w < U; ++w) {
-                        const int qq = q0 + w;
-                        const int src = g * G + (qq % G);
-                        col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
-                        a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
-                    }
-                    const int32_t rem = len - (b0 + q0);
-                    if (rem >= U) {
-                        float4 x[U][V];
-#pragma unroll
-                        for (int w = 0; w < U; ++w) {
-                            const float4 *b = col[w] < 0 ? sB + (size_t)(col[w] & 0x7fffffff) * K4 + gl
-                                                         : B4 + (size_t)col[w] * K4 + gl;
-#pragma unroll
-                            for (int v = 0; v < V; ++v) x[w][v] = b[v * G];
-                        }
-#pragma unroll
-                        for (int w = 0; w < U; ++w)
-#pragma unroll
-                            for (int v = 0; v < V; ++v) fma4(a[w], x[w][v], acc[v]);
-                    } else if (rem > 0) {
-#pragma unroll
-                        for (int w = 0; w < U - 1; ++w) {
-                            if (w < rem) {
-                                const float4 *b = col[w] < 0 ? sB + (size_t)(col[w] & 0x7fffffff) * K4 + gl
-                                                             : B4 + (size_t)col[w] * K4 + gl;
-#pragma unroll
-                                for (int v = 0; v < V; ++v) fma4(a[w], b[v * G], acc[v]);
-                            }
-                        }
-                    }
-                }
-#pragma unroll
-                for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
-            }
-            if (dst >= 0) {
-#pragma unroll
-                for (int v = 0; v < V; ++v) __stcs(C4 + (size_t)dst * K4 + gl + v * G, acc[v]);
-            } else if (dst != NOSTORE) {
-                const int64_t slot = -(int64_t)dst - 1;
-#pragma unroll
-                for (int v = 0; v < V; ++v) P4[slot * K4 + gl + v * G] = acc[v];
-            }
-        }
-        __syncthreads();   // every warp is done with this panel before the next one is staged
+    for (int v = 0; v < V; ++v) colok[v] = true;
+    if (threadIdx.x == 0) state = (unsigned long long)atomicAdd(counter, 1u) << 32;
+    __syncthreads();
+    int64_t t = 0;
+    int32_t tile = 0;
+    bool ok = aff_claim(&state, counter, n_tasks, ppt, T, n_items, lane, t, tile);
+    int4 u = ok ? __ldg(units + t * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+    while (ok) {
+        // claim and fetch the next task first, so its latency hides behind this one
+        int64_t t_next = 0;
+        int32_t tile_next = 0;
+        const bool ok_next = aff_claim(&state, counter, n_tasks, ppt, T, n_items, lane, t_next, tile_next);
+        const int4 u_next = ok_next ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+        spmm_unit<V, G, U, LD>(u, g, gl, tile * CTV + gl, colok, cv, reinterpret_cast<const VT *>(B4),
+                               reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), 0, 0);
+        ok = ok_next;
+        t = t_next;
+        tile = tile_next;
+        u = u_next;
     }
 }
 
@@ -437,34 +470,63 @@ __global__ void k_segment_counts(const int32_t *lpos, int64_t n_long, const int3
     }
 }
 
+// lengths of the short rows in compacted (position) order
+__global__ void k_short_len(const int32_t *is_short, const int32_t *sp, const int32_t *rowptr, int64_t M, int32_t *slen) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x)
+        if (is_short[p]) slen[sp[p]] = rowptr[p + 1] - rowptr[p];
+}
+
+// Short rows -> units.  The run of short rows of a segment is cut into windows of `win` consecutive rows
+// (win a multiple of RPW; 0 = no windows); inside a window the rows are placed by descending length (ties:
+// position), so the RPW rows of a warp task have similar lengths and the warp-uniform trip count (the
+// longest unit) wastes few lane slots -- the paper's load-balance concern applied within a
+// window of `win` rows, which keeps the permuted order's locality (all rows of a window run at about the
+// same time).  The per-row arithmetic is unchanged (one unit per row).
 __global__ void k_fill_short(const int32_t *is_short, const int32_t *sp, const int32_t *lidx, const int32_t *lpos,
-                             const int32_t *taskbase, const int32_t *rowptr, const int32_t *perm, int64_t M,
-                             int32_t rpw, int4 *units) {
+                             const int32_t *taskbase, const int32_t *rowptr, const int32_t *perm, const int32_t *slen,
+                             int32_t n_short, int64_t n_long, int64_t M, int32_t rpw, int32_t win, int4 *units) {
     for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
         if (!is_short[p]) continue;
         const int32_t k = lidx[p];                         // long rows before p = this run's segment
-        const int32_t idx = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
+        const int32_t before = k > 0 ? sp[lpos[k - 1]] : 0;
+        int32_t idx = sp[p] - before;
+        const int32_t len = rowptr[p + 1] - rowptr[p];
+        if (win > 0) {
+            const int32_t w0 = before + (idx / win) * win;
+            const int32_t upto = k < n_long ? sp[lpos[k]] : n_short;   // end of this run
+            const int32_t w1 = w0 + win < upto ? w0 + win : upto;
+            int32_t rank = 0;
+            const int32_t me = sp[p];
+            for (int32_t j = w0; j < w1; ++j) {
+                const int32_t lj = slen[j];
+                rank += (lj > len) || (lj == len && j < me);
+            }
+            idx = (idx / win) * win + rank;
+        }
         const int64_t task = (int64_t)taskbase[k] + idx / rpw;
-        units[task * rpw + idx % rpw] = make_int4(rowptr[p], rowptr[p + 1] - rowptr[p], perm[p], 0);
+        units[task * rpw + idx % rpw] = make_int4(rowptr[p], len, perm[p], 0);
     }
 }
 
-// warp per long row: its chunk groups follow the run of short rows of its segment
+// Warp per long row: its chunk groups follow the run of short rows of its segment.  The row is cut into
+// nch' = RPW * ceil(ceil(len / split) / RPW) chunks of balanced sizes (floor or ceil of len / nch', each
+// <= split), so the RPW chunks of every chunk group have equal trip counts.  The cut depends only on the
+// row length (and RPW), not on the row's position: C stays bit-identical under every permutation.
 __global__ void k_fill_long(const int32_t *lpos, int64_t n_long, const int32_t *sp, const int32_t *taskbase,
-                            const int32_t *pslot_ptr, const int32_t *rowptr, const int32_t *perm, int32_t split,
-                            int32_t rpw, int4 *units, int32_t *long_dst) {
+                            const int32_t *pslot_ptr, const int32_t *rowptr, const int32_t *perm, int32_t rpw,
+                            int4 *units, int32_t *long_dst) {
     const int lane = threadIdx.x & 31;
     for (int64_t k = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n_long;
          k += ((int64_t)gridDim.x * blockDim.x) >> 5) {
         const int32_t p = lpos[k];
         const int32_t s_k = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
         const int64_t t0 = (int64_t)taskbase[k] + (s_k + rpw - 1) / rpw;
-        const int32_t a = rowptr[p], len = rowptr[p + 1] - a, nch = (len + split - 1) / split;
+        const int32_t a = rowptr[p], len = rowptr[p + 1] - a;
         const int32_t ng = pslot_ptr[k + 1] - pslot_ptr[k];
-        for (int32_t c = lane; c < ng * rpw; c += 32) {
+        const int32_t nch = ng * rpw, base = len / nch, extra = len % nch;
+        for (int32_t c = lane; c < nch; c += 32) {
             const int32_t dst = -(pslot_ptr[k] + c / rpw) - 1;
-            units[(t0 + c / rpw) * rpw + c % rpw] =
-                c < nch ? make_int4(a + c * split, min(split, len - c * split), dst, 0) : make_int4(0, 0, dst, 0);
+            units[(t0 + c / rpw) * rpw + c % rpw] = make_int4(a + c * base + min(c, extra), base + (c < extra), dst, 0);
         }
         if (lane == 0) long_dst[k] = perm[p];
     }
@@ -523,13 +585,18 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
     if (n_tasks > 0) {
         k_fill_int4<<<g1((int64_t)n_tasks * rpw), 256, 0, s>>>(S.units.as<int4>(), (int64_t)n_tasks * rpw,
                                                                 make_int4(0, 0, NOSTORE, 0));
+        static const int win_env = [] { const char *e = getenv("SPMM_SORT_WIN"); return e ? atoi(e) : 32; }();
+        const int32_t win = win_env <= 0 ? 0 : (int32_t)ceil_div(win_env, rpw) * rpw;
+        DevBuf slen;
+        SPMM_TRY(slen.alloc(std::max(n_short, 1) * sizeof(int32_t), s));
+        k_short_len<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), rowptr, M, slen.as<int32_t>());
         k_fill_short<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), pl.as<int32_t>(), lpos.as<int32_t>(),
-                                           taskbase.as<int32_t>(), rowptr, h->perm.as<int32_t>(), M, rpw,
-                                           S.units.as<int4>());
+                                           taskbase.as<int32_t>(), rowptr, h->perm.as<int32_t>(), slen.as<int32_t>(),
+                                           n_short, n_long, M, rpw, win, S.units.as<int4>());
         if (n_long > 0)
             k_fill_long<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)n_long * 32, 256), 148 * 32)),
                           256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), taskbase.as<int32_t>(),
-                                       S.pslot_ptr.as<int32_t>(), rowptr, h->perm.as<int32_t>(), split, rpw,
+                                       S.pslot_ptr.as<int32_t>(), rowptr, h->perm.as<int32_t>(), rpw,
                                        S.units.as<int4>(), S.long_dst.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
     }
@@ -543,16 +610,16 @@ using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *,
 template <int V, bool MASK, int SCHED, int VAR>
 SpmmKernel pick_g(int G) {
     switch (G) {
-        case 1: return k_spmm<V, 1, MASK, SCHED, VAR>;
-        case 2: return k_spmm<V, 2, MASK, SCHED, VAR>;
-        case 4: return k_spmm<V, 4, MASK, SCHED, VAR>;
-        case 8: return k_spmm<V, 8, MASK, SCHED, VAR>;
-        case 16: return k_spmm<V, 16, MASK, SCHED, VAR>;
-        default: return k_spmm<V, 32, MASK, SCHED, VAR>;
+        case 1: return k_spmm<V, 1, MASK, SCHED, VAR, 4>;
+        case 2: return k_spmm<V, 2, MASK, SCHED, VAR, 4>;
+        case 4: return k_spmm<V, 4, MASK, SCHED, VAR, 4>;
+        case 8: return k_spmm<V, 8, MASK, SCHED, VAR, 4>;
+        case 16: return k_spmm<V, 16, MASK, SCHED, VAR, 4>;
+        default: return k_spmm<V, 32, MASK, SCHED, VAR, 4>;
     }
 }
 // run-time knobs (tuning experiments; defaults are the measured best): SPMM_SCHED (0 per-warp claiming,
-// 1 CTA-contiguous queue), SPMM_VARIANT (bit 0 L2 cache hints, bit 1 U=4)
+// 1 CTA-contiguous queue), SPMM_VARIANT (bit 0 L2 cache hints, bit 1 U=4), SPMM_W (4: LDG.128 only)
 template <int V, bool MASK>
 SpmmKernel pick_gs(int G, int sched, int var) {
     if (sched) return pick_g<V, MASK, 1, 0>(G);
@@ -563,32 +630,50 @@ SpmmKernel pick_gs(int G, int sched, int var) {
         default: return pick_g<V, MASK, 0, 0>(G);
     }
 }
-
-using PsKernel = void (*)(const int4 *, const int32_t *, const int32_t *, const int32_t *, int64_t, const int2 *,
-                          const float4 *, float4 *, int32_t, float4 *, unsigned int *);
-PsKernel pick_ps(int V, int G) {
-    if (G == 8) return V == 4 ? k_spmm_ps<4, 8> : V == 3 ? k_spmm_ps<3, 8> : V == 2 ? k_spmm_ps<2, 8> : k_spmm_ps<1, 8>;
-    if (G == 16) return V == 4 ? k_spmm_ps<4, 16> : V == 3 ? k_spmm_ps<3, 16> : V == 2 ? k_spmm_ps<2, 16> : k_spmm_ps<1, 16>;
-    if (G == 32) return V == 4 ? k_spmm_ps<4, 32> : V == 3 ? k_spmm_ps<3, 32> : V == 2 ? k_spmm_ps<2, 32> : k_spmm_ps<1, 32>;
-    return nullptr;
+// 256-bit lane loads (W = 8), exact fits only, per-warp claiming, VAR 0 or 1
+template <int VAR>
+SpmmKernel pick_w8(int V, int G) {
+    switch (V * 100 + G) {
+        case 104: return k_spmm<1, 4, false, 0, VAR, 8>;
+        case 108: return k_spmm<1, 8, false, 0, VAR, 8>;
+        case 204: return k_spmm<2, 4, false, 0, VAR, 8>;
+        case 208: return k_spmm<2, 8, false, 0, VAR, 8>;
+        case 408: return k_spmm<4, 8, false, 0, VAR, 8>;
+        case 416: return k_spmm<4, 16, false, 0, VAR, 8>;
+        case 432: return k_spmm<4, 32, false, 0, VAR, 8>;
+        default: return nullptr;
+    }
 }
 
 struct Config {
     SpmmKernel kern;
-    int V, G, tiles;
+    int V, G, tiles, W;
 };
 
-// Exact fit 4*V*G == K with V in {4,3,2,1} and G a power of two <= 32, preferring G >= 8 so that one
-// vector load of a group covers whole 128-byte lines (G*16 B >= 128 B: an L1 wavefront per line, measured
-// to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
-Config choose(int32_t K4, int sched, int var) {
+// Lane geometry.  W = 8 (one 256-bit load per lane and vector) when K % 8 == 0 and B, C are 32-byte aligned:
+// 8*V*G == K with G in {8, 4} preferred (a group's load covers whole 128-byte lines; G = 8 keeps 4 rows per
+// warp at K >= 64), else G in {16, 32} with V = 4.  Otherwise W = 4: exact fit 4*V*G == K with V in
+// {4,3,2,1} and G a power of two <= 32, preferring G >= 8 (G*16 B >= 128 B: an L1 wavefront per line,
+// measured to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
+Config choose(int32_t K4, int sched, int var, bool w8ok) {
+    if (w8ok && sched == 0 && (var & 2) == 0 && K4 % 2 == 0) {
+        const int32_t K8 = K4 / 2;
+        for (int G : {8, 4})
+            for (int V : {1, 2, 4})
+                if (V * G == K8) {
+                    SpmmKernel k = var ? pick_w8<1>(V, G) : pick_w8<0>(V, G);
+                    if (k) return {k, V, G, 1, 8};
+                }
+        for (int G : {16, 32})
+            if (4 * G == K8) return {var ? pick_w8<1>(4, G) : pick_w8<0>(4, G), 4, G, 1, 8};
+    }
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
         int G = K4 / V;
         if (G >= 8 && G <= 32 && (G & (G - 1)) == 0) {
             SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
                          : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
-            return {k, V, G, 1};
+            return {k, V, G, 1, 4};
         }
     }
     for (int V = 4; V >= 1; --V) {
@@ -597,25 +682,49 @@ Config choose(int32_t K4, int sched, int var) {
         if (G >= 1 && G <= 32 && (G & (G - 1)) == 0) {
             SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
                          : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
-            return {k, V, G, 1};
+            return {k, V, G, 1, 4};
         }
     }
     int G = 1;
     while (G < 32 && 4 * G < K4) G <<= 1;
     int tiles = (int)ceil_div(K4, 4 * G);
-    return {pick_gs<4, true>(G, sched, var), 4, G, tiles};
+    return {pick_gs<4, true>(G, sched, var), 4, G, tiles, 4};
 }
 
 }  // namespace
 
-static spmm_status launch_ps(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int V, int G,
-                             int32_t *launches) {
+using AffKernel = void (*)(const int4 *, int64_t, int32_t, int32_t, int64_t, const int2 *, const float4 *, float4 *,
+                          int32_t, float4 *, unsigned int *);
+// mode 3 geometry: column tile of 32*V floats; W = 8: G = 4 lanes x 32 B per 128-byte line, else W = 4: G = 8
+static AffKernel pick_aff(int V, int ld, int W) {
+    switch (W * 100 + V * 10 + ld) {
+        case 410: return k_spmm_aff<1, 8, 0, 4>;
+        case 412: return k_spmm_aff<1, 8, 2, 4>;
+        case 810: return k_spmm_aff<1, 4, 0, 8>;
+        case 812: return k_spmm_aff<1, 4, 2, 8>;
+        case 820: return k_spmm_aff<2, 4, 0, 8>;
+        case 822: return k_spmm_aff<2, 4, 2, 8>;
+        case 840: return k_spmm_aff<4, 4, 0, 8>;
+        case 842: return k_spmm_aff<4, 4, 2, 8>;
+        default: return nullptr;
+    }
+}
+
+static int env_int(const char *name, int dflt) {
+    const char *e = getenv(name);
+    return e ? atoi(e) : dflt;
+}
+
+// Kernel mode 3 (SM-affine, column tiles of 32*V columns, G = 8 lanes per row): needs K % (32*V) == 0.
+static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int V, int W,
+                              int32_t *launches) {
     const int32_t K4 = (int32_t)(K / 4);
-    static const int pr = [] { const char *e = getenv("SPMM_PANEL_ROWS"); return e ? atoi(e) : 256; }();
-    static const int smem_kb = [] { const char *e = getenv("SPMM_PS_SMEM_KB"); return e ? atoi(e) : 200; }();
-    const int32_t cap = (int32_t)std::max<int64_t>(1, ((int64_t)smem_kb * 1024) / (K * 4));
-    if (h->psched.K != K) SPMM_TRY(build_panel_schedule(h, K, pr, cap, s));
-    const PanelSchedule &S = h->psched;
+    static const int ppt = std::max(1, env_int("SPMM_AFF_PPT", 256));
+    static const int ld = env_int("SPMM_AFF_LD", 2);
+    const int32_t rpw = W == 8 ? 8 : 4;                    // G = 4 (W = 8) or 8 (W = 4)
+    if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
+    const Schedule &S = h->sched;
+    const int2 *cv = h->cv_p.as<int2>();
     float4 *C4 = reinterpret_cast<float4 *>(C);
     float4 *P4 = nullptr;
     if (S.n_pslots > 0) {
@@ -628,15 +737,16 @@ static spmm_status launch_ps(spmm_ctx *h, const float *B, int64_t K, float *C, c
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
-    if (S.n_units > 0) {
-        PsKernel kern = pick_ps(V, G);
-        const size_t smem = (size_t)cap * K * sizeof(float);
-        SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (S.n_tasks > 0) {
+        AffKernel kern = pick_aff(V, ld, W);
+        if (!kern) return fail(SPMM_ERR_INVALID_ARG, "unsupported SPMM_AFF_V / SPMM_AFF_LD combination");
+        const int32_t T = (int32_t)(K / (32 * V));
+        const int64_t n_items = ceil_div(S.n_tasks, ppt) * T;
+        SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 0));
         if (h->counters.bytes < sizeof(unsigned int)) SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
         SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, sizeof(unsigned int), s));
-        kern<<<(unsigned)std::min<int64_t>(h->num_sms, S.n_panels), PS_THREADS, smem, s>>>(
-            S.units.as<int4>(), S.panel_unit_ptr.as<int32_t>(), S.stage_ptr.as<int32_t>(), S.staged_cols.as<int32_t>(),
-            S.n_panels, S.cv_ps.as<int2>(), reinterpret_cast<const float4 *>(B), C4, K4, P4,
+        kern<<<(unsigned)std::min<int64_t>(h->num_sms, n_items), AFF_THREADS, 0, s>>>(
+            S.units.as<int4>(), S.n_tasks, ppt, T, n_items, cv, reinterpret_cast<const float4 *>(B), C4, K4, P4,
             h->counters.as<unsigned int>());
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
@@ -654,11 +764,18 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
-    static const int sched = [] { const char *e = getenv("SPMM_SCHED"); return e ? atoi(e) : 0; }();
-    static const int var = [] { const char *e = getenv("SPMM_VARIANT"); return e ? atoi(e) : 0; }();
-    const Config cfg = choose(K4, sched, var);
-    static const int kmode = [] { const char *e = getenv("SPMM_KERNEL"); return e ? atoi(e) : 1; }();
-    if (kmode == 2 && cfg.tiles == 1 && pick_ps(cfg.V, cfg.G) != nullptr) return launch_ps(h, B, K, C, s, cfg.V, cfg.G, launches);
+    static const int sched = env_int("SPMM_SCHED", 0);
+    static const int var = env_int("SPMM_VARIANT", 0);
+    static const int wmax = env_int("SPMM_W", 8);
+    const bool w8ok = wmax >= 8 && K % 8 == 0 && ((uintptr_t)B % 32) == 0 && ((uintptr_t)C % 32) == 0;
+    const Config cfg = choose(K4, sched, var, w8ok);
+    static const int kmode = env_int("SPMM_KERNEL", 1);
+    if (kmode == 3) {
+        static const int av = env_int("SPMM_AFF_V", 1);
+        const int aw = w8ok ? 8 : 4;
+        if (K % (32 * av) == 0 && pick_aff(av, env_int("SPMM_AFF_LD", 2), aw))
+            return launch_aff(h, B, K, C, s, av, aw, launches);
+    }
     const int32_t rpw = 32 / cfg.G;
     if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
     const Schedule &S = h->sched;

@@ -1,5 +1,5 @@
 #!/bin/bash
-# A/B over environment settings: ENVS="SPMM_KERNEL=1|SPMM_KERNEL=2,SPMM_PANEL_ROWS=128" CONFIGS="c3 c2"
+# A/B over environment settings: ENVS="SPMM_KERNEL=1|SPMM_KERNEL=3,SPMM_AFF_V=2" CONFIGS="c3 c2"
 mkdir -p gpurun_out
 export PYTHONUNBUFFERED=1
 if [ -n "$PYTEST_K" ]; then

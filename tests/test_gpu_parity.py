@@ -307,10 +307,14 @@ print("OK")
 
 
 @pytest.mark.parametrize("env", [{"SPMM_SCHED": "1"}, {"SPMM_VARIANT": "1"}, {"SPMM_VARIANT": "2"},
-                                 {"SPMM_VARIANT": "3"}, {"SPMM_KERNEL": "2"},
-                                 {"SPMM_KERNEL": "2", "SPMM_PANEL_ROWS": "64", "SPMM_PS_SMEM_KB": "8"}])
+                                 {"SPMM_VARIANT": "3"}, {"SPMM_W": "4"}, {"SPMM_SORT_WIN": "0"},
+                                 {"SPMM_SORT_WIN": "128"}, {"SPMM_KERNEL": "3"},
+                                 {"SPMM_KERNEL": "3", "SPMM_AFF_V": "2", "SPMM_AFF_LD": "0"},
+                                 {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
+                                 {"SPMM_W": "4", "SPMM_KERNEL": "3"}])
 def test_kernel_variants_exact(env):
-    """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4) are exact on integer inputs."""
+    """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4, 128-bit lane loads, schedule
+    windows, SM-affine column tiles) are exact on integer inputs and permutation-invariant on real inputs."""
     import os
     import subprocess
     import sys

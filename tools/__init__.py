@@ -47,3 +47,12 @@ def lru_misses(csr, order, cap_rows):
     o = None if order is None else np.ascontiguousarray(order, dtype=np.int32)
     return int(_lib.lru_misses(csr.M, csr.N, r.ctypes.data, c.ctypes.data, None if o is None else o.ctypes.data,
                                int(cap_rows)))
+
+
+def l2_read_bandwidth_sms(limit, bytes_=64 << 20, reps=20):
+    """L2->SM read bandwidth (bytes/s) of the SMs with smid < limit (the others idle)."""
+    build()
+    lib = ctypes.CDLL(_PROBE)
+    lib.l2probe_read_bw_sms.restype = ctypes.c_double
+    lib.l2probe_read_bw_sms.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_int]
+    return float(lib.l2probe_read_bw_sms(int(bytes_), int(reps), int(limit)))
