@@ -147,6 +147,15 @@ const char *spmm_last_error(void);
 /* Number of kernel launches issued by the most recent spmm_run on this thread (bench accounting). */
 int32_t spmm_last_run_launches(void);
 
+/* Measurement aid (bench.py's roofline of the dominant kernel): while enabled (enable != 0), every
+ * spmm_run on h records two CUDA events on its cuda_stream around the main SpMM kernel (the row-group
+ * kernel of a8; the empty-row zero fill and the split-row combine are separate launches outside them).
+ * spmm_last_kernel_ms synchronises the second event of the most recent run on h and returns the kernel's
+ * duration in milliseconds (0 when that run launched no SpMM kernel or timing is off).  Events are
+ * owned by the handle.  Errors: INVALID_ARG (NULL), STATE (wrong device), CUDA. */
+spmm_status spmm_set_kernel_timing(spmm_handle h, int enable);
+spmm_status spmm_last_kernel_ms(spmm_handle h, float *ms);
+
 #ifdef __cplusplus
 }
 #endif

@@ -58,7 +58,7 @@ _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
            "spmm_get_permuted_csr", "spmm_get_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_predict",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
-           "spmm_last_run_launches"]
+           "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
 
 def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
@@ -88,6 +88,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_status_string": (ctypes.c_char_p, [st]),
         "spmm_last_error": (ctypes.c_char_p, []),
         "spmm_last_run_launches": (i32, []),
+        "spmm_set_kernel_timing": (st, [vp, ctypes.c_int]),
+        "spmm_last_kernel_ms": (st, [vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -230,6 +232,16 @@ class SpMM:
     @staticmethod
     def last_run_launches() -> int:
         return int(load_library().spmm_last_run_launches())
+
+    def set_kernel_timing(self, enable: bool = True):
+        """CUDA events around the main SpMM kernel of every run (spmm_set_kernel_timing)."""
+        _check(load_library().spmm_set_kernel_timing(self._h, int(bool(enable))))
+
+    def last_kernel_ms(self) -> float:
+        """Duration of the main SpMM kernel of the most recent run (synchronises its end event)."""
+        ms = ctypes.c_float(0.0)
+        _check(load_library().spmm_last_kernel_ms(self._h, ctypes.byref(ms)))
+        return float(ms.value)
 
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -352,6 +352,8 @@ spmm_status spmm_destroy(spmm_handle h) {
     if (!h) return SPMM_OK;
     cudaStreamSynchronize(h->create_stream);
     cudaDeviceSynchronize();
+    if (h->ev0) cudaEventDestroy(h->ev0);
+    if (h->ev1) cudaEventDestroy(h->ev1);
     delete h;
     return SPMM_OK;
 }
@@ -372,5 +374,26 @@ const char *spmm_status_string(spmm_status s) {
 const char *spmm_last_error(void) { return g_last_error.c_str(); }
 
 int32_t spmm_last_run_launches(void) { return g_last_launches; }
+
+spmm_status spmm_set_kernel_timing(spmm_handle h, int enable) {
+    if (!h) return fail(SPMM_ERR_INVALID_ARG, "handle is NULL");
+    SPMM_TRY(check_device(h));
+    if (enable && !h->ev0) {
+        SPMM_CUDA(cudaEventCreate(&h->ev0));
+        SPMM_CUDA(cudaEventCreate(&h->ev1));
+    }
+    h->timing = enable != 0;
+    h->timed = false;
+    return SPMM_OK;
+}
+
+spmm_status spmm_last_kernel_ms(spmm_handle h, float *ms) {
+    if (!h || !ms) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    *ms = 0.f;
+    if (!h->timed) return SPMM_OK;
+    SPMM_CUDA(cudaEventSynchronize(h->ev1));
+    SPMM_CUDA(cudaEventElapsedTime(ms, h->ev0, h->ev1));
+    return SPMM_OK;
+}
 
 }  // extern "C"

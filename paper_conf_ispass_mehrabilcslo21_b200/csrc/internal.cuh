@@ -104,6 +104,10 @@ struct spmm_ctx {
     // host-run staging
     spmm::DevBuf stage_B, stage_C;
     int num_sms = 148;
+    // optional kernel timing (spmm_set_kernel_timing): events around the main SpMM kernel of spmm_run
+    int timing = 0;
+    bool timed = false;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 };
 
 namespace spmm {

@@ -745,10 +745,15 @@ static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, 
         SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 0));
         if (h->counters.bytes < sizeof(unsigned int)) SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
         SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, sizeof(unsigned int), s));
+        if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         kern<<<(unsigned)std::min<int64_t>(h->num_sms, n_items), AFF_THREADS, 0, s>>>(
             S.units.as<int4>(), S.n_tasks, ppt, T, n_items, cv, reinterpret_cast<const float4 *>(B), C4, K4, P4,
             h->counters.as<unsigned int>());
         SPMM_CUDA(cudaGetLastError());
+        if (h->timing) {
+            SPMM_CUDA(cudaEventRecord(h->ev1, s));
+            h->timed = true;
+        }
         ++*launches;
     }
     if (S.n_long > 0) {
@@ -761,6 +766,7 @@ static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, 
 
 spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches) {
     *launches = 0;
+    h->timed = false;
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
@@ -801,10 +807,15 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         if (h->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int))
             SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
         SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
+        if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         cfg.kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
                                                reinterpret_cast<const float4 *>(B), C4, K4, P4,
                                                h->counters.as<unsigned int>());
         SPMM_CUDA(cudaGetLastError());
+        if (h->timing) {
+            SPMM_CUDA(cudaEventRecord(h->ev1, s));
+            h->timed = true;
+        }
         ++*launches;
     }
     if (S.n_long > 0) {

@@ -75,6 +75,31 @@ def main():
         rd = to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
         traffic[f"{cfg}/{pol}"] = {"dram_bytes_per_launch": rd, "kernel": d["kernel"].split("(")[0],
                                    "duration": d["gpu__time_duration.sum"], "round": args.round}
+    # raw-page CSV exports (scripts/gpu_prof_env.sh: prof_<config>_<policy>_<tag>.raw.csv; tag "def" = defaults)
+    for rc in sorted(glob.glob(os.path.join(OUT, "prof_*.raw.csv"))):
+        m = re.match(r"prof_([a-z0-9]+)_(.+)_([a-z0-9]+)\.raw\.csv", os.path.basename(rc))
+        if not m:
+            continue
+        cfg, pol, tag = m.groups()
+        rows = list(csv.reader(open(rc)))
+        if len(rows) < 3:
+            continue
+        h, units, r = rows[0], rows[1], rows[2]
+        d = {"kernel": r[h.index("Kernel Name")] if "Kernel Name" in h else ""}
+        for k in KEYS:
+            if k in h:
+                d[k] = (r[h.index(k)], units[h.index(k)])
+        name = f"{cfg}_{pol}" + ("" if tag == "def" else f"_{tag}")
+        with open(os.path.join(PROF, f"{args.round}_ncu_{name}.txt"), "w") as f:
+            f.write(f"# ncu --set full --clock-control none, one launch of {d['kernel']}\n")
+            f.write(f"# python scripts/profile_spmm.py --config {cfg} --policy {pol} (env tag {tag})\n")
+            for k in KEYS:
+                if k in d:
+                    f.write(f"{k} {d[k][0]} {d[k][1]}\n")
+        if tag == "def":
+            rd = to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
+            traffic[f"{cfg}/{pol}"] = {"dram_bytes_per_launch": rd, "kernel": d["kernel"].split("(")[0],
+                                       "duration": d["gpu__time_duration.sum"], "round": args.round}
     with open(traffic_path, "w") as f:
         json.dump(traffic, f, indent=1, sort_keys=True)
     for bj in sorted(glob.glob(os.path.join(OUT, "bench*.json"))):

@@ -324,6 +324,26 @@ def test_kernel_variants_exact(env):
     assert r.returncode == 0 and "OK" in r.stdout, r.stderr[-2000:]
 
 
+def test_kernel_timing_api():
+    """spmm_set_kernel_timing / spmm_last_kernel_ms: events around the main kernel, 0 when off."""
+    a = syn.rmat(12, 12, 5, "local")
+    h = pkg.SpMM.from_csr(a)
+    B = torch.from_numpy(syn.dense(a.N, 64, 6)).cuda()
+    h.run(B)
+    assert h.last_kernel_ms() == 0.0
+    h.set_kernel_timing(True)
+    C = h.run(B)
+    ms = h.last_kernel_ms()
+    assert 0.0 < ms < 1000.0
+    torch.cuda.synchronize()
+    ref, bound = oracle.spmm(a, syn.dense(a.N, 64, 6))
+    assert np.all(np.abs(C.cpu().numpy() - ref) <= 1e-5 * bound + 1e-6)
+    h.set_kernel_timing(False)
+    h.run(B)
+    assert h.last_kernel_ms() == 0.0
+    h.close()
+
+
 def test_select_policy_runs():
     a = syn.rmat(12, 8, 7, "local")
     h = pkg.SpMM.from_csr(a)
