@@ -354,6 +354,9 @@ spmm_status spmm_destroy(spmm_handle h) {
     cudaDeviceSynchronize();
     if (h->ev0) cudaEventDestroy(h->ev0);
     if (h->ev1) cudaEventDestroy(h->ev1);
+    if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+    if (h->ev_join) cudaEventDestroy(h->ev_join);
+    if (h->side) cudaStreamDestroy(h->side);
     delete h;
     return SPMM_OK;
 }

@@ -108,6 +108,9 @@ struct spmm_ctx {
     int timing = 0;
     bool timed = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    // side stream for the empty-row zero fill (SPMM_ZERO_SIDE=1)
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace spmm {

@@ -308,7 +308,7 @@ print("OK")
 
 @pytest.mark.parametrize("env", [{"SPMM_SCHED": "1"}, {"SPMM_VARIANT": "1"}, {"SPMM_VARIANT": "2"},
                                  {"SPMM_VARIANT": "3"}, {"SPMM_W": "4"}, {"SPMM_SORT_WIN": "0"},
-                                 {"SPMM_SORT_WIN": "128"}, {"SPMM_KERNEL": "3"},
+                                 {"SPMM_SORT_WIN": "128"}, {"SPMM_ZERO_SIDE": "0"}, {"SPMM_KERNEL": "3"},
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_V": "2", "SPMM_AFF_LD": "0"},
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
                                  {"SPMM_W": "4", "SPMM_KERNEL": "3"}])
