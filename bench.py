@@ -35,13 +35,13 @@ CONFIGS = {
     "c1": dict(desc="configs[0]: power-law R-MAT S=12 natural, M=N=4096, nnz~40k, K=32", gen=("rmat", 12, 12, 1000, "natural"), K=32),
     "c2": dict(desc="configs[1]: banded FEM-like 27-point stencil 100^3, M=N=1M, ~27 nnz/row, K=64", gen=("stencil", 100, 2000), K=64),
     "c3": dict(desc="configs[2]: power-law R-MAT S=22 'local' (80% in-community columns), M=N=4M, nnz~100M, K=128",
-               gen=("rmat", 22, 26, 3000, "local"), K=128),
+               gen=("rmat", 22, 28, 3000, "local"), K=128),
     "c3rl": dict(desc="configs[2] stress variant: power-law R-MAT S=22 random-label, M=N=4M, nnz~100M, K=128",
-                 gen=("rmat", 22, 26, 3001, "random-label"), K=128),
-    "c5": dict(desc="configs[4]: power-law R-MAT S=24 'local', M=N=16M, nnz~500M, K=128", gen=("rmat", 24, 32, 5000, "local"), K=128),
+                 gen=("rmat", 22, 28, 3001, "random-label"), K=128),
+    "c5": dict(desc="configs[4]: power-law R-MAT S=24 'local', M=N=16M, nnz~500M, K=128", gen=("rmat", 24, 38, 5000, "local"), K=128),
 }
 HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1"]
-METRIC = "SpMM GFLOP/s and % HBM roofline per permutation policy"
+METRIC = "SpMM GFLOP/s and % HBM roofline per permutation policy at 1/2/4/8 B200"
 
 
 def make_matrix(cfg):
@@ -68,29 +68,61 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """SM clock + clock-event (throttle) reasons sampled during the timed region: NVML every 10 ms (pynvml, the
+    device matched by PCI bus id), else nvidia-smi every 200 ms."""
 
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+    # NVML clocks-event reason bits for NAMES (nvmlClocksEventReason*: HwSlowdown 0x8, HwThermalSlowdown 0x40,
+    # SwThermalSlowdown 0x20, SwPowerCap 0x4)
+    BITS = [0x8, 0x40, 0x20, 0x4]
 
     def __init__(self, index=0):
         self.index = index
-        self.samples = []
+        self.samples = []          # (sm_mhz, max_mhz, [reason flags])
+        self.source = None
         self._stop = threading.Event()
         self._t = None
 
+    def _nvml_handle(self):
+        import pynvml
+        import torch
+        pynvml.nvmlInit()
+        try:
+            pr = torch.cuda.get_device_properties(self.index)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+        except Exception:  # noqa: BLE001
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.index)
+
     def start(self):
+        try:
+            nv, hd = self._nvml_handle()
+            mx = float(nv.nvmlDeviceGetMaxClockInfo(hd, nv.NVML_CLOCK_SM))
+            self.source = "nvml 10 ms"
+        except Exception:  # noqa: BLE001
+            nv = hd = None
+            self.source = "nvidia-smi 200 ms"
+
         def run():
             while not self._stop.is_set():
                 try:
-                    out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                         timeout=5).stdout.strip()
-                    if out:
-                        self.samples.append([x.strip() for x in out.split(",")])
+                    if nv is not None:
+                        sm = float(nv.nvmlDeviceGetClockInfo(hd, nv.NVML_CLOCK_SM))
+                        r = int(nv.nvmlDeviceGetCurrentClocksEventReasons(hd))
+                        self.samples.append((sm, mx, [bool(r & b) for b in self.BITS]))
+                    else:
+                        out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                              "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                             timeout=5).stdout.strip()
+                        f = [x.strip() for x in out.split(",")]
+                        if len(f) >= 6 and f[0].replace(".", "").isdigit():
+                            self.samples.append((float(f[0]), float(f[1]),
+                                                 ["Active" in x and "Not" not in x for x in f[2:6]]))
                 except Exception:  # noqa: BLE001
                     pass
-                self._stop.wait(0.2)
+                self._stop.wait(0.01 if nv is not None else 0.2)
         self._t = threading.Thread(target=run, daemon=True)
         self._t.start()
 
@@ -98,13 +130,11 @@ class ClockSampler:
         self._stop.set()
         if self._t:
             self._t.join(timeout=10)
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
-        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
-        reasons = sorted({names[i] for s in self.samples for i in range(4) if len(s) > 2 + i and "Active" in s[2 + i]
-                          and "Not" not in s[2 + i]})
+        sm = [s[0] for s in self.samples]
+        mx = [s[1] for s in self.samples]
+        reasons = sorted({self.NAMES[i] for s in self.samples for i in range(4) if s[2][i]})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.samples)}
+                "reasons": reasons, "samples": len(self.samples), "source": self.source}
 
 
 def time_runs(torch, fn, steps, flush, stream, after=None):
@@ -309,7 +339,7 @@ def main():
         ts = time_runs(torch, lambda: h.run(Bd, Cd), args.policy_steps, flush, stream)
         ms = statistics.median(ts)
         pol_res[pol] = {"ms": ms, "gflops": flops / ms / 1e6, "build_ms": build_ms, "launches": h.last_run_launches(),
-                        "info": h.info()}
+                        "info": h.info(), "schedule": h.schedule_info()}
         if a_host is not None:
             # L2-capacity ceiling: B-row misses of an LRU of L2 size in this order
             import tools

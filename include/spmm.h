@@ -72,11 +72,15 @@ typedef struct {
     int64_t window;         /* greedy-chain window W (multiple of nw); 0 = whole matrix (paper-exact,
                                supported up to 32768 rows); default 1024                               */
     int32_t preorder;       /* chain policies: 0 = windows over the original order, 1 = MinHash key  */
-    int32_t reserved;
+    int32_t fuse_rows;      /* row fusion in spmm_run (a7/a8): 0 = auto -- take the short rows R consecutive
+                               positions at a time and walk the union of their columns once (each shared B
+                               row loaded once) when the unions hold <= 3/4 of those rows' nnz; 1 = off;
+                               2 = always (where the K geometry has a fused kernel: R = 4 at K = 32/64,
+                               R = 2 at K = 128).  C is bit-identical in every setting.                 */
     uint64_t seed;          /* MinHash seed                                                          */
 } spmm_params;
 
-/* Fill *p with the defaults (nw=nt=bw=32, split_nnz=128, window=1024, preorder=0, seed=0). */
+/* Fill *p with the defaults (nw=nt=bw=32, split_nnz=128, window=1024, preorder=0, fuse_rows=0, seed=0). */
 spmm_status spmm_default_params(spmm_params *p);
 
 /* Optional device allocator (e.g. PyTorch's caching allocator).  alloc(bytes, stream, ctx) returns a
@@ -109,6 +113,12 @@ spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colid
  * rows handled whole (nnz <= split_nnz), out[2]=split (long) rows, out[3]=split_nnz-chunks of the split
  * rows, out[4]=max row nnz. */
 spmm_status spmm_get_info(spmm_handle h, int64_t out[5]);
+
+/* Run schedule (a7) built by the most recent spmm_run on h: out[0] = rows per warp task (lane groups; 0 = no
+ * schedule yet), out[1] = row-fusion factor R in use (1 = none), out[2] = warp tasks, out[3] = fusion groups,
+ * out[4] = union records of those groups, out[5] = nnz of the fused rows (out[4] / out[5] = B-row loads per
+ * nnz on the fused rows).  Errors: INVALID_ARG (NULL). */
+spmm_status spmm_get_schedule_info(spmm_handle h, int64_t out[6]);
 
 /* The 24 Table II features (definitions DESIGN.md §"Features") computed on the device,
  * of the ORIGINAL order (use_current_order = 0) or of the current permutation (1), with nw/nt/bw from

@@ -47,7 +47,7 @@ class SpmmError(RuntimeError):
 
 class _Params(ctypes.Structure):
     _fields_ = [("nw", ctypes.c_int32), ("nt", ctypes.c_int32), ("bw", ctypes.c_int32), ("split_nnz", ctypes.c_int32),
-                ("window", ctypes.c_int64), ("preorder", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("window", ctypes.c_int64), ("preorder", ctypes.c_int32), ("fuse_rows", ctypes.c_int32),
                 ("seed", ctypes.c_uint64)]
 
 
@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_predict",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_predict",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -79,6 +79,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_get_perm": (st, [vp, vp]),
         "spmm_get_permuted_csr": (st, [vp, vp, vp, vp]),
         "spmm_get_info": (st, [vp, vp]),
+        "spmm_get_schedule_info": (st, [vp, vp]),
         "spmm_features": (st, [vp, ctypes.c_int, vp, vp, vp]),
         "spmm_run": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
@@ -139,10 +140,11 @@ def _stream_ptr(stream):
     return stream.cuda_stream
 
 
-def make_params(nw=32, nt=32, bw=32, split_nnz=128, window=1024, preorder=0, seed=0) -> _Params:
+def make_params(nw=32, nt=32, bw=32, split_nnz=128, window=1024, preorder=0, seed=0, fuse_rows=0) -> _Params:
     p = _Params()
     _check(load_library().spmm_default_params(ctypes.byref(p)))
     p.nw, p.nt, p.bw, p.split_nnz, p.window, p.preorder, p.seed = nw, nt, bw, split_nnz, window, preorder, seed
+    p.fuse_rows = fuse_rows
     return p
 
 
@@ -204,6 +206,13 @@ class SpMM:
         _check(load_library().spmm_get_info(self._h, out.ctypes.data))
         return dict(empty_rows=int(out[0]), whole_rows=int(out[1]), split_rows=int(out[2]), chunks=int(out[3]),
                     max_row_nnz=int(out[4]))
+
+    def schedule_info(self) -> dict:
+        """The a7 run schedule of the most recent run (spmm_get_schedule_info)."""
+        out = np.empty(6, dtype=np.int64)
+        _check(load_library().spmm_get_schedule_info(self._h, out.ctypes.data))
+        return dict(rows_per_task=int(out[0]), fuse=int(out[1]), tasks=int(out[2]), groups=int(out[3]),
+                    records=int(out[4]), fused_nnz=int(out[5]))
 
     def features(self, current_order=False, nw=32, nt=32, bw=32, stream=None) -> np.ndarray:
         out = np.empty(24, dtype=np.float64)

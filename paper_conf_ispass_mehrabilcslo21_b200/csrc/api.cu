@@ -97,9 +97,9 @@ spmm_status check_device(spmm_ctx *h) {
 
 spmm_status check_params(const spmm_params &p) {
     if (p.nw <= 0 || p.nw > 1024 || p.nt <= 0 || p.bw <= 0 || p.split_nnz < 1 || p.window < 0 ||
-        (p.window % p.nw) != 0 || (p.preorder != 0 && p.preorder != 1))
+        (p.window % p.nw) != 0 || (p.preorder != 0 && p.preorder != 1) || p.fuse_rows < 0 || p.fuse_rows > 2)
         return fail(SPMM_ERR_INVALID_ARG, "invalid spmm_params (nw/nt/bw > 0, nw <= 1024, split_nnz >= 1, "
-                                          "window >= 0 and a multiple of nw, preorder in {0,1})");
+                                          "window >= 0 and a multiple of nw, preorder in {0,1}, fuse_rows in {0,1,2})");
     return SPMM_OK;
 }
 
@@ -257,6 +257,18 @@ spmm_status spmm_get_info(spmm_handle h, int64_t out[5]) {
     out[2] = h->rc.n_long;
     out[3] = h->rc.n_chunks;
     out[4] = h->max_row_nnz;
+    return SPMM_OK;
+}
+
+spmm_status spmm_get_schedule_info(spmm_handle h, int64_t out[6]) {
+    if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    const Schedule &S = h->sched;
+    out[0] = S.rpw;
+    out[1] = S.rpw ? S.fuse : 1;
+    out[2] = S.rpw ? S.n_tasks : 0;
+    out[3] = S.rpw ? S.n_groups : 0;
+    out[4] = S.rpw ? S.n_records : 0;
+    out[5] = S.rpw ? S.fused_nnz : 0;
     return SPMM_OK;
 }
 

@@ -66,8 +66,21 @@ struct RowClasses {
 // non-empty short rows of the permuted order, or RPW consecutive chunks of one long row (a chunk group,
 // reduced across the warp into one partial).  Units: int4 (start, len, dst, 0); dst >= 0: C row,
 // dst == INT_MIN: padding, dst < 0: chunk group -> partial slot -(dst+1).
+// Row fusion (spmm_params.fuse_rows): the short rows of a run are taken R consecutive positions at a time
+// (a fusion group); the group's unit walks the sorted UNION of the R rows' columns once, so a B row shared
+// by several of them is loaded once and feeds every member's accumulator (each member still accumulates its
+// own terms in ascending column order: the rounding of every row is unchanged).  Records: R = 2 -> int4
+// (col, mask, v0, v1); R = 4 -> 2 x int4 (col, mask, v0, v1, v2, v3, 0, 0); mask bit r = row r has the column.
+// Fused unit: int4 (first record, union length, group id, 1); gdst[group * R + r] = C row of member r.
 struct Schedule {
     int32_t rpw = 0;          // 0 = not built
+    int32_t fuse_req = 1;     // R the schedule was requested with (1 = none)
+    int32_t fuse = 1;         // R actually used (1 = no fused units)
+    int64_t n_groups = 0;     // fusion groups
+    int64_t n_records = 0;    // union records over all groups
+    int64_t fused_nnz = 0;    // nnz of the rows in fusion groups
+    DevBuf recs;              // int4[n_records * (R / 2)]
+    DevBuf gdst;              // int32[n_groups * R]
     int64_t n_tasks = 0;
     DevBuf units;             // int4[n_tasks * rpw]
     int64_t n_long = 0;

@@ -218,6 +218,104 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
     }
 }
 
+// A fused unit (row fusion, Schedule): the G lanes of group g walk the sorted union of the columns of R
+// consecutive rows once.  Per union record the group broadcasts (col, mask, v_0..v_{R-1}) with R + 2
+// shuffles, loads the B row once (V vectors per lane) and feeds member r's accumulator with v_r where mask
+// bit r is set (predicated FFMA2: a member without the column adds nothing, so each member's accumulator is
+// the same sequential ascending-column chain as in spmm_unit -- bit-identical C).  Stores: C[gdst[r]].
+template <int R> struct RecT;
+template <> struct RecT<2> { int4 a; };
+template <> struct RecT<4> { int4 a, b; };
+__device__ __forceinline__ RecT<2> ld_rec(const RecT<2> *p) { return RecT<2>{__ldg(&p->a)}; }
+__device__ __forceinline__ RecT<4> ld_rec(const RecT<4> *p) { return RecT<4>{__ldg(&p->a), __ldg(&p->b)}; }
+__device__ __forceinline__ int rec_word(const RecT<2> &r, int i) {
+    return i == 0 ? r.a.x : i == 1 ? r.a.y : i == 2 ? r.a.z : r.a.w;
+}
+__device__ __forceinline__ int rec_word(const RecT<4> &r, int i) {
+    return i == 0 ? r.a.x : i == 1 ? r.a.y : i == 2 ? r.a.z : i == 3 ? r.a.w : i == 4 ? r.b.x : r.b.y;
+}
+__device__ __forceinline__ RecT<2> rec_zero(RecT<2>) { return RecT<2>{make_int4(0, 0, 0, 0)}; }
+__device__ __forceinline__ RecT<4> rec_zero(RecT<4>) { return RecT<4>{make_int4(0, 0, 0, 0), make_int4(0, 0, 0, 0)}; }
+
+template <int V, int G, int R, int U, class VT>
+__device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const int gl, const int col0,
+                                                const bool (&colok)[V], const RecT<R> *__restrict__ recs,
+                                                const int32_t *__restrict__ gdst, const VT *__restrict__ BV,
+                                                VT *__restrict__ CV, const int32_t KV) {
+    constexpr int BATCH = G >= 8 ? G : 8;        // records per group per batch
+    constexpr int PL = BATCH / G;                // records held per lane
+    const int32_t start = u.x, len = u.y, gid = u.z;
+    const int32_t maxlen = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)len);
+    VT acc[R][V];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+        for (int v = 0; v < V; ++v) vzero(acc[r][v]);
+    RecT<R> cur[PL];
+#pragma unroll
+    for (int p = 0; p < PL; ++p) {
+        const int32_t o = p * G + gl;
+        cur[p] = o < len ? ld_rec(recs + start + o) : rec_zero(RecT<R>{});
+    }
+    for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
+        RecT<R> nxt[PL];
+#pragma unroll
+        for (int p = 0; p < PL; ++p) {
+            const int32_t o = b0 + BATCH + p * G + gl;
+            nxt[p] = o < len ? ld_rec(recs + start + o) : rec_zero(RecT<R>{});
+        }
+#pragma unroll
+        for (int q0 = 0; q0 < BATCH; q0 += U) {
+            int32_t col[U];
+            uint32_t mask[U];
+            float a[U][R];
+#pragma unroll
+            for (int w = 0; w < U; ++w) {
+                const int qq = q0 + w;
+                const int src = g * G + (qq % G);
+                col[w] = __shfl_sync(0xffffffffu, rec_word(cur[qq / G], 0), src);
+                mask[w] = (uint32_t)__shfl_sync(0xffffffffu, rec_word(cur[qq / G], 1), src);
+#pragma unroll
+                for (int r = 0; r < R; ++r)
+                    a[w][r] = __int_as_float(__shfl_sync(0xffffffffu, rec_word(cur[qq / G], 2 + r), src));
+            }
+            const int32_t rem = len - (b0 + q0);
+            if (rem > 0) {
+                VT x[U][V];
+#pragma unroll
+                for (int w = 0; w < U; ++w) {
+                    const VT *b = BV + (size_t)col[w] * KV + col0;
+#pragma unroll
+                    for (int v = 0; v < V; ++v) {
+                        if (colok[v] && w < rem) x[w][v] = ld_b<0>(b + v * G, 0);
+                        else vzero(x[w][v]);
+                    }
+                }
+#pragma unroll
+                for (int w = 0; w < U; ++w)
+#pragma unroll
+                    for (int r = 0; r < R; ++r)
+                        if (w < rem && ((mask[w] >> r) & 1u))
+#pragma unroll
+                            for (int v = 0; v < V; ++v) vfma(a[w][r], x[w][v], acc[r][v]);
+            }
+        }
+#pragma unroll
+        for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
+    }
+    if (gid >= 0) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int32_t dst = __ldg(gdst + (size_t)gid * R + r);
+            if (dst >= 0) {
+#pragma unroll
+                for (int v = 0; v < V; ++v)
+                    if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[r][v]);
+            }
+        }
+    }
+}
+
 // Kernel mode 1 (default): row-group SpMM over the a7 warp-task list.
 // V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
 // VAR bit 0: L2 cache-policy hints (LD 1); bit 1: U = 4 nnz per step for V = 4.
@@ -267,11 +365,17 @@ __device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *g
     return __shfl_sync(0xffffffffu, task, 0);
 }
 
-template <int V, int G, bool MASK, int SCHED, int VAR, int W>
-__global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
+// FR > 1: the kernel also runs fused tasks (row fusion, Schedule) -- a task's type is its first unit's w
+// field (1 = fused), uniform over the warp by construction.
+// VAR bit 2: __launch_bounds__ minimum of 4 CTAs per SM (<= 64 registers); bit 3: two-deep task pipeline
+// with an L2 prefetch of the next task's (col, val) / record range (prefetch.global.L2) issued one task ahead.
+template <int V, int G, bool MASK, int SCHED, int VAR, int W, int FR = 1, int FU = 2>
+__global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 3 : 2) : ((VAR & 4) ? 4 : 3)) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
-                                                       unsigned int *__restrict__ counter) {
+                                                       unsigned int *__restrict__ counter,
+                                                       const int4 *__restrict__ recs,
+                                                       const int32_t *__restrict__ gdst) {
     using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
     constexpr int CTV = V * G;
@@ -299,20 +403,59 @@ __global__ void __launch_bounds__(SPMM_THREADS, 3) k_spmm(const int4 *__restrict
         if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
         tk = __shfl_sync(0xffffffffu, tk, 0);
     }
+    constexpr bool PF = (VAR & 8) != 0 && SCHED == 0;
     int64_t t = tk;
     int4 u = t < n_tasks ? __ldg(units + t * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+    int64_t t1 = 0;
+    int4 u1 = make_int4(0, 0, NOSTORE, 0);
+    if (PF) {
+        if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+        t1 = __shfl_sync(0xffffffffu, tk, 0);
+        u1 = t1 < n_tasks ? __ldg(units + t1 * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+    }
     while (t < n_tasks) {
         // claim and fetch the next task first, so its latency hides behind this one
         int64_t t_next;
-        if (SCHED == 1) {
-            t_next = claim_task(&q, counter + blockIdx.y, lane);
-        } else {
+        int4 u_next;
+        if (PF) {
+            // two-deep: u1 (fetched one task ago) is in registers -- prefetch its A range into L2, then
+            // claim the task after it
+            if (t1 < n_tasks && u1.y > 0) {
+                const bool f1 = FR > 1 && u1.w == 1;
+                const int rb = f1 ? 16 * (FR / 2) : 8;
+                const char *lo = f1 ? reinterpret_cast<const char *>(recs) + (size_t)u1.x * rb
+                                    : reinterpret_cast<const char *>(cv) + (size_t)u1.x * 8;
+                const size_t l0 = reinterpret_cast<uintptr_t>(lo) >> 7;
+                const size_t l1 = (reinterpret_cast<uintptr_t>(lo) + (size_t)u1.y * rb - 1) >> 7;
+                for (size_t l = l0 + gl; l <= l1; l += G)
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(reinterpret_cast<const void *>(l << 7)));
+            }
             if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
-            t_next = __shfl_sync(0xffffffffu, tk, 0);
+            const int64_t t2 = __shfl_sync(0xffffffffu, tk, 0);
+            const int4 u2 = t2 < n_tasks ? __ldg(units + t2 * RPW + g) : make_int4(0, 0, NOSTORE, 0);
+            t_next = t1;
+            u_next = u1;
+            t1 = t2;
+            u1 = u2;
+        } else {
+            if (SCHED == 1) {
+                t_next = claim_task(&q, counter + blockIdx.y, lane);
+            } else {
+                if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+                t_next = __shfl_sync(0xffffffffu, tk, 0);
+            }
+            u_next = t_next < n_tasks ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
         }
-        const int4 u_next = t_next < n_tasks ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
-        spmm_unit<V, G, U, LD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4),
-                               KV, reinterpret_cast<VT *>(P4), pol_b, pol_a);
+        bool fused = false;
+        if (FR > 1) fused = __shfl_sync(0xffffffffu, u.w, 0) == 1;
+        if (FR > 1 && fused) {
+            spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU>(u, g, gl, col0, colok,
+                                                     reinterpret_cast<const RecT<(FR > 1 ? FR : 2)> *>(recs), gdst,
+                                                     reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV);
+        } else {
+            spmm_unit<V, G, U, LD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
+                                   reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), pol_b, pol_a);
+        }
         t = t_next;
         u = u_next;
     }
@@ -518,13 +661,14 @@ __global__ void k_fill_short(const int32_t *is_short, const int32_t *sp, const i
 // row length (and RPW), not on the row's position: C stays bit-identical under every permutation.
 __global__ void k_fill_long(const int32_t *lpos, int64_t n_long, const int32_t *sp, const int32_t *taskbase,
                             const int32_t *pslot_ptr, const int32_t *rowptr, const int32_t *perm, int32_t rpw,
-                            int4 *units, int32_t *long_dst) {
+                            int32_t fr, int4 *units, int32_t *long_dst) {
     const int lane = threadIdx.x & 31;
     for (int64_t k = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < n_long;
          k += ((int64_t)gridDim.x * blockDim.x) >> 5) {
         const int32_t p = lpos[k];
         const int32_t s_k = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
-        const int64_t t0 = (int64_t)taskbase[k] + (s_k + rpw - 1) / rpw;
+        const int32_t su = (s_k + fr - 1) / fr;          // short units before it (rows, or fusion groups)
+        const int64_t t0 = (int64_t)taskbase[k] + (su + rpw - 1) / rpw;
         const int32_t a = rowptr[p], len = rowptr[p + 1] - a;
         const int32_t ng = pslot_ptr[k + 1] - pslot_ptr[k];
         const int32_t nch = ng * rpw, base = len / nch, extra = len % nch;
@@ -540,11 +684,126 @@ __global__ void k_fill_int4(int4 *a, int64_t n, int4 v) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) a[i] = v;
 }
 
+// ---- row fusion (Schedule) ------------------------------------------------------------------------
+// per segment k: fusion groups ng_k = ceil(s_k / R) of its short-row run; tasks = ceil(ng_k / RPW) + chunk groups
+__global__ void k_segment_counts_fused(const int32_t *lpos, int64_t n_long, const int32_t *sp, int32_t n_short,
+                                       const int32_t *rowptr, int32_t split, int32_t rpw, int32_t R, int32_t *tasks,
+                                       int32_t *groups, int32_t *ngroups) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k <= n_long; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t before = k > 0 ? sp[lpos[k - 1]] : 0;
+        const int32_t upto = k < n_long ? sp[lpos[k]] : n_short;
+        const int32_t ng = (upto - before + R - 1) / R;
+        int32_t nch = 0;
+        if (k < n_long) {
+            const int32_t len = rowptr[lpos[k] + 1] - rowptr[lpos[k]];
+            nch = (len + split - 1) / split;
+        }
+        const int32_t gk = (nch + rpw - 1) / rpw;
+        tasks[k] = (ng + rpw - 1) / rpw + gk;
+        groups[k] = gk;
+        ngroups[k] = ng;
+    }
+}
+
+// member slots of the fusion groups: gpos[g * R + r] = position of member r (-1: none), gseg[g] = segment
+__global__ void k_group_members(const int32_t *is_short, const int32_t *sp, const int32_t *lidx, const int32_t *lpos,
+                                const int32_t *gbase, int64_t M, int32_t R, int32_t *gpos, int32_t *gseg) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        if (!is_short[p]) continue;
+        const int32_t k = lidx[p];
+        const int32_t idx = sp[p] - (k > 0 ? sp[lpos[k - 1]] : 0);
+        const int64_t g = (int64_t)gbase[k] + idx / R;
+        gpos[g * R + idx % R] = (int32_t)p;
+        if (idx % R == 0) gseg[g] = k;
+    }
+}
+
+// R-way merge of the members' sorted column lists (strictly increasing within a row, A15).  FILL = false:
+// ucnt[g] = union length, gnnz[g] = sum of member lengths; FILL = true: write the records at rbase[g] and
+// the members' C rows (perm) to gdst.
+template <bool FILL>
+__global__ void k_union(const int32_t *gpos, int64_t n_groups, int32_t R, const int32_t *rowptr, const int2 *cv,
+                        const int32_t *perm, int32_t *ucnt, int32_t *gnnz, const int32_t *rbase, int4 *recs,
+                        int32_t *gdst) {
+    for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < n_groups; g += (int64_t)gridDim.x * blockDim.x) {
+        int32_t j[4], e[4], c[4];
+        int32_t tot = 0;
+        for (int r = 0; r < 4; ++r) {
+            const int32_t p = r < R ? gpos[g * R + r] : -1;
+            j[r] = p >= 0 ? rowptr[p] : 0;
+            e[r] = p >= 0 ? rowptr[p + 1] : 0;
+            c[r] = j[r] < e[r] ? cv[j[r]].x : INT_MAX;
+            tot += e[r] - j[r];
+            if (FILL && r < R) gdst[g * R + r] = p >= 0 ? perm[p] : NOSTORE;
+        }
+        int32_t n = 0;
+        int4 *out = FILL ? recs + (int64_t)rbase[g] * (R / 2) : nullptr;
+        for (;;) {
+            const int32_t m = min(min(c[0], c[1]), min(c[2], c[3]));
+            if (m == INT_MAX) break;
+            int32_t mask = 0, v[4] = {0, 0, 0, 0};
+            for (int r = 0; r < 4; ++r) {
+                if (c[r] == m) {
+                    mask |= 1 << r;
+                    v[r] = cv[j[r]].y;
+                    ++j[r];
+                    c[r] = j[r] < e[r] ? cv[j[r]].x : INT_MAX;
+                }
+            }
+            if (FILL) {
+                if (R == 2) {
+                    out[n] = make_int4(m, mask, v[0], v[1]);
+                } else {
+                    out[2 * n] = make_int4(m, mask, v[0], v[1]);
+                    out[2 * n + 1] = make_int4(v[2], v[3], 0, 0);
+                }
+            }
+            ++n;
+        }
+        if (!FILL) {
+            ucnt[g] = n;
+            gnnz[g] = tot;
+        }
+    }
+}
+
+// Fusion groups -> fused units.  As for rows (k_fill_short): the groups of a segment are cut into windows of
+// `win` consecutive groups, inside which they are placed by descending union length (ties: group id).
+__global__ void k_fill_fused(const int32_t *gseg, int64_t n_groups, const int32_t *gbase, const int32_t *ngroups,
+                             const int32_t *taskbase, const int32_t *ucnt, const int32_t *rbase, int32_t rpw,
+                             int32_t win, int4 *units) {
+    for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < n_groups; g += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t k = gseg[g];
+        const int32_t g0 = gbase[k];
+        int32_t idx = (int32_t)(g - g0);
+        const int32_t len = ucnt[g];
+        if (win > 0) {
+            const int32_t w0 = g0 + (idx / win) * win;
+            const int32_t w1 = min(w0 + win, g0 + ngroups[k]);
+            int32_t rank = 0;
+            for (int32_t q = w0; q < w1; ++q) {
+                const int32_t lq = ucnt[q];
+                rank += (lq > len) || (lq == len && q < g);
+            }
+            idx = (idx / win) * win + rank;
+        }
+        const int64_t task = (int64_t)taskbase[k] + idx / rpw;
+        units[task * rpw + idx % rpw] = make_int4(rbase[g], len, (int32_t)g, 1);
+    }
+}
+
 inline unsigned g1(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 32)); }
 
-spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
+// R > 1: row fusion requested (fuse_rows 0 = auto: keep it only when the unions hold <= 3/4 of the fused
+// rows' nnz; 2 = always).  Falls back to R = 1 (plain row units) otherwise.
+spmm_status build_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s) {
     Schedule &S = h->sched;
     S.rpw = 0;
+    S.fuse_req = R;
+    S.fuse = 1;
+    S.n_groups = S.n_records = S.fused_nnz = 0;
+    S.recs.release();
+    S.gdst.release();
     const int64_t M = h->M;
     const int32_t split = h->params.split_nnz;
     const int32_t *rowptr = h->rowptr_p.as<int32_t>();
@@ -575,9 +834,59 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
     SPMM_TRY(groups.alloc((n_long + 1) * sizeof(int32_t), s));
     SPMM_TRY(taskbase.alloc((n_long + 2) * sizeof(int32_t), s));
     SPMM_TRY(S.pslot_ptr.alloc((n_long + 2) * sizeof(int32_t), s));
-    k_segment_counts<<<g1(n_long + 1), 256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), n_short, rowptr,
-                                                    split, rpw, tasks.as<int32_t>(), groups.as<int32_t>());
-    SPMM_CUDA(cudaGetLastError());
+    static const int win_env = [] { const char *e = getenv("SPMM_SORT_WIN"); return e ? atoi(e) : 32; }();
+    const int32_t win = win_env <= 0 ? 0 : (int32_t)ceil_div(win_env, rpw) * rpw;
+    // row fusion: groups of R consecutive short rows of each run, their column unions
+    DevBuf ngroups, gbase, gpos, gseg, ucnt, gnnz, rbase;
+    int32_t n_fgroups = 0;
+    if (R > 1 && n_short > 0) {
+        SPMM_TRY(ngroups.alloc((n_long + 1) * sizeof(int32_t), s));
+        SPMM_TRY(gbase.alloc((n_long + 2) * sizeof(int32_t), s));
+        k_segment_counts_fused<<<g1(n_long + 1), 256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), n_short,
+                                                              rowptr, split, rpw, R, tasks.as<int32_t>(),
+                                                              groups.as<int32_t>(), ngroups.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        SPMM_TRY(exclusive_scan_i32(ngroups.as<int32_t>(), gbase.as<int32_t>(), n_long + 1, &n_fgroups, s));
+        SPMM_TRY(gpos.alloc((size_t)n_fgroups * R * sizeof(int32_t), s));
+        SPMM_TRY(gseg.alloc((size_t)n_fgroups * sizeof(int32_t), s));
+        SPMM_TRY(ucnt.alloc((size_t)(n_fgroups + 1) * sizeof(int32_t), s));
+        SPMM_TRY(gnnz.alloc((size_t)(n_fgroups + 1) * sizeof(int32_t), s));
+        SPMM_TRY(rbase.alloc((size_t)(n_fgroups + 1) * sizeof(int32_t), s));
+        SPMM_CUDA(cudaMemsetAsync(gpos.p, 0xff, (size_t)n_fgroups * R * sizeof(int32_t), s));
+        k_group_members<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), pl.as<int32_t>(), lpos.as<int32_t>(),
+                                              gbase.as<int32_t>(), M, R, gpos.as<int32_t>(), gseg.as<int32_t>());
+        k_union<false><<<g1(n_fgroups), 256, 0, s>>>(gpos.as<int32_t>(), n_fgroups, R, rowptr, h->cv_p.as<int2>(),
+                                                      nullptr, ucnt.as<int32_t>(), gnnz.as<int32_t>(), nullptr,
+                                                      nullptr, nullptr);
+        SPMM_CUDA(cudaGetLastError());
+        int32_t n_rec = 0, n_fnnz = 0;
+        SPMM_TRY(exclusive_scan_i32(gnnz.as<int32_t>(), rbase.as<int32_t>(), n_fgroups, &n_fnnz, s));
+        SPMM_TRY(exclusive_scan_i32(ucnt.as<int32_t>(), rbase.as<int32_t>(), n_fgroups, &n_rec, s));
+        // auto: keep fusion when the unions save enough B-row loads to pay for the wider records and the
+        // predicated FMAs (measured break-even: union / nnz ~0.6 at R = 4, ~0.75 at R = 2)
+        const int64_t num = 3, den = R == 4 ? 5 : 4;
+        const bool keep = h->params.fuse_rows == 2 || (int64_t)n_rec * den <= (int64_t)n_fnnz * num;
+        if (keep) {
+            S.fuse = R;
+            S.n_groups = n_fgroups;
+            S.n_records = n_rec;
+            S.fused_nnz = n_fnnz;
+            SPMM_TRY(S.recs.alloc(std::max<int64_t>((int64_t)n_rec * (R / 2), 1) * sizeof(int4), s));
+            SPMM_TRY(S.gdst.alloc(std::max<int64_t>((int64_t)n_fgroups * R, 1) * sizeof(int32_t), s));
+            k_union<true><<<g1(n_fgroups), 256, 0, s>>>(gpos.as<int32_t>(), n_fgroups, R, rowptr, h->cv_p.as<int2>(),
+                                                         h->perm.as<int32_t>(), nullptr, nullptr, rbase.as<int32_t>(),
+                                                         S.recs.as<int4>(), S.gdst.as<int32_t>());
+            SPMM_CUDA(cudaGetLastError());
+        } else {
+            n_fgroups = 0;
+        }
+    }
+    const int32_t fr = S.fuse;
+    if (fr == 1) {
+        k_segment_counts<<<g1(n_long + 1), 256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), n_short, rowptr,
+                                                        split, rpw, tasks.as<int32_t>(), groups.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
     int32_t n_tasks = 0, n_groups = 0;
     SPMM_TRY(exclusive_scan_i32(tasks.as<int32_t>(), taskbase.as<int32_t>(), n_long + 1, &n_tasks, s));
     SPMM_TRY(exclusive_scan_i32(groups.as<int32_t>(), S.pslot_ptr.as<int32_t>(), n_long + 1, &n_groups, s));
@@ -589,18 +898,24 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
     if (n_tasks > 0) {
         k_fill_int4<<<g1((int64_t)n_tasks * rpw), 256, 0, s>>>(S.units.as<int4>(), (int64_t)n_tasks * rpw,
                                                                 make_int4(0, 0, NOSTORE, 0));
-        static const int win_env = [] { const char *e = getenv("SPMM_SORT_WIN"); return e ? atoi(e) : 32; }();
-        const int32_t win = win_env <= 0 ? 0 : (int32_t)ceil_div(win_env, rpw) * rpw;
-        DevBuf slen;
-        SPMM_TRY(slen.alloc(std::max(n_short, 1) * sizeof(int32_t), s));
-        k_short_len<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), rowptr, M, slen.as<int32_t>());
-        k_fill_short<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), pl.as<int32_t>(), lpos.as<int32_t>(),
-                                           taskbase.as<int32_t>(), rowptr, h->perm.as<int32_t>(), slen.as<int32_t>(),
-                                           n_short, n_long, M, rpw, win, S.units.as<int4>());
+        if (fr > 1) {
+            if (n_fgroups > 0)
+                k_fill_fused<<<g1(n_fgroups), 256, 0, s>>>(gseg.as<int32_t>(), n_fgroups, gbase.as<int32_t>(),
+                                                           ngroups.as<int32_t>(), taskbase.as<int32_t>(),
+                                                           ucnt.as<int32_t>(), rbase.as<int32_t>(), rpw, win,
+                                                           S.units.as<int4>());
+        } else {
+            DevBuf slen;
+            SPMM_TRY(slen.alloc(std::max(n_short, 1) * sizeof(int32_t), s));
+            k_short_len<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), rowptr, M, slen.as<int32_t>());
+            k_fill_short<<<g1(M), 256, 0, s>>>(fs.as<int32_t>(), ps.as<int32_t>(), pl.as<int32_t>(), lpos.as<int32_t>(),
+                                               taskbase.as<int32_t>(), rowptr, h->perm.as<int32_t>(), slen.as<int32_t>(),
+                                               n_short, n_long, M, rpw, win, S.units.as<int4>());
+        }
         if (n_long > 0)
             k_fill_long<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)n_long * 32, 256), 148 * 32)),
                           256, 0, s>>>(lpos.as<int32_t>(), n_long, ps.as<int32_t>(), taskbase.as<int32_t>(),
-                                       S.pslot_ptr.as<int32_t>(), rowptr, h->perm.as<int32_t>(), rpw,
+                                       S.pslot_ptr.as<int32_t>(), rowptr, h->perm.as<int32_t>(), rpw, fr,
                                        S.units.as<int4>(), S.long_dst.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
     }
@@ -609,7 +924,7 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, cudaStream_t s) {
 }
 
 using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
-                            unsigned int *);
+                            unsigned int *, const int4 *, const int32_t *);
 
 template <int V, bool MASK, int SCHED, int VAR>
 SpmmKernel pick_g(int G) {
@@ -649,9 +964,62 @@ SpmmKernel pick_w8(int V, int G) {
     }
 }
 
+// fused-capable variants (row fusion, W = 8, per-warp claiming, VAR 0): R rows per group, U records per
+// inner step (U*V B loads in flight per lane, as in the unfused kernel).  R = 4 at V = 1 (SPMM_FUSE_R=2: R = 2).
+int fuse_r_env() {
+    static const int r = [] { const char *e = getenv("SPMM_FUSE_R"); return e ? atoi(e) : 4; }();
+    return r == 2 ? 2 : 4;
+}
+int fuse_u_env() {
+    static const int u = [] { const char *e = getenv("SPMM_FUSE_U"); return e ? atoi(e) : 4; }();
+    return u == 2 ? 2 : 4;
+}
+template <int VAR>
+SpmmKernel pick_w8_fused_v(int V, int G, int R) {
+    if (V == 1 && fuse_u_env() == 2) {     // U = 2 records per step at 3 CTAs/SM (A/B: SPMM_FUSE_U=2)
+        switch (R * 10 + G) {
+            case 24: return k_spmm<1, 4, false, 0, VAR, 8, 2, 2>;
+            case 28: return k_spmm<1, 8, false, 0, VAR, 8, 2, 2>;
+            case 44: return k_spmm<1, 4, false, 0, VAR, 8, 4, 2>;
+            case 48: return k_spmm<1, 8, false, 0, VAR, 8, 4, 2>;
+            default: return nullptr;
+        }
+    }
+    switch (R * 1000 + V * 100 + G) {
+        case 2104: return k_spmm<1, 4, false, 0, VAR, 8, 2, 4>;
+        case 2108: return k_spmm<1, 8, false, 0, VAR, 8, 2, 4>;
+        case 2208: return k_spmm<2, 8, false, 0, VAR, 8, 2, 2>;
+        case 4104: return k_spmm<1, 4, false, 0, VAR, 8, 4, 4>;
+        case 4108: return k_spmm<1, 8, false, 0, VAR, 8, 4, 4>;
+        default: return nullptr;
+    }
+}
+// The fused kernel runs at 2 CTAs/SM (its R*V accumulators need > 80 registers), so it always takes the
+// next-task L2 prefetch (VAR bit 3): measured 0.336 -> 0.321 ms at C2, K = 64 (the unfused kernel at 3
+// CTAs/SM gains nothing from it).  SPMM_VARIANT=16 turns it off (A/B).
+SpmmKernel pick_w8_fused(int var, int V, int G, int R) {
+    return (var & 16) ? pick_w8_fused_v<0>(V, G, R) : pick_w8_fused_v<8>(V, G, R);
+}
+int fuse_rows_for(int V, int G) {
+    const int R = V == 1 ? fuse_r_env() : 2;
+    return pick_w8_fused(0, V, G, R) ? R : 1;
+}
+
+SpmmKernel pick_w8v(int var, int V, int G) {
+    switch (var) {
+        case 1: return pick_w8<1>(V, G);
+        case 4: return pick_w8<4>(V, G);
+        case 8: return pick_w8<8>(V, G);
+        case 12: return pick_w8<12>(V, G);
+        default: return pick_w8<0>(V, G);
+    }
+}
+
 struct Config {
     SpmmKernel kern;
     int V, G, tiles, W;
+    SpmmKernel kern_fused = nullptr;   // the same geometry with fused tasks (nullptr: no row fusion)
+    int R = 1;
 };
 
 // Lane geometry.  W = 8 (one 256-bit load per lane and vector) when K % 8 == 0 and B, C are 32-byte aligned:
@@ -661,15 +1029,23 @@ struct Config {
 // measured to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
 Config choose(int32_t K4, int sched, int var, bool w8ok) {
     if (w8ok && sched == 0 && (var & 2) == 0 && K4 % 2 == 0) {
+        const int vu = var & 15;   // bit 4 only selects the fused kernel's prefetch
         const int32_t K8 = K4 / 2;
         for (int G : {8, 4})
             for (int V : {1, 2, 4})
                 if (V * G == K8) {
-                    SpmmKernel k = var ? pick_w8<1>(V, G) : pick_w8<0>(V, G);
-                    if (k) return {k, V, G, 1, 8};
+                    SpmmKernel k = pick_w8v(vu, V, G);
+                    if (k) {
+                        Config c{k, V, G, 1, 8};
+                        if ((vu & 3) == 0) {
+                            c.R = fuse_rows_for(V, G);
+                            c.kern_fused = c.R > 1 ? pick_w8_fused(var, V, G, c.R) : nullptr;
+                        }
+                        return c;
+                    }
                 }
         for (int G : {16, 32})
-            if (4 * G == K8) return {var ? pick_w8<1>(4, G) : pick_w8<0>(4, G), 4, G, 1, 8};
+            if (4 * G == K8) return {pick_w8v(vu, 4, G), 4, G, 1, 8};
     }
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
@@ -726,7 +1102,7 @@ static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, 
     static const int ppt = std::max(1, env_int("SPMM_AFF_PPT", 256));
     static const int ld = env_int("SPMM_AFF_LD", 2);
     const int32_t rpw = W == 8 ? 8 : 4;                    // G = 4 (W = 8) or 8 (W = 4)
-    if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
+    if (h->sched.rpw != rpw || h->sched.fuse_req != 1) SPMM_TRY(build_schedule(h, rpw, 1, s));
     const Schedule &S = h->sched;
     const int2 *cv = h->cv_p.as<int2>();
     float4 *C4 = reinterpret_cast<float4 *>(C);
@@ -788,8 +1164,12 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
             return launch_aff(h, B, K, C, s, av, aw, launches);
     }
     const int32_t rpw = 32 / cfg.G;
-    if (h->sched.rpw != rpw) SPMM_TRY(build_schedule(h, rpw, s));
+    // row fusion: fuse_rows 1 = off; SPMM_FUSE=0 disables it process-wide (A/B knob)
+    static const int fuse_env = env_int("SPMM_FUSE", 1);
+    const int32_t R = (h->params.fuse_rows != 1 && fuse_env != 0 && cfg.kern_fused) ? cfg.R : 1;
+    if (h->sched.rpw != rpw || h->sched.fuse_req != R) SPMM_TRY(build_schedule(h, rpw, R, s));
     const Schedule &S = h->sched;
+    const SpmmKernel kern = S.fuse > 1 ? cfg.kern_fused : cfg.kern;
     float4 *C4 = reinterpret_cast<float4 *>(C);
     float4 *P4 = nullptr;
     if (S.n_pslots > 0) {
@@ -823,7 +1203,7 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     }
     if (S.n_tasks > 0) {
         int occ = 0;
-        SPMM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, cfg.kern, SPMM_THREADS, 0));
+        SPMM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, SPMM_THREADS, 0));
         occ = std::max(occ, 1);
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(S.n_tasks, SPMM_THREADS / 32),
                                                                       (int64_t)h->num_sms * occ));
@@ -832,9 +1212,9 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
             SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
         SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
         if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
-        cfg.kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
-                                               reinterpret_cast<const float4 *>(B), C4, K4, P4,
-                                               h->counters.as<unsigned int>());
+        kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
+                                           reinterpret_cast<const float4 *>(B), C4, K4, P4,
+                                           h->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
         if (h->timing) {
             SPMM_CUDA(cudaEventRecord(h->ev1, s));

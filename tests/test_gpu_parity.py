@@ -302,6 +302,20 @@ for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_2_1"):
     assert np.all(np.abs(C - ref) <= 1e-5 * bound + 1e-6), pol
     if first is None: first = C
     assert np.array_equal(C.view(np.int32), first.view(np.int32)), pol
+# row fusion forced on a stencil (fused tasks + a split row's chunk tasks in one launch)
+st = syn.stencil27(12, 5, int_values=True)
+rows = [st.colidx[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
+vals = [st.value[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
+rows[100] = list(range(0, st.N, 3)); vals[100] = [1.0 + (t % 3) for t in range(len(rows[100]))]
+st = syn.from_lists(st.M, st.N, rows, vals)
+hs = pkg.SpMM.from_csr(st)
+for K in (32, 64, 128):
+    Bs = syn.dense(st.N, K, 6, int_values=True)
+    refs, _ = oracle.spmm(st, Bs)
+    for pol in ("identity", "cta_aware"):
+        hs.permute(pol, fuse_rows=2)
+        C = hs.run(torch.from_numpy(Bs).cuda()).cpu().numpy()
+        assert np.array_equal(C.astype(np.float64), refs), (K, pol)
 print("OK")
 """
 
@@ -311,10 +325,13 @@ print("OK")
                                  {"SPMM_SORT_WIN": "128"}, {"SPMM_ZERO_SIDE": "0"}, {"SPMM_KERNEL": "3"},
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_V": "2", "SPMM_AFF_LD": "0"},
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
-                                 {"SPMM_W": "4", "SPMM_KERNEL": "3"}])
+                                 {"SPMM_W": "4", "SPMM_KERNEL": "3"}, {"SPMM_VARIANT": "4"}, {"SPMM_VARIANT": "8"},
+                                 {"SPMM_VARIANT": "12"}, {"SPMM_FUSE_R": "2"}, {"SPMM_FUSE": "0"},
+                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}])
 def test_kernel_variants_exact(env):
     """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4, 128-bit lane loads, schedule
-    windows, SM-affine column tiles) are exact on integer inputs and permutation-invariant on real inputs."""
+    windows, SM-affine column tiles, 4 CTAs/SM, next-task L2 prefetch, row fusion R = 2 / off) are exact on
+    integer inputs and permutation-invariant on real inputs."""
     import os
     import subprocess
     import sys
@@ -354,4 +371,65 @@ def test_select_policy_runs():
         assert pol4 in pkg.PAPER4_POLICIES
         h.permute(pol)
         assert np.array_equal(h.perm(), oracle.permute(a, pol, window=1024))
+    h.close()
+
+
+FUSE_GENS = {
+    "stencil16": lambda: syn.stencil27(16, 1003),
+    "stencil_int": lambda: syn.stencil27(13, 1006, int_values=True),
+    "banded": lambda: syn.banded(6000, 24, 40, 1007),
+    "rmat12_natural": lambda: syn.rmat(12, 12, 1000, "natural"),
+    "block": lambda: syn.blockcluster(4099, 9000, 32, 4, 20, 1005),
+}
+
+
+@pytest.mark.parametrize("gen", list(FUSE_GENS))
+@pytest.mark.parametrize("K", [32, 64, 128, 256])
+def test_row_fusion_bit_identical(gen, K):
+    """Row fusion (fuse_rows 0 auto / 2 forced) walks the union of R consecutive rows' columns; every row keeps
+    its own ascending-column FMA chain, so C is bit-identical to the unfused schedule (fuse_rows = 1) and within
+    the north-star tolerance of the oracle, for every policy (including split rows and ragged last groups)."""
+    a = FUSE_GENS[gen]()
+    int_vals = gen.endswith("_int")
+    B = syn.dense(a.N, K, 78, int_values=int_vals)
+    C_ref, bound = oracle.spmm(a, B)
+    h = pkg.SpMM.from_csr(a)
+    for pol in ("identity", "nnz_sort", "cta_aware"):
+        outs = {}
+        for fuse in (1, 0, 2):
+            h.permute(pol, fuse_rows=fuse, split_nnz=16 if pol == "nnz_sort" else 128)
+            C = run_c(h, B)
+            info = h.schedule_info()
+            if fuse == 1:
+                assert info["fuse"] == 1
+            if fuse == 2 and h.info()["whole_rows"] > 0:
+                assert info["fuse"] == {32: 4, 64: 4, 128: 2, 256: 1}[K], info
+                if info["fuse"] > 1:
+                    assert info["groups"] > 0 and info["records"] <= info["fused_nnz"]
+            outs[fuse] = C
+            if int_vals:
+                assert np.array_equal(C.astype(np.float64), C_ref), (gen, K, pol, fuse)
+            else:
+                ok, worst = within_tol(C, C_ref, bound)
+                assert ok, (gen, K, pol, fuse, worst)
+        assert np.array_equal(outs[0].view(np.int32), outs[1].view(np.int32)), (gen, K, pol)
+        assert np.array_equal(outs[2].view(np.int32), outs[1].view(np.int32)), (gen, K, pol)
+    h.close()
+
+
+def test_row_fusion_auto_decision():
+    """Auto fusion engages on a stencil (consecutive rows share 2/3 of their columns) and stays off on a
+    random-label power-law matrix (consecutive rows share almost nothing)."""
+    st = syn.stencil27(20, 1008)
+    h = pkg.SpMM.from_csr(st)
+    h.permute("identity")
+    run_c(h, syn.dense(st.N, 64, 1))
+    info = h.schedule_info()
+    assert info["fuse"] == 4 and info["records"] * 4 <= info["fused_nnz"] * 3, info
+    h.close()
+    rl = syn.rmat(13, 8, 1009, "random-label")
+    h = pkg.SpMM.from_csr(rl)
+    h.permute("identity")
+    run_c(h, syn.dense(rl.N, 64, 1))
+    assert h.schedule_info()["fuse"] == 1
     h.close()
