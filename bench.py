@@ -459,12 +459,19 @@ def main():
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(a_full, B_host.numpy(), K)
-    traffic = None
+    # DRAM bytes of one k_spmm launch on this config from the committed ncu --set full capture (scripts/
+    # collect_profiles.py); the selected policy's capture if there is one, else the closest-timed profiled policy
+    traffic, traffic_from = None, None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(prof):
-        d = json.load(open(prof)).get(f"{args.config}/{best}")
-        if d:
+    if os.path.exists(prof) and world == 1:
+        allp = json.load(open(prof))
+        cands = [p for p in pol_res if f"{args.config}/{p}" in allp]
+        if cands:
+            pick = best if best in cands else min(cands, key=lambda p: abs(pol_res[p]["ms"] - pol_res[best]["ms"]))
+            d = allp[f"{args.config}/{pick}"]
             traffic = d.get("dram_bytes_per_launch")
+            traffic_from = f"ncu --set full of {d.get('kernel', 'k_spmm')} on {args.config}/{pick} ({d.get('round')})"
+
     for pol, r in pol_res.items():
         r["roofline_frac"] = alg_bytes / (r["ms"] * 1e-3) / 1e9 / peak
         r["speedup_vs_identity"] = pol_res["identity"]["ms"] / r["ms"] if "identity" in pol_res else None
@@ -475,9 +482,11 @@ def main():
         "config": {"workload": cfg["desc"], "M": int(meta[:, 0].sum().item()), "N": N, "nnz": nnz_total, "K": K,
                    "policy": best, "window": args.window, "parallelism": f"rows sharded by nnz over {world} GPU(s)",
                    "l2": "256 MiB scratch written between timed steps (L2 flush); B, C also > L2",
-                   "selection": "exhaustive timing over " + ",".join(pol_res)},
+                   "selection": "exhaustive timing over " + ",".join(pol_res),
+                   "schedule": h.schedule_info()},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": traffic, "algorithmic_bytes_per_launch": kern_bytes, "distinct_columns": ncols,
+                     "traffic": traffic, "traffic_from": traffic_from,
+                     "algorithmic_bytes_per_launch": kern_bytes, "distinct_columns": ncols,
                      "kernel": "k_spmm (row-group SpMM, rank 0 shard): CUDA events recorded by the library on the "
                                "launch stream around the kernel (spmm_set_kernel_timing), mean over the timed steps",
                      "kernel_ms": kern_ms, "share_of_step": (kern_ms / statistics.mean(ts)) if kern_ms else None,

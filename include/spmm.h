@@ -75,7 +75,7 @@ typedef struct {
     int32_t fuse_rows;      /* row fusion in spmm_run (a7/a8): 0 = auto -- take the short rows R consecutive
                                positions at a time and walk the union of their columns once (each shared B
                                row loaded once) when the unions hold <= 3/4 of those rows' nnz; 1 = off;
-                               2 = always (where the K geometry has a fused kernel: R = 4 at K = 32/64,
+                               2 = always (where the K geometry has a fused kernel: R = 4 at K = 64,
                                R = 2 at K = 128).  C is bit-identical in every setting.                 */
     uint64_t seed;          /* MinHash seed                                                          */
 } spmm_params;

@@ -454,7 +454,8 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
                                                      reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV);
         } else {
             spmm_unit<V, G, U, LD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
-                                   reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), pol_b, pol_a);
+                                                     reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), pol_b,
+                                                     pol_a);
         }
         t = t_next;
         u = u_next;
@@ -978,18 +979,14 @@ template <int VAR>
 SpmmKernel pick_w8_fused_v(int V, int G, int R) {
     if (V == 1 && fuse_u_env() == 2) {     // U = 2 records per step at 3 CTAs/SM (A/B: SPMM_FUSE_U=2)
         switch (R * 10 + G) {
-            case 24: return k_spmm<1, 4, false, 0, VAR, 8, 2, 2>;
             case 28: return k_spmm<1, 8, false, 0, VAR, 8, 2, 2>;
-            case 44: return k_spmm<1, 4, false, 0, VAR, 8, 4, 2>;
             case 48: return k_spmm<1, 8, false, 0, VAR, 8, 4, 2>;
             default: return nullptr;
         }
     }
     switch (R * 1000 + V * 100 + G) {
-        case 2104: return k_spmm<1, 4, false, 0, VAR, 8, 2, 4>;
         case 2108: return k_spmm<1, 8, false, 0, VAR, 8, 2, 4>;
         case 2208: return k_spmm<2, 8, false, 0, VAR, 8, 2, 2>;
-        case 4104: return k_spmm<1, 4, false, 0, VAR, 8, 4, 4>;
         case 4108: return k_spmm<1, 8, false, 0, VAR, 8, 4, 4>;
         default: return nullptr;
     }
@@ -1000,7 +997,11 @@ SpmmKernel pick_w8_fused_v(int V, int G, int R) {
 SpmmKernel pick_w8_fused(int var, int V, int G, int R) {
     return (var & 16) ? pick_w8_fused_v<0>(V, G, R) : pick_w8_fused_v<8>(V, G, R);
 }
+// Row fusion only where it measured faster: G = 8 lanes per row (K = 64: R = 4, K = 128: R = 2).
+// At K = 32 (G = 4) a B row is one 128-byte line and the 32-byte records cost as much as they save (0.199 ->
+// 0.197 ms at C2, 0.229 ms with the prefetch pipeline).
 int fuse_rows_for(int V, int G) {
+    if (G != 8) return 1;
     const int R = V == 1 ? fuse_r_env() : 2;
     return pick_w8_fused(0, V, G, R) ? R : 1;
 }

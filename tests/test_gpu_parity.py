@@ -403,7 +403,7 @@ def test_row_fusion_bit_identical(gen, K):
             if fuse == 1:
                 assert info["fuse"] == 1
             if fuse == 2 and h.info()["whole_rows"] > 0:
-                assert info["fuse"] == {32: 4, 64: 4, 128: 2, 256: 1}[K], info
+                assert info["fuse"] == {32: 1, 64: 4, 128: 2, 256: 1}[K], info
                 if info["fuse"] > 1:
                     assert info["groups"] > 0 and info["records"] <= info["fused_nnz"]
             outs[fuse] = C
