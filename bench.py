@@ -217,36 +217,45 @@ def run_reference(args):
     }))
 
 
-def shard_inputs(torch, dist, a_full, world, rank, dev, pkg):
+def shard_inputs(torch, dist, a_full, world, rank, dev, pkg, compact=False):
     """Rank 0 holds the generated matrix; every rank gets its nnz-balanced row shard as CUDA tensors
-    (NCCL send/recv for N>1).  Returns (M_r, lo, rowidx, colidx, value) with rowidx rebased to 0."""
+    (NCCL send/recv for N>1).  Returns (M_r, lo, (rowidx, colidx, value), meta, cols) with rowidx rebased to 0.
+    compact (N>1, sharded.py compact_B): the shard's columns are renumbered to their index in its sorted list of
+    distinct columns `cols` (int64, device), so the rank needs only B[cols] (|cols| x K)."""
+    from paper_conf_ispass_mehrabilcslo21_b200.sharded import compact_shard, make_shard, shard_columns
     if rank == 0:
         bounds = pkg.spmm_partition_by_nnz(a_full.rowidx, world)
+        cols_all = [shard_columns(a_full.rowidx, a_full.colidx, bounds, r) for r in range(world)] if compact else None
         meta = torch.tensor([[int(bounds[r + 1] - bounds[r]), int(a_full.rowidx[bounds[r + 1]] - a_full.rowidx[bounds[r]]),
-                              int(bounds[r])] for r in range(world)], dtype=torch.int64, device=dev)
+                              int(bounds[r]), len(cols_all[r]) if compact else a_full.N] for r in range(world)],
+                            dtype=torch.int64, device=dev)
     else:
-        meta = torch.empty((world, 3), dtype=torch.int64, device=dev)
+        meta = torch.empty((world, 4), dtype=torch.int64, device=dev)
     if world > 1:
         dist.broadcast(meta, src=0)
     parts = None
     if rank == 0:
         parts = []
         for r in range(world):
-            lo, hi = int(bounds[r]), int(bounds[r + 1])
-            r0, r1 = int(a_full.rowidx[lo]), int(a_full.rowidx[hi])
-            parts.append((torch.from_numpy(a_full.rowidx[lo:hi + 1] - r0), torch.from_numpy(a_full.colidx[r0:r1]),
-                          torch.from_numpy(a_full.value[r0:r1])))
+            sh = make_shard(a_full.M, a_full.N, a_full.rowidx, a_full.colidx, a_full.value, bounds, r)
+            if compact:
+                sh = compact_shard(sh, cols_all[r])
+            parts.append((torch.from_numpy(sh.rowidx), torch.from_numpy(sh.colidx), torch.from_numpy(sh.value))
+                         + ((torch.from_numpy(cols_all[r]),) if compact else ()))
         for r in range(1, world):
             for t in parts[r]:
                 dist.send(t.to(dev), dst=r)
         mine = tuple(t.to(dev) for t in parts[0])
     else:
-        Mr, nnzr = int(meta[rank, 0]), int(meta[rank, 1])
+        Mr, nnzr, nc = int(meta[rank, 0]), int(meta[rank, 1]), int(meta[rank, 3])
         mine = (torch.empty(Mr + 1, dtype=torch.int64, device=dev), torch.empty(nnzr, dtype=torch.int32, device=dev),
                 torch.empty(nnzr, dtype=torch.float32, device=dev))
+        if compact:
+            mine = mine + (torch.empty(nc, dtype=torch.int64, device=dev),)
         for t in mine:
             dist.recv(t, src=0)
-    return int(meta[rank, 0]), int(meta[rank, 2]), mine, meta
+    cols = mine[3] if compact else None
+    return int(meta[rank, 0]), int(meta[rank, 2]), mine[:3], meta, cols, (cols_all if rank == 0 else None)
 
 
 def main():
@@ -265,6 +274,8 @@ def main():
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-ceiling", action="store_true", help="skip the host LRU model of L2 reuse")
     ap.add_argument("--out", default=None, help="also write the JSON line to this file")
+    ap.add_argument("--b-exchange", default="rows", choices=["rows", "broadcast"],
+                    help="N>1: send each rank only the B rows its shard references (rows) or broadcast all of B")
     args = ap.parse_args()
     assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
     if args.impl == "reference":
@@ -289,15 +300,18 @@ def main():
     t0 = time.perf_counter()
     a_full = make_matrix(cfg) if rank == 0 else None
     gen_s = time.perf_counter() - t0
-    Mr, lo, (rowidx_d, colidx_d, value_d), meta = shard_inputs(torch, dist, a_full, world, rank, dev, pkg)
+    compact = world > 1 and args.b_exchange == "rows"
+    Mr, lo, (rowidx_d, colidx_d, value_d), meta, cols_d, cols_all = shard_inputs(torch, dist, a_full, world, rank,
+                                                                                dev, pkg, compact=compact)
     N = a_full.N if rank == 0 else None
     nN = torch.tensor([N or 0], dtype=torch.int64, device=dev)
     if world > 1:
         dist.broadcast(nN, src=0)
-    N = int(nN.item())
+    N = int(nN.item())                 # global N (B rows)
+    N_loc = int(meta[rank, 3].item()) if compact else N   # B rows this rank holds
     nnz_r = int(colidx_d.numel())
     nnz_total = int(meta[:, 1].sum().item())
-    seen = torch.zeros(N, dtype=torch.bool, device=dev)
+    seen = torch.zeros(N_loc, dtype=torch.bool, device=dev)
     seen[colidx_d.long()] = True
     ncols = int(seen.sum().item())
     del seen
@@ -305,11 +319,23 @@ def main():
     flops = 2.0 * nnz_r * K
     total_flops = 2.0 * nnz_total * K
 
-    # B: drawn on rank 0 (host), broadcast over NCCL to the other ranks (outside the timed region)
+    # B: drawn on rank 0 (host); N>1: broadcast over NCCL, or (--b-exchange rows, default) each rank receives
+    # only the rows its shard references (NCCL send of B[cols_p]; sharded.py compact_B) -- outside the timed region
     B_host = torch.from_numpy(syn.dense(N, K, bseed)) if rank == 0 else None
-    Bd = B_host.to(dev) if rank == 0 else torch.empty((N, K), dtype=torch.float32, device=dev)
-    if world > 1:
-        dist.broadcast(Bd, src=0)
+    if compact:
+        if rank == 0:
+            Bfull = B_host.to(dev)
+            for r in range(1, world):
+                dist.send(Bfull.index_select(0, torch.from_numpy(cols_all[r]).to(dev)).contiguous(), dst=r)
+            Bd = Bfull.index_select(0, cols_d).contiguous()
+            del Bfull
+        else:
+            Bd = torch.empty((N_loc, K), dtype=torch.float32, device=dev)
+            dist.recv(Bd, src=0)
+    else:
+        Bd = B_host.to(dev) if rank == 0 else torch.empty((N, K), dtype=torch.float32, device=dev)
+        if world > 1:
+            dist.broadcast(Bd, src=0)
     Cd = torch.empty((Mr, K), dtype=torch.float32, device=dev)
     flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
 
@@ -317,7 +343,7 @@ def main():
         flush_buf.fill_(1.0)
 
     pkg.use_torch_allocator(True)
-    h = pkg.SpMM(Mr, N, rowidx_d, colidx_d, value_d)
+    h = pkg.SpMM(Mr, N_loc, rowidx_d, colidx_d, value_d)
     torch.cuda.synchronize()
     feat_t0 = time.perf_counter()
     feats = h.features()
@@ -402,16 +428,25 @@ def main():
     # ---- e2e through the public API with host buffers ----
     # N=1: spmm_run_host (H2D of B, SpMM, D2H of C).  N>1: rank 0 H2D of B, NCCL broadcast, SpMM on every
     # shard, D2H of every C shard; max over ranks.
+    # N>1 with per-rank B rows: every rank's step starts from ITS rows of B in pinned host memory (the host keeps
+    # the input partitioned per GPU, prepared outside the timed region like any input) and copies them over its
+    # own PCIe link; with --b-exchange broadcast, rank 0 copies all of B and NCCL broadcasts it.
     Cp = torch.empty((Mr, K), dtype=torch.float32).pin_memory()
-    Bp = B_host.pin_memory() if rank == 0 else None
+    if world == 1 or not compact:
+        Bp = B_host.pin_memory() if rank == 0 else None
+    else:
+        Bp = Bd.cpu().pin_memory()
 
     def e2e_step():
         if world == 1:
             h.run_host(Bp, Cp)
         else:
-            if rank == 0:
+            if compact:
                 Bd.copy_(Bp, non_blocking=True)
-            dist.broadcast(Bd, src=0)
+            else:
+                if rank == 0:
+                    Bd.copy_(Bp, non_blocking=True)
+                dist.broadcast(Bd, src=0)
             h.run(Bd, Cd)
             Cp.copy_(Cd, non_blocking=True)
             torch.cuda.current_stream().synchronize()
@@ -429,26 +464,46 @@ def main():
     e2e_t = torch.tensor([statistics.mean(e2e_ts)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    h2d = int(meta[:, 3].sum().item()) * K * 4 if compact else N * K * 4
     e2e = {"value": total_flops / float(e2e_t.item()) / 1e6, "unit": "GFLOP/s",
-           "h2d_bytes_per_step": int(N * K * 4), "d2h_bytes_per_step": int(int(meta[:, 0].sum().item()) * K * 4),
+           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(int(meta[:, 0].sum().item()) * K * 4),
            "ms_per_step": float(e2e_t.item()),
-           "path": "spmm_run_host" if world == 1 else "H2D(B) on rank 0 + NCCL broadcast + spmm_run + D2H(C shards)"}
+           "path": "spmm_run_host" if world == 1 else
+           ("per-rank H2D of its B rows (pinned) + spmm_run + D2H of its C shard" if compact else
+            "H2D(B) on rank 0 + NCCL broadcast + spmm_run + D2H(C shards)")}
 
-    # ---- cuSPARSE comparator (torch.sparse CSR @ dense -> cusparseSpMM), same inputs, same flush ----
+    # ---- cuSPARSE comparator: cusparseSpMM CSR ALG1/ALG2/ALG3 and the default algorithm, row-major B and C,
+    # best-of (tools/cusparse_ref.cu), same inputs, same L2 flush, rank 0 shard ----
     cus = None
     if not args.no_cusparse and rank == 0:
-        try:
-            A_t = torch.sparse_csr_tensor(rowidx_d, colidx_d.long(), value_d, size=(Mr, N))
-            for _ in range(3):
-                A_t @ Bd
-            cts = time_runs(torch, lambda: A_t @ Bd, max(3, args.policy_steps), flush, stream)
-            cms = statistics.median(cts)
-            cus = {"ms": cms, "gflops": flops / cms / 1e6, "speedup_best_vs_cusparse": cms / pol_res[best]["ms"],
+        import tools
+        rp32 = rowidx_d.to(torch.int32)
+        Cc = torch.empty_like(Cd)
+        h.run(Bd, Cd)                 # our C of the selected policy, for the sanity diff
+        torch.cuda.synchronize()
+        per_alg = {}
+        for alg, name in ((0, "default"), (1, "csr_alg1"), (2, "csr_alg2"), (3, "csr_alg3")):
+            try:
+                cts = tools.cusparse_spmm_times(Mr, N_loc, nnz_r, rp32.data_ptr(), colidx_d.data_ptr(), value_d.data_ptr(),
+                                                Bd.data_ptr(), K, Cc.data_ptr(), alg, max(3, args.policy_steps),
+                                                (flush_buf.data_ptr(), flush_buf.numel() * 4), stream.cuda_stream)
+                torch.cuda.synchronize()
+                # sanity: the library's C against ours (both fp32; reported, not asserted)
+                diff = float((Cc - Cd).abs().max().item())
+                per_alg[name] = {"ms": statistics.median(cts), "max_abs_diff_vs_ours": diff}
+            except Exception as e:  # noqa: BLE001
+                per_alg[name] = {"error": str(e)[:160]}
+        ok = {k: v for k, v in per_alg.items() if "ms" in v}
+        if ok:
+            bname = min(ok, key=lambda k: ok[k]["ms"])
+            cms = ok[bname]["ms"]
+            cus = {"ms": cms, "gflops": flops / cms / 1e6, "best_alg": bname, "per_alg": per_alg,
+                   "speedup_best_vs_cusparse": cms / pol_res[best]["ms"],
                    "speedup_identity_vs_cusparse": cms / pol_res["identity"]["ms"] if "identity" in pol_res else None,
-                   "via": "torch.sparse_csr @ dense (cusparseSpMM, default algorithm), rank 0 shard"}
-            del A_t
-        except Exception as e:  # noqa: BLE001
-            cus = {"error": str(e)[:200]}
+                   "via": "cusparseSpMM (CUSPARSE_SPMM_CSR_ALG1/2/3, default), row-major, best-of, rank 0 shard"}
+        else:
+            cus = {"error": "no cuSPARSE algorithm ran", "per_alg": per_alg}
+        del Cc, rp32
 
     if rank != 0:
         if world > 1:
@@ -481,6 +536,7 @@ def main():
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": cfg["desc"], "M": int(meta[:, 0].sum().item()), "N": N, "nnz": nnz_total, "K": K,
                    "policy": best, "window": args.window, "parallelism": f"rows sharded by nnz over {world} GPU(s)",
+                   "b_exchange": ("per-rank B rows (compact shards)" if compact else "broadcast") if world > 1 else None,
                    "l2": "256 MiB scratch written between timed steps (L2 flush); B, C also > L2",
                    "selection": "exhaustive timing over " + ",".join(pol_res),
                    "schedule": h.schedule_info()},

@@ -8,8 +8,14 @@ One process per GPU (torchrun), torch.distributed for the plumbing:
   4. each rank runs spmm_run on its shard -- C stays row-sharded in original row order;
   5. optionally C is all-gathered (shards padded to the largest shard, gathered, trimmed).
 
-The only data-path collectives are the B broadcast and the optional C all-gather: the SpMM itself
-has no exchange step.  `local_factory` builds the per-rank SpMM object; it defaults to the CUDA
+With compact_B=True a rank holds only the B rows its shard touches: the shard's
+columns are renumbered to their rank in the sorted list cols_p of distinct columns it references (a
+monotone map, so every row keeps its ascending column order and C is bit-identical), and `distribute_B`
+sends each rank B[cols_p] from the source (NCCL point-to-point) instead of broadcasting all N rows --
+|cols_p| / N of the volume, and a B working set that shrinks with P.
+
+The only data-path collectives are the B broadcast (or the per-rank B-row sends) and the optional C
+all-gather: the SpMM itself has no exchange step.  `local_factory` builds the per-rank SpMM object; it defaults to the CUDA
 library (paper_conf_ispass_mehrabilcslo21_b200.SpMM).  Tests inject a CPU stand-in so the host logic
 (partition, shard slicing, broadcast, reassembly) is checked with gloo on CPU.
 """
@@ -47,10 +53,23 @@ def make_shard(M: int, N: int, rowidx, colidx, value, bounds, rank: int) -> Shar
                  np.asarray(colidx[r0:r1], dtype=np.int32), np.asarray(value[r0:r1], dtype=np.float32))
 
 
+def shard_columns(rowidx, colidx, bounds, rank: int) -> np.ndarray:
+    """Sorted distinct columns referenced by shard `rank` (int64)."""
+    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
+    r0, r1 = int(rowidx[lo]), int(rowidx[hi])
+    return np.unique(np.asarray(colidx[r0:r1], dtype=np.int64))
+
+
+def compact_shard(sh: Shard, cols: np.ndarray) -> Shard:
+    """Renumber the shard's columns to their index in `cols` (monotone: row order of columns preserved)."""
+    cc = np.searchsorted(cols, sh.colidx).astype(np.int32)
+    return Shard(sh.lo, sh.hi, sh.M, int(len(cols)), sh.rowidx, cc, sh.value)
+
+
 class ShardedSpMM:
     """C = A.B with A row-sharded across the ranks of `group` (default: the world)."""
 
-    def __init__(self, M, N, rowidx, colidx, value, group=None, local_factory=None, device=None):
+    def __init__(self, M, N, rowidx, colidx, value, group=None, local_factory=None, device=None, compact_B=False):
         import torch.distributed as dist
         self.dist = dist
         self.group = group
@@ -58,7 +77,15 @@ class ShardedSpMM:
         self.world = dist.get_world_size(group)
         self.M, self.N = int(M), int(N)
         self.bounds = partition(np.asarray(rowidx, dtype=np.int64), self.world)
-        self.shard = make_shard(M, N, rowidx, colidx, value, self.bounds, self.rank)
+        self.compact_B = bool(compact_B)
+        self.cols = None
+        if self.compact_B:
+            # every rank holds the full CSR here, so every rank can derive every shard's column list
+            self.cols_all = [shard_columns(rowidx, colidx, self.bounds, p) for p in range(self.world)]
+            self.cols = self.cols_all[self.rank]
+            self.shard = compact_shard(make_shard(M, N, rowidx, colidx, value, self.bounds, self.rank), self.cols)
+        else:
+            self.shard = make_shard(M, N, rowidx, colidx, value, self.bounds, self.rank)
         self.device = device
         if local_factory is None:
             from . import SpMM
@@ -73,6 +100,29 @@ class ShardedSpMM:
         """B must be allocated (N x K) on every rank; rank `src` holds the values."""
         self.dist.broadcast(B, src=src, group=self.group)
         return B
+
+    def distribute_B(self, B, K=None, src: int = 0, dtype=None, device=None):
+        """compact_B: rank `src` passes the full B (N x K); every rank returns its compact B_p = B[cols_p]
+        (|cols_p| x K), sent point-to-point from `src`.  Other ranks may pass B=None (give K)."""
+        import torch
+        assert self.compact_B, "distribute_B needs compact_B=True (else use broadcast_B)"
+        if self.rank == src:
+            K = B.shape[1]
+            reqs = []
+            for p in range(self.world):
+                if p == src:
+                    continue
+                idx = torch.from_numpy(self.cols_all[p]).to(B.device)
+                reqs.append(self.dist.isend(B.index_select(0, idx).contiguous(),
+                                            dst=self.dist.get_global_rank(self.group, p) if self.group else p,
+                                            group=self.group))
+            mine = B.index_select(0, torch.from_numpy(self.cols).to(B.device)).contiguous()
+            for r in reqs:
+                r.wait()
+            return mine
+        mine = torch.empty((len(self.cols), int(K)), dtype=dtype or torch.float32, device=device)
+        self.dist.recv(mine, src=self.dist.get_global_rank(self.group, src) if self.group else src, group=self.group)
+        return mine
 
     def run(self, B, C_local=None):
         """Local SpMM on this rank's row shard (B resident on every rank). Returns the C shard."""

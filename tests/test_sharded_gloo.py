@@ -41,18 +41,26 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, K, results):
+def _worker(rank, world, port, K, results, compact=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from paper_conf_ispass_mehrabilcslo21_b200.sharded import ShardedSpMM
         a = syn.rmat(10, 8, 99, "natural", int_values=True)
-        sh = ShardedSpMM(a.M, a.N, a.rowidx, a.colidx, a.value, local_factory=OracleLocal)
+        sh = ShardedSpMM(a.M, a.N, a.rowidx, a.colidx, a.value, local_factory=OracleLocal, compact_B=compact)
         sh.permute("nnz_sort")
         B = torch.from_numpy(syn.dense(a.N, K, 5, int_values=True)) if rank == 0 else torch.zeros((a.N, K))
-        sh.broadcast_B(B, src=0)
-        C_local = sh.run(B)
+        if compact:
+            Bl = sh.distribute_B(B if rank == 0 else None, K=K, src=0)
+            assert Bl.shape == (sh.shard.N, K) and sh.shard.N < a.N
+            # the compact rows are exactly B[cols_p] and the shard's columns index them
+            assert np.array_equal(Bl.numpy(), syn.dense(a.N, K, 5, int_values=True)[sh.cols])
+            assert int(sh.shard.colidx.max()) < sh.shard.N
+            C_local = sh.run(Bl)
+        else:
+            sh.broadcast_B(B, src=0)
+            C_local = sh.run(B)
         C = sh.allgather_C(C_local)
         ref, _ = oracle.spmm(a, syn.dense(a.N, K, 5, int_values=True))
         nnz_local = sh.shard.nnz
@@ -62,12 +70,15 @@ def _worker(rank, world, port, K, results):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("compact", [False, True])
 @pytest.mark.parametrize("world", [2, 3])
-def test_sharded_gloo(world):
+def test_sharded_gloo(world, compact):
+    """Partition, shard slicing, B exchange (broadcast, or per-rank compact B rows: SURVEY.md §8(f) f2(i)),
+    local SpMM and the C all-gather reassemble the oracle's C exactly (integer-valued inputs)."""
     mgr = mp.Manager()
     results = mgr.dict()
     port = _free_port()
-    mp.spawn(_worker, args=(world, port, 8, results), nprocs=world, join=True)
+    mp.spawn(_worker, args=(world, port, 8, results, compact), nprocs=world, join=True)
     assert len(results) == world
     lo_hi = sorted((results[r][4], results[r][5]) for r in range(world))
     assert lo_hi[0][0] == 0 and all(lo_hi[i][1] == lo_hi[i + 1][0] for i in range(world - 1))
@@ -75,3 +86,36 @@ def test_sharded_gloo(world):
         ok, nnz_local, nnz, maxrow, _, _ = results[r]
         assert ok, f"rank {r}: reassembled C differs from the oracle"
         assert nnz_local <= -(-nnz // world) + maxrow
+
+
+def _bench_worker(rank, world, port, compact, results):
+    """bench.py's own N>1 input path (rank 0 generates, shards by nnz, optionally compacts the columns) on gloo/CPU."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import bench
+        import paper_conf_ispass_mehrabilcslo21_b200 as pkg
+        a = syn.rmat(10, 8, 98, "local", int_values=True)
+        Mr, lo, (r, c, v), meta, cols, _ = bench.shard_inputs(torch, dist, a if rank == 0 else None, world, rank,
+                                                               torch.device("cpu"), pkg, compact=compact)
+        r, c, v = r.numpy(), c.numpy(), v.numpy()
+        orig_c = cols.numpy()[c] if compact else c
+        r0 = a.rowidx[lo]
+        ok = (np.array_equal(r, a.rowidx[lo:lo + Mr + 1] - r0) and np.array_equal(orig_c, a.colidx[r0:r0 + len(c)])
+              and np.array_equal(v, a.value[r0:r0 + len(v)]))
+        if compact:
+            ok = ok and np.array_equal(cols.numpy(), np.unique(a.colidx[r0:r0 + len(c)])) and int(meta[rank, 3]) == len(cols)
+        results[rank] = (bool(ok), int(Mr), int(a.M))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("compact", [False, True])
+def test_bench_shard_inputs_gloo(compact):
+    """bench.py --gpus 2 input distribution: shards cover the rows exactly; compact shards index B[cols]."""
+    mgr = mp.Manager()
+    results = mgr.dict()
+    mp.spawn(_bench_worker, args=(2, _free_port(), compact, results), nprocs=2, join=True)
+    assert all(results[r][0] for r in range(2)), dict(results)
+    assert results[0][1] + results[1][1] == results[0][2]

@@ -1,4 +1,5 @@
-"""Measurement helpers (not the method, not the oracle): an L2-capacity LRU model of B-row reuse."""
+"""Measurement helpers (not the method, not the oracle): an L2-capacity LRU model of B-row reuse, an L2->SM
+bandwidth probe and the cuSPARSE SpMM baseline (tools/cusparse_ref.cu)."""
 import ctypes
 import os
 import subprocess
@@ -21,7 +22,32 @@ def build():
     if not os.path.exists(_PROBE) or os.path.getmtime(_PROBE) < os.path.getmtime(psrc):
         subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
                                "-shared", "-Xcompiler", "-fPIC", psrc, "-o", _PROBE])
+    csrc = os.path.join(_HERE, "cusparse_ref.cu")
+    if not os.path.exists(_CUSP) or os.path.getmtime(_CUSP) < os.path.getmtime(csrc):
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2",
+                               "-shared", "-Xcompiler", "-fPIC", csrc, "-o", _CUSP, "-lcusparse"])
     return _LIB
+
+
+_CUSP = os.path.join(_HERE, "libcusparse_ref.so")
+
+
+def cusparse_spmm_times(M, N, nnz, rowptr, colidx, value, B, K, C, alg, reps, flush, stream):
+    """cuSPARSE SpMM (CSR ALG1/2/3 or default, row-major B/C) per-rep CUDA-event times in ms, L2 flushed before
+    each rep.  Device pointers as ints (int32 rowptr/colidx).  Raises RuntimeError with the status on failure."""
+    build()
+    lib = ctypes.CDLL(_CUSP)
+    f = lib.cusparse_ref_spmm
+    f.restype = ctypes.c_int
+    f.argtypes = [ctypes.c_int64] * 3 + [ctypes.c_void_p] * 4 + [ctypes.c_int64, ctypes.c_void_p, ctypes.c_int,
+                                                                 ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t,
+                                                                 ctypes.c_void_p, ctypes.c_void_p]
+    out = np.zeros(reps, dtype=np.float32)
+    fptr, fbytes = flush if flush else (None, 0)
+    rc = f(M, N, nnz, rowptr, colidx, value, B, K, C, int(alg), int(reps), fptr, fbytes, stream, out.ctypes.data)
+    if rc != 0:
+        raise RuntimeError(f"cusparse_ref_spmm alg {alg}: status {rc}")
+    return out.tolist()
 
 
 def l2_read_bandwidth(bytes_=64 << 20, reps=50):
