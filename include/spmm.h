@@ -137,6 +137,17 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
  * Synchronises cuda_stream before returning. */
 spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *C_host, void *cuda_stream);
 
+/* Pipelined end-to-end variant for a stream of n right-hand sides (serving): for i = 0..n-1, C_host[i] =
+ * A . B_host[i] (each B_host[i]: HOST float32 [N][K] row-major, each C_host[i]: HOST float32 [M][K], original
+ * row order; all should be pinned so the copies are asynchronous).  Double-buffered handle-owned device
+ * slots and two handle-owned copy streams: the H2D of B_{i+1} and the D2H of C_{i-1} overlap the SpMM of step
+ * i (PCIe is full duplex), so a step costs about max(H2D, D2H) instead of their sum.  Every step still copies
+ * its whole B in and its whole C out.  All work is ordered after what is already queued on cuda_stream; the
+ * call synchronises cuda_stream before returning (all C_host[i] complete).  Errors as spmm_run_host (every
+ * pair is checked before any work is queued); n = 0 is a no-op. */
+spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_host, int64_t K,
+                                float *const *C_host, void *cuda_stream);
+
 /* Predictor inference (§V.B): z = (log1p(f) - mu)/sigma; h1 = relu(W1 z + b1) (64);
  * h2 = relu(W2 h1 + b2) (32); t = W3 h2 + b3 (n_policies predicted times); policy = argmin t, ties to
  * the lowest index.  weights: HOST float32, flat mu[24] sigma[24] W1[64][24] b1[64] W2[32][64] b2[32]

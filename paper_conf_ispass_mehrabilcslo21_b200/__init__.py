@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_predict",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -83,6 +83,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_features": (st, [vp, ctypes.c_int, vp, vp, vp]),
         "spmm_run": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
+        "spmm_run_host_batch": (st, [vp, i64, vp, i64, vp, vp]),
         "spmm_predict": (st, [vp, vp, i64, i32, vp, vp]),
         "spmm_partition_by_nnz": (st, [vp, i64, i32, vp]),
         "spmm_destroy": (st, [vp]),
@@ -237,6 +238,19 @@ class SpMM:
         c, _, _ = _ptr(C_host)
         _check(load_library().spmm_run_host(self._h, b, K, c, _stream_ptr(stream)))
         return C_host
+
+    def run_host_batch(self, Bs, Cs, stream=None):
+        """Pipelined end-to-end over a list of host B's (pinned) into a list of host C's (spmm_run_host_batch):
+        the H2D of the next B and the D2H of the previous C overlap the current SpMM."""
+        assert len(Bs) == len(Cs)
+        n = len(Bs)
+        if n == 0:
+            return Cs
+        K = int(Bs[0].shape[1])
+        bp = (ctypes.c_void_p * n)(*[_ptr(b)[0] for b in Bs])
+        cp = (ctypes.c_void_p * n)(*[_ptr(c)[0] for c in Cs])
+        _check(load_library().spmm_run_host_batch(self._h, n, bp, K, cp, _stream_ptr(stream)))
+        return Cs
 
     @staticmethod
     def last_run_launches() -> int:

@@ -243,7 +243,7 @@ spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colid
         std::vector<int2> cv(h->nnz);
         SPMM_CUDA(cudaMemcpy(cv.data(), h->cv_p.p, h->nnz * sizeof(int2), cudaMemcpyDeviceToHost));
         for (int64_t j = 0; j < h->nnz; ++j) {
-            colidx[j] = cv[j].x;
+            colidx[j] = cv[j].x & 0x7fffffff;   // bit 31: SPMM_HOT experiment tag
             std::memcpy(&value[j], &cv[j].y, sizeof(float));
         }
     }
@@ -317,6 +317,60 @@ spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *
     return SPMM_OK;
 }
 
+spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_host, int64_t K,
+                                float *const *C_host, void *cuda_stream) {
+    g_last_launches = 0;
+    if (!h || n < 0 || (n > 0 && (!B_host || !C_host))) return fail(SPMM_ERR_INVALID_ARG, "NULL argument or n < 0");
+    for (int64_t i = 0; i < n; ++i) SPMM_TRY(check_run_args(h, B_host[i], K, C_host[i], false));
+    SPMM_TRY(check_device(h));
+    if (n == 0) return SPMM_OK;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    const size_t bB = (size_t)h->N * K * sizeof(float), bC = (size_t)h->M * K * sizeof(float);
+    // two slots each: step i uses slot i & 1 (B rows padded to 256 B so both slots stay 32-byte aligned)
+    const size_t sB = (bB + 255) / 256 * 256, sC = (bC + 255) / 256 * 256;
+    if (h->stage_B.bytes < 2 * sB) SPMM_TRY(h->stage_B.alloc(2 * sB, s));
+    if (h->stage_C.bytes < 2 * sC) SPMM_TRY(h->stage_C.alloc(2 * sC, s));
+    if (!h->cin) {
+        SPMM_CUDA(cudaStreamCreateWithFlags(&h->cin, cudaStreamNonBlocking));
+        SPMM_CUDA(cudaStreamCreateWithFlags(&h->cout, cudaStreamNonBlocking));
+        SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_start, cudaEventDisableTiming));
+        for (int k = 0; k < 2; ++k) {
+            SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_in[k], cudaEventDisableTiming));
+            SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_comp[k], cudaEventDisableTiming));
+            SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_out[k], cudaEventDisableTiming));
+        }
+    }
+    // everything below is ordered after the work already queued on s
+    SPMM_CUDA(cudaEventRecord(h->ev_start, s));
+    SPMM_CUDA(cudaStreamWaitEvent(h->cin, h->ev_start, 0));
+    SPMM_CUDA(cudaStreamWaitEvent(h->cout, h->ev_start, 0));
+    int32_t launches = 0;
+    for (int64_t i = 0; i < n; ++i) {
+        const int k = (int)(i & 1);
+        float *Bs = reinterpret_cast<float *>(h->stage_B.as<char>() + k * sB);
+        float *Cs = reinterpret_cast<float *>(h->stage_C.as<char>() + k * sC);
+        // H2D of B_i once step i-2 (same slot) has finished reading it
+        if (i >= 2) SPMM_CUDA(cudaStreamWaitEvent(h->cin, h->ev_comp[k], 0));
+        if (bB) SPMM_CUDA(cudaMemcpyAsync(Bs, B_host[i], bB, cudaMemcpyHostToDevice, h->cin));
+        SPMM_CUDA(cudaEventRecord(h->ev_in[k], h->cin));
+        // SpMM i once B_i is in and the D2H of step i-2 has drained the C slot
+        SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_in[k], 0));
+        if (i >= 2) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_out[k], 0));
+        int32_t l = 0;
+        SPMM_TRY(launch_spmm(h, Bs, K, Cs, s, &l));
+        launches += l;
+        SPMM_CUDA(cudaEventRecord(h->ev_comp[k], s));
+        // D2H of C_i (overlaps the H2D of B_{i+1}: PCIe is full duplex)
+        SPMM_CUDA(cudaStreamWaitEvent(h->cout, h->ev_comp[k], 0));
+        if (bC) SPMM_CUDA(cudaMemcpyAsync(C_host[i], Cs, bC, cudaMemcpyDeviceToHost, h->cout));
+        SPMM_CUDA(cudaEventRecord(h->ev_out[k], h->cout));
+    }
+    for (int k = 0; k < 2 && k < n; ++k) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_out[k], 0));
+    SPMM_CUDA(cudaStreamSynchronize(s));
+    g_last_launches = launches;
+    return SPMM_OK;
+}
+
 spmm_status spmm_predict(const double features[24], const float *w, int64_t n_weights, int32_t P, int32_t *policy_out,
                          double *times_out) {
     if (!features || !w || !policy_out || P <= 0) return fail(SPMM_ERR_INVALID_ARG, "NULL argument or P <= 0");
@@ -369,6 +423,14 @@ spmm_status spmm_destroy(spmm_handle h) {
     if (h->ev_fork) cudaEventDestroy(h->ev_fork);
     if (h->ev_join) cudaEventDestroy(h->ev_join);
     if (h->side) cudaStreamDestroy(h->side);
+    if (h->ev_start) cudaEventDestroy(h->ev_start);
+    for (int k = 0; k < 2; ++k) {
+        if (h->ev_in[k]) cudaEventDestroy(h->ev_in[k]);
+        if (h->ev_comp[k]) cudaEventDestroy(h->ev_comp[k]);
+        if (h->ev_out[k]) cudaEventDestroy(h->ev_out[k]);
+    }
+    if (h->cin) cudaStreamDestroy(h->cin);
+    if (h->cout) cudaStreamDestroy(h->cout);
     delete h;
     return SPMM_OK;
 }

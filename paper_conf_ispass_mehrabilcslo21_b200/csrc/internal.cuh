@@ -110,12 +110,16 @@ struct spmm_ctx {
     spmm::DevBuf rowptr_p; // int32[M+1]
     spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
     spmm::RowClasses rc;
+    int hot_tagged = 0;     // SPMM_HOT experiment: cv_p columns carry the bit-31 hot tag (reset by permute)
     spmm::Schedule sched;
     // run scratch (partials of split rows), grown on demand
     spmm::DevBuf partials;
     spmm::DevBuf counters;  // dynamic warp-task counters, one per column tile
-    // host-run staging
+    // host-run staging (spmm_run_host: one slot; spmm_run_host_batch: two slots each, double-buffered)
     spmm::DevBuf stage_B, stage_C;
+    cudaStream_t cin = nullptr, cout = nullptr;          // spmm_run_host_batch copy streams
+    cudaEvent_t ev_start = nullptr, ev_in[2] = {nullptr, nullptr}, ev_comp[2] = {nullptr, nullptr},
+                ev_out[2] = {nullptr, nullptr};
     int num_sms = 148;
     // optional kernel timing (spmm_set_kernel_timing): events around the main SpMM kernel of spmm_run
     int timing = 0;

@@ -2,8 +2,9 @@
 window 1024, torch allocator): sampled outputs the oracle computes one by one, and the permutation /
 features checked against the oracle (-m gpu).
 
-* C2  27-point stencil 100^3 (configs[1]), K=64
-* C3  R-MAT S=22 "local", nnz 93M (configs[2]), K=128
+* C2  27-point stencil 100^3 (configs[1]), K=64 (row fusion engaged by default: R = 4)
+* C3  R-MAT S=22 "local", nnz 99.6M (configs[2]), K=128
+* C5  R-MAT S=24 "local", nnz 505M (configs[4], bench.py's default workload), K=128
 Sorted policies are compared in full; chain policies on sampled windows (each window's chain depends
 only on its own rows, so the oracle runs on the window's rows alone -- SURVEY.md §8(d) "Permutation
 parity at C5 checks ... a seeded random sample of windows plus the first and last").
@@ -32,7 +33,7 @@ def sub_rows(a, rows):
     return syn.CSR(len(rows), a.N, r, a.colidx[idx], a.value[idx])
 
 
-@pytest.fixture(scope="module", params=["c2", "c3"])
+@pytest.fixture(scope="module", params=["c2", "c3", "c5"])
 def full(request):
     cfg = bench.CONFIGS[request.param]
     a = bench.make_matrix(cfg)

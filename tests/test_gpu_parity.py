@@ -254,6 +254,24 @@ def test_device_inputs_and_host_run():
     h.close()
 
 
+def test_run_host_batch_pipelined():
+    """spmm_run_host_batch: n right-hand sides through double-buffered slots and overlapped copies give exactly
+    the C of spmm_run for each B (bit-identical), for n = 1, 2, 5 and both K geometries (fused and not)."""
+    a = syn.stencil27(14, 71)
+    for K in (64, 128):
+        h = pkg.SpMM.from_csr(a)
+        h.permute("cta_aware")
+        for n in (1, 2, 5):
+            Bs = [torch.from_numpy(syn.dense(a.N, K, 100 + i)).pin_memory() for i in range(n)]
+            Cs = [torch.full((a.M, K), float("nan")).pin_memory() for _ in range(n)]
+            h.run_host_batch(Bs, Cs)
+            for i in range(n):
+                ref = run_c(h, Bs[i].numpy())
+                assert np.array_equal(Cs[i].numpy().view(np.int32), ref.view(np.int32)), (K, n, i)
+        h.run_host_batch([], [])
+        h.close()
+
+
 def test_torch_allocator_and_streams():
     pkg.use_torch_allocator(True)
     try:
@@ -327,7 +345,7 @@ print("OK")
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
                                  {"SPMM_W": "4", "SPMM_KERNEL": "3"}, {"SPMM_VARIANT": "4"}, {"SPMM_VARIANT": "8"},
                                  {"SPMM_VARIANT": "12"}, {"SPMM_FUSE_R": "2"}, {"SPMM_FUSE": "0"},
-                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}])
+                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}, {"SPMM_VARIANT": "64", "SPMM_HOT": "100"}])
 def test_kernel_variants_exact(env):
     """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4, 128-bit lane loads, schedule
     windows, SM-affine column tiles, 4 CTAs/SM, next-task L2 prefetch, row fusion R = 2 / off) are exact on
