@@ -56,6 +56,8 @@ def _load():
         lib.oracle_partition_by_nnz.argtypes = [vp, i64, i32, vp]
         lib.oracle_minhash_keys.restype = None
         lib.oracle_minhash_keys.argtypes = [i64, vp, vp, i32, u64, vp]
+        lib.oracle_features_b200.restype = None
+        lib.oracle_features_b200.argtypes = [i64, i64, vp, vp, vp, i64, vp]
         lib.oracle_mlp_forward.restype = i32
         lib.oracle_mlp_forward.argtypes = [vp, vp, i32, vp]
         _lib = lib
@@ -119,6 +121,22 @@ def features(csr, perm=None, nw=32, nt=32, bw=32) -> np.ndarray:
     f = np.empty(24, dtype=np.float64)
     _load().oracle_features(csr.M, csr.N, r.ctypes.data, c.ctypes.data, pp, nw, nt, bw, f.ctypes.data)
     return f
+
+
+B200_FEATURES = ["fusion_union_r2", "fusion_union_r4", "window1024_distinct_cols", "b_row_byte_share",
+                 "empty_row_fraction", "split_row_nnz_fraction", "lane_slot_efficiency"]
+
+
+def features_b200(csr, K, perm=None) -> np.ndarray:
+    """The 7 B200 platform features g0..g6 (oracle.c c3b) of the matrix in its order (or perm's)."""
+    r, c = _c(csr.rowidx, np.int64), _c(csr.colidx, np.int32)
+    pp = None
+    if perm is not None:
+        perm = _c(perm, np.int32)
+        pp = perm.ctypes.data
+    g = np.empty(7, dtype=np.float64)
+    _load().oracle_features_b200(csr.M, csr.N, r.ctypes.data, c.ctypes.data, pp, int(K), g.ctypes.data)
+    return g
 
 
 def partition_by_nnz(rowidx, P: int) -> np.ndarray:

@@ -452,6 +452,88 @@ void oracle_features(int64_t M, int64_t N, const int64_t *rowidx, const int32_t 
     free_blocks(&bl);
 }
 
+/* ------------------------------------------------------------------------------------
+ * c3b. B200 platform features (the paper: platform-aware features are crucial,
+ * P:L267).  Definitions (DESIGN.md §"Readings" A24-A26), on the matrix in the given order
+ * (perm != NULL: position p holds row perm[p]); len_p = nnz of the row at position p; cols_p its columns:
+ *  g0  U2 / nnz, U2 = sum over groups of 2 consecutive positions [2g, 2g+2) of |union of their cols|
+ *      (the B-row loads per nnz of row fusion with R = 2)
+ *  g1  U4 / nnz, the same with groups of 4 consecutive positions
+ *  g2  D / nnz, D = sum over windows of 1024 consecutive positions of |union of their cols| (distinct B rows
+ *      a window of concurrently processed rows reads, per nnz)
+ *  g3  4K*Cn / (4(M+1) + 8 nnz + 4K*Cn + 4MK), Cn = number of distinct columns with >= 1 nnz (the B-row
+ *      share of the north star's algorithmic bytes at width K)
+ *  g4  (number of positions with len_p = 0) / M
+ *  g5  (sum of len_p over positions with len_p > 128) / nnz  (nnz in split rows at split_nnz = 128)
+ *  g6  lane-slot efficiency of the short rows: the positions with 0 < len_p <= 128, in position order, are cut
+ *      into windows of 32 consecutive ones; inside a window the lengths are sorted in descending order and
+ *      taken RPW at a time (RPW = 8 if K <= 32, 4 if K <= 256, else 2: rows per warp task of the kernel at
+ *      width K); g6 = (sum of the lengths) / (sum over those groups of RPW * their largest length)
+ * Every ratio is (double)int64 / (double)int64 and 0 when its denominator is 0.
+ * ---------------------------------------------------------------------------------- */
+static int64_t union_count(const int64_t *rowidx, const int32_t *colidx, const int32_t *perm, int64_t p0,
+                           int64_t p1, char *mark, int32_t *touched) {
+    /* |union of cols of positions [p0, p1)| with a 0/1 array over columns (cleared again before returning) */
+    int64_t n = 0;
+    for (int64_t p = p0; p < p1; ++p) {
+        int64_t i = perm ? perm[p] : p;
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j)
+            if (!mark[colidx[j]]) { mark[colidx[j]] = 1; touched[n++] = colidx[j]; }
+    }
+    for (int64_t t = 0; t < n; ++t) mark[touched[t]] = 0;
+    return n;
+}
+
+static int cmp_i64_desc(const void *pa, const void *pb) {
+    int64_t a = *(const int64_t *)pa, b = *(const int64_t *)pb;
+    return (a < b) - (a > b);
+}
+
+static double ratio(int64_t a, int64_t b) { return b ? (double)a / (double)b : 0.0; }
+
+void oracle_features_b200(int64_t M, int64_t N, const int64_t *rowidx, const int32_t *colidx, const int32_t *perm,
+                          int64_t K, double *g) {
+    int64_t nnz = M ? rowidx[M] : 0;
+    char *mark = (char *)calloc((size_t)(N ? N : 1), 1);
+    int32_t *touched = (int32_t *)malloc((size_t)(nnz ? nnz : 1) * sizeof(int32_t));
+    int64_t u2 = 0, u4 = 0, d = 0;
+    for (int64_t p = 0; p < M; p += 2) u2 += union_count(rowidx, colidx, perm, p, p + 2 < M ? p + 2 : M, mark, touched);
+    for (int64_t p = 0; p < M; p += 4) u4 += union_count(rowidx, colidx, perm, p, p + 4 < M ? p + 4 : M, mark, touched);
+    for (int64_t p = 0; p < M; p += 1024)
+        d += union_count(rowidx, colidx, perm, p, p + 1024 < M ? p + 1024 : M, mark, touched);
+    int64_t cn = union_count(rowidx, colidx, NULL, 0, M, mark, touched);   /* order-independent */
+    g[0] = ratio(u2, nnz);
+    g[1] = ratio(u4, nnz);
+    g[2] = ratio(d, nnz);
+    g[3] = ratio(4 * K * cn, 4 * (M + 1) + 8 * nnz + 4 * K * cn + 4 * M * K);
+    int64_t nempty = 0, nsplit = 0;
+    for (int64_t p = 0; p < M; ++p) {
+        int64_t len = row_nnz(rowidx, perm ? perm[p] : p);
+        if (len == 0) ++nempty;
+        if (len > 128) nsplit += len;
+    }
+    g[4] = ratio(nempty, M);
+    g[5] = ratio(nsplit, nnz);
+    int64_t rpw = K <= 32 ? 8 : K <= 256 ? 4 : 2;
+    int64_t *sl = (int64_t *)malloc((size_t)(M ? M : 1) * sizeof(int64_t));
+    int64_t ns = 0;
+    for (int64_t p = 0; p < M; ++p) {
+        int64_t len = row_nnz(rowidx, perm ? perm[p] : p);
+        if (len > 0 && len <= 128) sl[ns++] = len;
+    }
+    int64_t sum = 0, slots = 0;
+    for (int64_t w0 = 0; w0 < ns; w0 += 32) {
+        int64_t w1 = w0 + 32 < ns ? w0 + 32 : ns;
+        qsort(sl + w0, (size_t)(w1 - w0), sizeof(int64_t), cmp_i64_desc);
+        for (int64_t t = w0; t < w1; ++t) sum += sl[t];
+        for (int64_t t = w0; t < w1; t += rpw) slots += rpw * sl[t];    /* sl[t] = largest of the group */
+    }
+    g[6] = ratio(sum, slots);
+    free(sl);
+    free(touched);
+    free(mark);
+}
+
 /* c4. Partition by nnz (row-sharded mode, north star (4)):
  * bounds[0]=0, bounds[P]=M, bounds[p] = min{ r in [0,M] : rowidx[r] >= ceil(p*nnz/P) }. */
 void oracle_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds) {
