@@ -126,6 +126,18 @@ spmm_status spmm_get_schedule_info(spmm_handle h, int64_t out[6]);
 spmm_status spmm_features(spmm_handle h, int use_current_order, const spmm_params *params, double out[24],
                           void *cuda_stream);
 
+/* B200 platform features g0..g6 ("platform-aware features are crucial", P:L267,
+ * P:L330-332; definitions DESIGN.md readings A24-A26) of the ORIGINAL order (use_current_order = 0) or of the
+ * current permutation, for right-hand-side width K: out[0] / out[1] = column-union of 2 / 4 consecutive rows
+ * per nnz (row fusion's B-row loads per nnz), out[2] = distinct columns per 1024-row window per nnz, out[3] =
+ * B-row share 4K*Cn / (4(M+1) + 8 nnz + 4K*Cn + 4MK) of the algorithmic bytes (Cn = distinct columns),
+ * out[4] = empty-row fraction, out[5] = fraction of nnz in rows longer than 128, out[6] = lane-slot efficiency
+ * of the short rows at the kernel's rows per warp task for K.  Integer counts on the device, ratios
+ * (double)int64 / (double)int64 (0 on an empty denominator): bit-identical to the oracle.  out: 7 doubles,
+ * HOST.  Scratch up to 12 bytes per nnz (a (window, column) key sort).  Synchronises cuda_stream.
+ * Errors: INVALID_ARG (NULL, K <= 0), STATE, OOM, CUDA. */
+spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, double out[7], void *cuda_stream);
+
 /* C = A . B on the device (beta = 0: C is fully overwritten; empty rows get zeros).
  * B: device, float32 row-major [N][K]; C: device, float32 row-major [M][K] in ORIGINAL row order.
  * Asynchronous on cuda_stream; reads the handle only, but shares its long-row scratch, so calls on

@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -81,6 +81,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_get_info": (st, [vp, vp]),
         "spmm_get_schedule_info": (st, [vp, vp]),
         "spmm_features": (st, [vp, ctypes.c_int, vp, vp, vp]),
+        "spmm_features_b200": (st, [vp, ctypes.c_int, i64, vp, vp]),
         "spmm_run": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host_batch": (st, [vp, i64, vp, i64, vp, vp]),
@@ -220,6 +221,13 @@ class SpMM:
         p = make_params(nw=nw, nt=nt, bw=bw, window=0)
         _check(load_library().spmm_features(self._h, int(bool(current_order)), ctypes.byref(p), out.ctypes.data,
                                             _stream_ptr(stream)))
+        return out
+
+    def features_b200(self, K, current_order=False, stream=None) -> np.ndarray:
+        """The 7 B200 platform features g0..g6 (spmm_features_b200) for right-hand-side width K."""
+        out = np.empty(7, dtype=np.float64)
+        _check(load_library().spmm_features_b200(self._h, int(bool(current_order)), int(K), out.ctypes.data,
+                                                 _stream_ptr(stream)))
         return out
 
     def run(self, B, C=None, stream=None):

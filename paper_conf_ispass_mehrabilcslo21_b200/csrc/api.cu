@@ -286,6 +286,17 @@ spmm_status spmm_features(spmm_handle h, int use_current_order, const spmm_param
     }
 }
 
+spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, double out[7], void *cuda_stream) {
+    if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    if (K <= 0) return fail(SPMM_ERR_INVALID_ARG, "K must be positive");
+    SPMM_TRY(check_device(h));
+    try {
+        return compute_features_b200(h, use_current_order != 0, K, out, (cudaStream_t)cuda_stream);
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
+}
+
 static spmm_status check_run_args(spmm_handle h, const void *B, int64_t K, const void *C, bool device) {
     if (!h || (h->M > 0 && !C) || (h->N > 0 && h->nnz > 0 && !B)) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     if (K <= 0) return fail(SPMM_ERR_INVALID_ARG, "K must be positive");

@@ -13,6 +13,7 @@
 // "row p" is original row p (use_current_order = 0) or the row at position p of the current permutation.
 #include "internal.cuh"
 #include <algorithm>
+#include <climits>
 #include <vector>
 
 namespace spmm {
@@ -220,6 +221,205 @@ spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params 
     put3_vec(out + 15, hdd);
     put3_vec(out + 18, htt);
     put3(out + 21, hs[3]);
+    return SPMM_OK;
+}
+
+// ---- B200 platform features g0..g6 (readings A24-A26) ------------------------
+//   g0/g1  union of the columns of R = 2 / 4 consecutive positions, summed, per nnz (row fusion's B loads per nnz)
+//   g2     distinct columns per window of 1024 consecutive positions, summed, per nnz
+//   g3     4K*Cn / (4(M+1) + 8nnz + 4K*Cn + 4MK), Cn = distinct columns with >= 1 nnz
+//   g4     empty positions / M;  g5  nnz in rows longer than 128 / nnz
+//   g6     lane-slot efficiency of the short rows (0 < len <= 128): windows of 32 in position order, lengths
+//          sorted descending, RPW at a time (8 if K <= 32, 4 if K <= 256, else 2): sum len / sum RPW * group max
+// Integer counting on the device; the ratios are formed on the host as (double)int64 / (double)int64.
+namespace {
+
+enum { B_U2 = 0, B_U4, B_WIN, B_CN, B_EMPTY, B_SPLIT, B_SSUM, B_SLOTS, B_NCNT };
+
+__device__ __forceinline__ void warp_add(unsigned long long *dst, unsigned long long v) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(dst, v);
+}
+
+// thread per group of R consecutive positions: R-way merge of the (strictly increasing) column lists
+template <int R>
+__global__ void k_b200_union(OrigCSR A, int64_t M, unsigned long long *out) {
+    const int64_t ng = (M + R - 1) / R;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t g0 = (int64_t)blockIdx.x * blockDim.x; g0 < ng; g0 += stride) {
+        const int64_t g = g0 + threadIdx.x;
+        unsigned long long n = 0;
+        if (g < ng) {
+            int32_t j[R], e[R], c[R];
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const int64_t p = g * R + r;
+                j[r] = p < M ? A.begin(p) : 0;
+                e[r] = p < M ? A.end(p) : 0;
+                c[r] = j[r] < e[r] ? A.col(j[r]) : INT_MAX;
+            }
+            for (;;) {
+                int32_t m = c[0];
+#pragma unroll
+                for (int r = 1; r < R; ++r) m = min(m, c[r]);
+                if (m == INT_MAX) break;
+#pragma unroll
+                for (int r = 0; r < R; ++r)
+                    if (c[r] == m) { ++j[r]; c[r] = j[r] < e[r] ? A.col(j[r]) : INT_MAX; }
+                ++n;
+            }
+        }
+        warp_add(out, n);
+    }
+}
+
+__global__ void k_b200_rows(OrigCSR A, int64_t M, int32_t *len, int32_t *is_short, unsigned long long *out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t p0 = (int64_t)blockIdx.x * blockDim.x; p0 < M; p0 += stride) {
+        const int64_t p = p0 + threadIdx.x;
+        int32_t l = 0;
+        if (p < M) {
+            l = A.end(p) - A.begin(p);
+            len[p] = l;
+            is_short[p] = l > 0 && l <= 128;
+        }
+        warp_add(out + B_EMPTY, (p < M && l == 0) ? 1ULL : 0ULL);
+        warp_add(out + B_SPLIT, l > 128 ? (unsigned long long)l : 0ULL);
+    }
+}
+
+// keys (window << 32 | col) of every nnz in position order (warp per position)
+__global__ void k_b200_winkeys(OrigCSR A, int64_t M, const int32_t *pos_off, uint64_t *keys, uint32_t *vals) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; p < M;
+         p += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int32_t a = A.begin(p), l = A.end(p) - a, o = pos_off[p];
+        const uint64_t w = (uint64_t)(p >> 10) << 32;
+        for (int32_t t = lane; t < l; t += 32) {
+            keys[o + t] = w | (uint32_t)A.col(a + t);
+            vals[o + t] = 0u;
+        }
+    }
+}
+
+__global__ void k_b200_distinct(const uint64_t *keys, int64_t n, unsigned long long *out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t j0 = (int64_t)blockIdx.x * blockDim.x; j0 < n; j0 += stride) {
+        const int64_t j = j0 + threadIdx.x;
+        warp_add(out, (j < n && (j == 0 || keys[j] != keys[j - 1])) ? 1ULL : 0ULL);
+    }
+}
+
+__global__ void k_b200_colflags(const int32_t *colidx, int64_t nnz, uint8_t *flag) {
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x)
+        flag[colidx[j]] = 1;
+}
+
+__global__ void k_b200_count_flags(const uint8_t *flag, int64_t n, unsigned long long *out) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t j0 = (int64_t)blockIdx.x * blockDim.x; j0 < n; j0 += stride) {
+        const int64_t j = j0 + threadIdx.x;
+        warp_add(out, (j < n && flag[j]) ? 1ULL : 0ULL);
+    }
+}
+
+__global__ void k_b200_scatter_short(const int32_t *is_short, const int32_t *sidx, const int32_t *len, int64_t M,
+                                     int32_t *slen) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x)
+        if (is_short[p]) slen[sidx[p]] = len[p];
+}
+
+// thread per window of 32 short rows: insertion sort descending, then RPW-groups
+__global__ void k_b200_slots(const int32_t *slen, int64_t ns, int32_t rpw, unsigned long long *out) {
+    const int64_t nwin = (ns + 31) / 32;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t w0 = (int64_t)blockIdx.x * blockDim.x; w0 < nwin; w0 += stride) {
+        const int64_t w = w0 + threadIdx.x;
+        unsigned long long sum = 0, slots = 0;
+        if (w < nwin) {
+            int32_t v[32];
+            const int n = (int)(ns - w * 32 < 32 ? ns - w * 32 : 32);
+            for (int t = 0; t < n; ++t) {
+                int32_t x = slen[w * 32 + t];
+                sum += (unsigned long long)x;
+                int u = t;
+                while (u > 0 && v[u - 1] < x) { v[u] = v[u - 1]; --u; }
+                v[u] = x;
+            }
+            for (int t = 0; t < n; t += rpw) slots += (unsigned long long)rpw * (unsigned long long)v[t];
+        }
+        warp_add(out + B_SSUM, sum);
+        warp_add(out + B_SLOTS, slots);
+    }
+}
+
+inline unsigned gb(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+inline double ratio(unsigned long long a, unsigned long long b) { return b ? (double)a / (double)b : 0.0; }
+
+}  // namespace
+
+spmm_status compute_features_b200(spmm_ctx *h, bool current_order, int64_t K, double out[7], cudaStream_t s) {
+    const int64_t M = h->M, N = h->N, nnz = h->nnz;
+    for (int i = 0; i < 7; ++i) out[i] = 0.0;
+    if (M == 0) return SPMM_OK;
+    OrigCSR A{h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), current_order ? h->perm.as<int32_t>() : nullptr};
+    DevBuf cnt, len, is_short, sidx, slen, off, keys, vals, flag;
+    SPMM_TRY(cnt.alloc(B_NCNT * sizeof(unsigned long long), s));
+    SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, cnt.bytes, s));
+    unsigned long long *C = cnt.as<unsigned long long>();
+    k_b200_union<2><<<gb(ceil_div(M, 2)), 256, 0, s>>>(A, M, C + B_U2);
+    k_b200_union<4><<<gb(ceil_div(M, 4)), 256, 0, s>>>(A, M, C + B_U4);
+    SPMM_TRY(len.alloc(M * sizeof(int32_t), s));
+    SPMM_TRY(is_short.alloc(M * sizeof(int32_t), s));
+    k_b200_rows<<<gb(M), 256, 0, s>>>(A, M, len.as<int32_t>(), is_short.as<int32_t>(), C);
+    SPMM_CUDA(cudaGetLastError());
+    if (nnz > 0) {
+        // window distinct columns: sort (window, col) keys, count distinct
+        SPMM_TRY(off.alloc((M + 1) * sizeof(int32_t), s));
+        SPMM_TRY(exclusive_scan_i32(len.as<int32_t>(), off.as<int32_t>(), M, nullptr, s));
+        SPMM_TRY(keys.alloc(nnz * sizeof(uint64_t), s));
+        SPMM_TRY(vals.alloc(nnz * sizeof(uint32_t), s));
+        k_b200_winkeys<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(M * 32, 256), 148 * 64)), 256, 0,
+                         s>>>(A, M, off.as<int32_t>(), keys.as<uint64_t>(), vals.as<uint32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        int hi = 32;
+        while (hi < 64 && (((M - 1) >> 10) >> (hi - 32)) > 0) ++hi;
+        SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), vals.as<uint32_t>(), nnz, 0, ((hi + 7) / 8) * 8, s));
+        k_b200_distinct<<<gb(nnz), 256, 0, s>>>(keys.as<uint64_t>(), nnz, C + B_WIN);
+        keys.release();
+        vals.release();
+        // distinct columns overall
+        SPMM_TRY(flag.alloc(std::max<int64_t>(N, 1), s));
+        SPMM_CUDA(cudaMemsetAsync(flag.p, 0, flag.bytes, s));
+        k_b200_colflags<<<gb(nnz), 256, 0, s>>>(h->colidx.as<int32_t>(), nnz, flag.as<uint8_t>());
+        k_b200_count_flags<<<gb(N), 256, 0, s>>>(flag.as<uint8_t>(), N, C + B_CN);
+        SPMM_CUDA(cudaGetLastError());
+    }
+    // lane-slot efficiency of the short rows
+    SPMM_TRY(sidx.alloc((M + 1) * sizeof(int32_t), s));
+    int32_t ns = 0;
+    SPMM_TRY(exclusive_scan_i32(is_short.as<int32_t>(), sidx.as<int32_t>(), M, &ns, s));
+    if (ns > 0) {
+        SPMM_TRY(slen.alloc(ns * sizeof(int32_t), s));
+        k_b200_scatter_short<<<gb(M), 256, 0, s>>>(is_short.as<int32_t>(), sidx.as<int32_t>(), len.as<int32_t>(), M,
+                                                  slen.as<int32_t>());
+        const int32_t rpw = K <= 32 ? 8 : K <= 256 ? 4 : 2;
+        k_b200_slots<<<gb(ceil_div(ns, 32)), 256, 0, s>>>(slen.as<int32_t>(), ns, rpw, C);
+        SPMM_CUDA(cudaGetLastError());
+    }
+    unsigned long long hc[B_NCNT];
+    SPMM_CUDA(cudaMemcpyAsync(hc, cnt.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
+    SPMM_CUDA(cudaStreamSynchronize(s));
+    const unsigned long long nz = (unsigned long long)nnz;
+    out[0] = ratio(hc[B_U2], nz);
+    out[1] = ratio(hc[B_U4], nz);
+    out[2] = ratio(hc[B_WIN], nz);
+    const unsigned long long kb = 4ULL * (unsigned long long)K * hc[B_CN];
+    out[3] = ratio(kb, 4ULL * (unsigned long long)(M + 1) + 8ULL * nz + kb + 4ULL * (unsigned long long)M * K);
+    out[4] = ratio(hc[B_EMPTY], (unsigned long long)M);
+    out[5] = ratio(hc[B_SPLIT], nz);
+    out[6] = ratio(hc[B_SSUM], hc[B_SLOTS]);
     return SPMM_OK;
 }
 

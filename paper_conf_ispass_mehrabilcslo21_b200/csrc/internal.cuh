@@ -144,6 +144,7 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
 spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s);
 spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24],
                              cudaStream_t s);
+spmm_status compute_features_b200(spmm_ctx *h, bool current_order, int64_t K, double out[7], cudaStream_t s);
 spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches);
 
 // signatures of the rows (sorted unique col/bw), used by chains and features

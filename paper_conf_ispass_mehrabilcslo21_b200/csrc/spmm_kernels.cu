@@ -1064,7 +1064,7 @@ struct Config {
 // measured to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
 Config choose(int32_t K4, int sched, int var, bool w8ok) {
     if (w8ok && sched == 0 && (var & 2) == 0 && K4 % 2 == 0) {
-        const int vu = var & 15;   // bit 4 only selects the fused kernel's prefetch
+        const int vu = var & ~16;  // bit 4 only selects the fused kernel's prefetch
         const int32_t K8 = K4 / 2;
         for (int G : {8, 4})
             for (int V : {1, 2, 4})
@@ -1072,7 +1072,7 @@ Config choose(int32_t K4, int sched, int var, bool w8ok) {
                     SpmmKernel k = pick_w8v(vu, V, G);
                     if (k) {
                         Config c{k, V, G, 1, 8};
-                        if ((vu & 3) == 0) {
+                        if ((vu & 3) == 0 && (vu & 64) == 0) {   // no fused kernel reads hot-tagged columns
                             c.R = fuse_rows_for(V, G);
                             c.kern_fused = c.R > 1 ? pick_w8_fused(var, V, G, c.R) : nullptr;
                         }

@@ -77,6 +77,7 @@ def test_fullsize_sorts_and_features(full):
         h.permute(pol, window=W)
         assert np.array_equal(h.perm(), oracle.permute(a, pol)), (name, pol)
     np.testing.assert_array_equal(h.features(), oracle.features(a))
+    np.testing.assert_array_equal(h.features_b200(K), oracle.features_b200(a, K))
 
 
 @pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_1"])

@@ -158,6 +158,29 @@ def test_features_bit_exact(mats, gen, params):
     h.close()
 
 
+@pytest.mark.parametrize("gen", list(GENS))
+@pytest.mark.parametrize("K", [32, 128, 512])
+def test_features_b200_bit_exact(mats, gen, K):
+    """spmm_features_b200 (f4) equals the oracle's g0..g6 bit for bit, original and permuted orders."""
+    a = mats[gen]
+    h = pkg.SpMM.from_csr(a)
+    np.testing.assert_array_equal(h.features_b200(K), oracle.features_b200(a, K))
+    for pol in ("nnz_sort", "cta_aware"):
+        h.permute(pol)
+        np.testing.assert_array_equal(h.features_b200(K, current_order=True), oracle.features_b200(a, K, h.perm()))
+    h.close()
+
+
+def test_features_b200_edges():
+    for a in (syn.from_lists(0, 10, []), syn.from_lists(5, 10, [[]] * 5),
+              syn.from_lists(3, 3000, [list(range(0, 3000, 7)), [], [5]]),     # one split row (> 128 nnz)
+              syn.rmat(11, 6, 33, "natural")):
+        h = pkg.SpMM.from_csr(a)
+        for K in (4, 64, 1024):
+            np.testing.assert_array_equal(h.features_b200(K), oracle.features_b200(a, K))
+        h.close()
+
+
 def test_e1_worked_example(e1):
     a = syn.from_lists(e1["M"], e1["N"], e1["rows"])
     h = pkg.SpMM.from_csr(a)
