@@ -167,6 +167,13 @@ spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_
 spmm_status spmm_predict(const double features[24], const float *mlp_weights, int64_t n_weights,
                          int32_t n_policies, int32_t *policy_out, double *times_out);
 
+/* The same inference for F input features (e.g. F = 31: the 24 Table II features followed by the 7 B200
+ * platform features of spmm_features_b200, f4): weights mu[F] sigma[F] W1[64][F] b1[64] W2[32][64] b2[32]
+ * W3[P][32] b3[P]; n_weights must equal 2F + 64F + 64 + 2048 + 32 + 33P.  spmm_predict is spmm_predict_n
+ * with F = 24. */
+spmm_status spmm_predict_n(const double *features, int32_t n_features, const float *mlp_weights, int64_t n_weights,
+                           int32_t n_policies, int32_t *policy_out, double *times_out);
+
 /* Row-sharded mode (north star (4)): bounds[0]=0, bounds[P]=M,
  * bounds[p] = min{ r : rowidx[r] >= ceil(p*nnz/P) }.  rowidx: HOST int64[M+1]; bounds: HOST int64[P+1]. */
 spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds);

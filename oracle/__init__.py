@@ -58,6 +58,8 @@ def _load():
         lib.oracle_minhash_keys.argtypes = [i64, vp, vp, i32, u64, vp]
         lib.oracle_features_b200.restype = None
         lib.oracle_features_b200.argtypes = [i64, i64, vp, vp, vp, i64, vp]
+        lib.oracle_mlp_forward_n.restype = i32
+        lib.oracle_mlp_forward_n.argtypes = [vp, i32, vp, i32, vp]
         lib.oracle_mlp_forward.restype = i32
         lib.oracle_mlp_forward.argtypes = [vp, vp, i32, vp]
         _lib = lib
@@ -158,4 +160,12 @@ def mlp_forward(feat, weights, P):
     w = _c(weights, np.float32)
     out = np.empty(P, dtype=np.float64)
     best = _load().oracle_mlp_forward(f.ctypes.data, w.ctypes.data, P, out.ctypes.data)
+    return int(best), out
+
+
+def mlp_forward_n(feat, weights, P):
+    f = _c(feat, np.float64)
+    w = _c(weights, np.float32)
+    out = np.empty(P, dtype=np.float64)
+    best = _load().oracle_mlp_forward_n(f.ctypes.data, len(f), w.ctypes.data, P, out.ctypes.data)
     return int(best), out

@@ -576,3 +576,34 @@ int32_t oracle_mlp_forward(const double *feat, const float *w, int32_t P, double
     }
     return best;
 }
+
+/* The predictor's forward for F input features (f4: the 24 Table II features followed by the 7 B200 platform
+ * features of c3b), same definition as oracle_mlp_forward (reading A19): z = (log1p(f) - mu) / sigma,
+ * two ReLU layers 64 and 32, P outputs, argmin with ties to the lowest index.  Layout mu[F] sigma[F] W1[64][F]
+ * b1[64] W2[32][64] b2[32] W3[P][32] b3[P].  Pinned in tests/test_abi.py against a numpy float64 forward. */
+int32_t oracle_mlp_forward_n(const double *feat, int32_t F, const float *w, int32_t P, double *out) {
+    const float *mu = w, *sg = w + F, *W1 = w + 2 * (int64_t)F, *b1 = W1 + 64 * (int64_t)F, *W2 = b1 + 64,
+                *b2 = W2 + 32 * 64, *W3 = b2 + 32, *b3 = W3 + (int64_t)P * 32;
+    double *x = (double *)malloc((size_t)F * sizeof(double));
+    double h1[64], h2[32];
+    for (int i = 0; i < F; ++i) x[i] = (log1p(feat[i]) - (double)mu[i]) / (double)sg[i];
+    for (int o = 0; o < 64; ++o) {
+        double s = b1[o];
+        for (int i = 0; i < F; ++i) s += (double)W1[(int64_t)o * F + i] * x[i];
+        h1[o] = s > 0 ? s : 0;
+    }
+    for (int o = 0; o < 32; ++o) {
+        double s = b2[o];
+        for (int i = 0; i < 64; ++i) s += (double)W2[o * 64 + i] * h1[i];
+        h2[o] = s > 0 ? s : 0;
+    }
+    int32_t best = 0;
+    for (int o = 0; o < P; ++o) {
+        double s = b3[o];
+        for (int i = 0; i < 32; ++i) s += (double)W3[o * 32 + i] * h2[i];
+        out[o] = s;
+        if (s < out[best]) best = o;
+    }
+    free(x);
+    return best;
+}

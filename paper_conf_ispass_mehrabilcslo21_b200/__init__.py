@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -86,6 +86,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host_batch": (st, [vp, i64, vp, i64, vp, vp]),
         "spmm_predict": (st, [vp, vp, i64, i32, vp, vp]),
+        "spmm_predict_n": (st, [vp, i32, vp, i64, i32, vp, vp]),
         "spmm_partition_by_nnz": (st, [vp, i64, i32, vp]),
         "spmm_destroy": (st, [vp]),
         "spmm_status_string": (ctypes.c_char_p, [st]),
@@ -306,22 +307,39 @@ def spmm_predict(features, weights, n_policies):
     return int(pol.value), times
 
 
+def spmm_predict_n(features, weights, n_policies):
+    """spmm_predict for any number of input features (e.g. 24 Table II + 7 B200 features)."""
+    f = np.ascontiguousarray(features, dtype=np.float64)
+    w = np.ascontiguousarray(weights, dtype=np.float32)
+    pol = ctypes.c_int32()
+    times = np.empty(n_policies, dtype=np.float64)
+    _check(load_library().spmm_predict_n(f.ctypes.data, len(f), w.ctypes.data, len(w), n_policies, ctypes.byref(pol),
+                                         times.ctypes.data))
+    return int(pol.value), times
+
+
 PREDICTOR_POLICIES = HOT_PATH_POLICIES          # classes of the bundled predictor (reading A20)
 PAPER4_POLICIES = ["identity", "dcsr", "lpt", "warp_aware"]   # the paper's four classes (P:L273)
 
 
-def predictor_weights(K: int, paper_classes: bool = False) -> np.ndarray:
-    """Bundled MLP weights (spmm_predict layout) trained on the C4 corpus for the nearest trained K."""
-    d = os.path.join(_HERE, "predictor4" if paper_classes else "predictor")
+def predictor_weights(K: int, paper_classes: bool = False, b200: bool = False) -> np.ndarray:
+    """Bundled MLP weights (spmm_predict layout) trained on the C4 corpus for the nearest trained K
+    (b200: the 31-feature model with the B200 platform features, f4)."""
+    d = os.path.join(_HERE, "predictor4" if paper_classes else ("predictor_b200" if b200 else "predictor"))
     ks = sorted(int(f[5:-4]) for f in os.listdir(d) if f.startswith("mlp_K") and f.endswith(".npy"))
     k = min(ks, key=lambda x: (abs(np.log2(x) - np.log2(K)), x))
     return np.load(os.path.join(d, f"mlp_K{k}.npy"))
 
 
-def select_policy(h: "SpMM", K: int, paper_classes: bool = False) -> str:
+def select_policy(h: "SpMM", K: int, paper_classes: bool = False, b200: bool = False) -> str:
     """a10 predicted selection: features of the original order on the GPU (spmm_features), MLP inference
-    in the library (spmm_predict), argmin of the predicted times."""
+    in the library (spmm_predict), argmin of the predicted times.  b200: the 24 features plus
+    the 7 B200 platform features (spmm_features_b200, f4) through spmm_predict_n."""
     classes = PAPER4_POLICIES if paper_classes else PREDICTOR_POLICIES
+    if b200 and not paper_classes:
+        f = np.concatenate([h.features(current_order=False), h.features_b200(K, current_order=False)])
+        pol, _ = spmm_predict_n(f, predictor_weights(K, b200=True), len(classes))
+        return classes[pol]
     pol, _ = spmm_predict(h.features(current_order=False), predictor_weights(K, paper_classes), len(classes))
     return classes[pol]
 

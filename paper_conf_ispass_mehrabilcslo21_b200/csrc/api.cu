@@ -382,18 +382,19 @@ spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_
     return SPMM_OK;
 }
 
-spmm_status spmm_predict(const double features[24], const float *w, int64_t n_weights, int32_t P, int32_t *policy_out,
-                         double *times_out) {
-    if (!features || !w || !policy_out || P <= 0) return fail(SPMM_ERR_INVALID_ARG, "NULL argument or P <= 0");
-    if (n_weights != 48 + 64 * 24 + 64 + 32 * 64 + 32 + 33 * (int64_t)P)
-        return fail(SPMM_ERR_INVALID_ARG, "n_weights does not match the 24-64-32-P layout");
-    const float *mu = w, *sg = w + 24, *W1 = w + 48, *b1 = W1 + 64 * 24, *W2 = b1 + 64, *b2 = W2 + 32 * 64,
+spmm_status spmm_predict_n(const double *features, int32_t F, const float *w, int64_t n_weights, int32_t P,
+                           int32_t *policy_out, double *times_out) {
+    if (!features || !w || !policy_out || P <= 0 || F <= 0) return fail(SPMM_ERR_INVALID_ARG, "NULL argument, P <= 0 or F <= 0");
+    if (n_weights != 2 * (int64_t)F + 64 * (int64_t)F + 64 + 32 * 64 + 32 + 33 * (int64_t)P)
+        return fail(SPMM_ERR_INVALID_ARG, "n_weights does not match the F-64-32-P layout");
+    const float *mu = w, *sg = w + F, *W1 = w + 2 * F, *b1 = W1 + 64 * (int64_t)F, *W2 = b1 + 64, *b2 = W2 + 32 * 64,
                 *W3 = b2 + 32, *b3 = W3 + (int64_t)P * 32;
-    double z[24], h1[64], h2[32];
-    for (int i = 0; i < 24; ++i) z[i] = (std::log1p(features[i]) - (double)mu[i]) / (double)sg[i];
+    std::vector<double> z(F);
+    double h1[64], h2[32];
+    for (int i = 0; i < F; ++i) z[i] = (std::log1p(features[i]) - (double)mu[i]) / (double)sg[i];
     for (int o = 0; o < 64; ++o) {
         double s = b1[o];
-        for (int i = 0; i < 24; ++i) s += (double)W1[o * 24 + i] * z[i];
+        for (int i = 0; i < F; ++i) s += (double)W1[(int64_t)o * F + i] * z[i];
         h1[o] = s > 0 ? s : 0;
     }
     for (int o = 0; o < 32; ++o) {
@@ -411,6 +412,11 @@ spmm_status spmm_predict(const double features[24], const float *w, int64_t n_we
     }
     *policy_out = best;
     return SPMM_OK;
+}
+
+spmm_status spmm_predict(const double features[24], const float *w, int64_t n_weights, int32_t P, int32_t *policy_out,
+                         double *times_out) {
+    return spmm_predict_n(features, 24, w, n_weights, P, policy_out, times_out);
 }
 
 spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds) {

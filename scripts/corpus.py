@@ -1,5 +1,6 @@
 """C4 (BASELINE.json configs[3]): a synthetic corpus spanning the paper's feature ranges, every hot-path
-policy timed on the B200 (the exhaustive-timing label) plus the 24 features.
+policy timed on the B200 (the exhaustive-timing label) plus the 24 features and the
+7 B200 platform features per K (f4, spmm_features_b200).
 
   python scripts/corpus.py --n-per-family 50 --out gpurun_out/corpus.jsonl
 
@@ -76,6 +77,7 @@ def main():
         fam, params, a = draw(i, args.max_log2m)
         h = pkg.SpMM.from_csr(a)
         feats = h.features().tolist()
+        feats_b200 = {str(K): h.features_b200(K).tolist() for K in Ks}   # f4 platform features (g0..g6)
         Bs = {K: torch.from_numpy(syn.dense(a.N, K, 77 + i)).cuda() for K in Ks}
         C = torch.empty((a.M, max(Ks)), device="cuda")
         times = {K: {} for K in Ks}
@@ -99,6 +101,7 @@ def main():
                     ts.append(e0.elapsed_time(e1))
                 times[K][pol] = statistics.median(ts)
         rec = dict(i=i, family=fam, params=params, name=a.name, M=a.M, N=a.N, nnz=a.nnz, features=feats,
+                   features_b200=feats_b200,
                    times_ms={str(K): v for K, v in times.items()}, build_ms=build, seconds=time.perf_counter() - t0)
         out.write(json.dumps(rec) + "\n")
         out.flush()

@@ -9,7 +9,7 @@ argmin of the predicted times.  Reported like the paper: classification
 matrix (Fig. 13), predicted-selection speedup vs the exhaustive-timing oracle (the paper's
 1.37x vs 1.41x), loss distribution (Fig. 14: within 4% / 10%, mean), regression error CDF (Fig. 12),
 the per-policy Table-I analogue, the softmax-classifier variant and the matrix-only-feature
-ablation.  Weights are written in spmm_predict's flat layout and the library's C inference
+ablation, and (f4) the same regression with the 7 B200 platform features appended.  Weights are written in spmm_predict's flat layout and the library's C inference
 (spmm_predict) is checked against the torch forward.
 """
 import argparse
@@ -38,14 +38,17 @@ class MLP(torch.nn.Module):
         return self.l3(torch.relu(self.l2(torch.relu(self.l1(z)))))
 
 
-def load(path, K, policies):
+def load(path, K, policies, b200=False):
+    """X: the 24 Table II features (+ the 7 B200 platform features at this K when b200, f4)."""
     X, T, meta = [], [], []
     for line in open(path):
         r = json.loads(line)
         t = r["times_ms"].get(str(K))
         if not t or any(p not in t for p in policies):
             continue
-        X.append(r["features"])
+        if b200 and str(K) not in r.get("features_b200", {}):
+            continue
+        X.append(r["features"] + (r["features_b200"][str(K)] if b200 else []))
         T.append([t[p] for p in policies])
         meta.append((r["i"], r["family"], r["name"]))
     return np.array(X, dtype=np.float64), np.array(T, dtype=np.float64), meta
@@ -160,6 +163,21 @@ def main():
         # matrix-only feature ablation
         netm, mum, sgm = train(X[tr], Y[tr], w, MATRIX_ONLY, epochs=args.epochs, seed=K)
         res["matrix_only_features"] = evaluate(T[te], predict(netm, mum, sgm, X[te], MATRIX_ONLY).argmin(1), policies)
+        # f4: the same regression with the 7 B200 platform features appended (F = 31), same split and weights
+        Xb, Tb, _ = load(args.corpus, K, policies, b200=True)
+        if len(Xb) == len(X):
+            feats31 = list(range(31))
+            netb, mub, sgb = train(Xb[tr], Y[tr], w, feats31, epochs=args.epochs, seed=K)
+            chb = predict(netb, mub, sgb, Xb[te], feats31).argmin(1)
+            res["with_b200_features"] = evaluate(T[te], chb, policies)
+            wb = flat_weights(netb, mub, sgb)
+            agree = sum(int(pkg.spmm_predict_n(f, wb, P)[0] == c) for f, c in zip(Xb[te], chb))
+            res["with_b200_features"]["c_inference_agreement"] = agree / max(len(te), 1)
+            os.makedirs(args.weights_dir + "_b200", exist_ok=True)
+            np.save(os.path.join(args.weights_dir + "_b200", f"mlp_K{K}.npy"), wb)
+            rb = res["with_b200_features"]
+            print(f"   +B200 features: acc={rb['accuracy']:.2f} predicted {rb['speedup_predicted']:.3f}x "
+                  f"gain {rb['oracle_gain_fraction']:.2f} loss {rb['mean_loss']:.3f} C-agree {rb['c_inference_agreement']:.2f}")
         report["per_K"][str(K)] = res
         r = res["regression"]
         print(f"K={K}: n={len(X)} acc={r['accuracy']:.2f} oracle {r['speedup_oracle']:.3f}x predicted "

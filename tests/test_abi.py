@@ -67,6 +67,41 @@ def test_predict_matches_oracle(P):
         np.testing.assert_allclose(times, ref, rtol=1e-12, atol=1e-12)
 
 
+def np_forward(f, w, F, P):
+    """Independent numpy float64 forward of the F-64-32-P layout (pins oracle_mlp_forward_n)."""
+    w = w.astype(np.float64)
+    o = 0
+    mu, sg = w[o:o + F], w[o + F:o + 2 * F]; o += 2 * F
+    W1 = w[o:o + 64 * F].reshape(64, F); o += 64 * F
+    b1 = w[o:o + 64]; o += 64
+    W2 = w[o:o + 2048].reshape(32, 64); o += 2048
+    b2 = w[o:o + 32]; o += 32
+    W3 = w[o:o + 32 * P].reshape(P, 32); o += 32 * P
+    b3 = w[o:o + P]
+    z = (np.log1p(f) - mu) / sg
+    h1 = np.maximum(W1 @ z + b1, 0)
+    h2 = np.maximum(W2 @ h1 + b2, 0)
+    return W3 @ h2 + b3
+
+
+@pytest.mark.parametrize("F,P", [(24, 6), (31, 6), (31, 4), (5, 3)])
+def test_predict_n_matches_oracle_and_numpy(F, P):
+    rng = np.random.default_rng(F * 10 + P)
+    n = 2 * F + 64 * F + 64 + 32 * 64 + 32 + 33 * P
+    w = (rng.standard_normal(n) * 0.3).astype(np.float32)
+    w[F:2 * F] = np.abs(w[F:2 * F]) + 0.5
+    for t in range(5):
+        f = np.abs(rng.standard_normal(F)) * 10 ** rng.integers(0, 6)
+        ref = np_forward(f, w, F, P)
+        best, orc = oracle.mlp_forward_n(f, w, P)
+        np.testing.assert_allclose(orc, ref, rtol=1e-10, atol=1e-10)
+        pol, times = pkg.spmm_predict_n(f, w, P)
+        assert pol == best == int(np.argmin(orc))
+        np.testing.assert_allclose(times, orc, rtol=1e-12, atol=1e-12)
+        if F == 24:
+            assert pkg.spmm_predict(f, w, P)[0] == pol
+
+
 def test_predict_rejects_bad_layout():
     with pytest.raises(pkg.SpmmError):
         pkg.spmm_predict(np.zeros(24), np.zeros(10, np.float32), 4)
