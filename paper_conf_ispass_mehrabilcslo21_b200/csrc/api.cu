@@ -243,7 +243,7 @@ spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colid
         std::vector<int2> cv(h->nnz);
         SPMM_CUDA(cudaMemcpy(cv.data(), h->cv_p.p, h->nnz * sizeof(int2), cudaMemcpyDeviceToHost));
         for (int64_t j = 0; j < h->nnz; ++j) {
-            colidx[j] = cv[j].x & 0x7fffffff;   // bit 31: SPMM_HOT experiment tag
+            colidx[j] = cv[j].x;
             std::memcpy(&value[j], &cv[j].y, sizeof(float));
         }
     }

@@ -110,7 +110,6 @@ struct spmm_ctx {
     spmm::DevBuf rowptr_p; // int32[M+1]
     spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
     spmm::RowClasses rc;
-    int hot_tagged = 0;     // SPMM_HOT experiment: cv_p columns carry the bit-31 hot tag (reset by permute)
     spmm::Schedule sched;
     // run scratch (partials of split rows), grown on demand
     spmm::DevBuf partials;

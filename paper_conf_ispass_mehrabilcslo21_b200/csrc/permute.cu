@@ -529,7 +529,6 @@ spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s) {
     }
     // a7 row-class counts (the K-dependent run schedule is built by the first spmm_run)
     h->sched.rpw = 0;
-    h->hot_tagged = 0;
     h->rc.n_long = h->rc.n_chunks = 0;
     if (M == 0 || h->max_row_nnz <= split) return SPMM_OK;
     DevBuf flag, nch, tmp;

@@ -81,11 +81,6 @@ __device__ __forceinline__ uint64_t policy_evict_last() {
     asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-__device__ __forceinline__ uint64_t policy_evict_normal() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
 __device__ __forceinline__ uint64_t policy_evict_first() {
     uint64_t p;
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -96,7 +91,7 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
 template <int LD>
 __device__ __forceinline__ float4 ld_b(const float4 *ptr, uint64_t pol) {
     float4 r;
-    if (LD == 1 || LD == 3) {
+    if (LD == 1) {
         asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;" : SPMM_V4_OUT : "l"(ptr), "l"(pol));
     } else {
         r = __ldg(ptr);
@@ -106,7 +101,7 @@ __device__ __forceinline__ float4 ld_b(const float4 *ptr, uint64_t pol) {
 template <int LD>
 __device__ __forceinline__ float8 ld_b(const float8 *ptr, uint64_t pol) {
     float8 r;
-    if (LD == 1 || LD == 3) {
+    if (LD == 1) {
         asm("ld.global.nc.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;" : SPMM_V8_OUT : "l"(ptr), "l"(pol));
     } else {
         asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];" : SPMM_V8_OUT : "l"(ptr));
@@ -174,15 +169,6 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                 col[w] = __shfl_sync(0xffffffffu, cur[qq / G].x, src);
                 a[w] = __int_as_float(__shfl_sync(0xffffffffu, cur[qq / G].y, src));
             }
-            uint64_t pw[U];                          // LD 3: hot columns (bit 31 tag) evict_last, others normal
-#pragma unroll
-            for (int w = 0; w < U; ++w) {
-                pw[w] = pol_b;
-                if (LD == 3) {
-                    pw[w] = col[w] < 0 ? pol_b : pol_a;
-                    col[w] &= 0x7fffffff;
-                }
-            }
             const int32_t rem = len - (b0 + q0);    // nnz left for this group
             if (rem >= U) {                          // full step: U*V independent B loads in flight
                 VT x[U][V];
@@ -191,7 +177,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                     const VT *b = BV + (size_t)col[w] * KV + col0;
 #pragma unroll
                     for (int v = 0; v < V; ++v) {
-                        if (colok[v]) x[w][v] = ld_b<LD>(b + v * G, pw[w]);
+                        if (colok[v]) x[w][v] = ld_b<LD>(b + v * G, pol_b);
                         else vzero(x[w][v]);
                     }
                 }
@@ -206,7 +192,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                         const VT *b = BV + (size_t)col[w] * KV + col0;
 #pragma unroll
                         for (int v = 0; v < V; ++v)
-                            if (colok[v]) vfma(a[w], ld_b<LD>(b + v * G, pw[w]), acc[v]);
+                            if (colok[v]) vfma(a[w], ld_b<LD>(b + v * G, pol_b), acc[v]);
                     }
                 }
             }
@@ -394,7 +380,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
     using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
     constexpr int CTV = V * G;
-    constexpr int LD = (VAR & 1) ? 1 : (VAR & 64) ? 3 : 0;   // VAR bit 6: hot-column L2 hints (SPMM_HOT)
+    constexpr int LD = (VAR & 1) ? 1 : 0;
     constexpr int U = (V * W >= 12 && !(VAR & 2)) ? 2 : 4;   // nnz per inner step (B loads in flight per lane: U*V)
     const int32_t KV = K4 * 4 / W;
     const int lane = threadIdx.x & 31;
@@ -403,8 +389,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
     bool colok[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < KV);
-    const uint64_t pol_b = (LD == 1 || LD == 3) ? policy_evict_last() : 0,
-                   pol_a = LD == 1 ? policy_evict_first() : LD == 3 ? policy_evict_normal() : 0;
+    const uint64_t pol_b = LD == 1 ? policy_evict_last() : 0, pol_a = LD == 1 ? policy_evict_first() : 0;
 
     __shared__ TaskQueue q;
     unsigned int tk = 0;
@@ -749,7 +734,7 @@ __global__ void k_union(const int32_t *gpos, int64_t n_groups, int32_t R, const 
             const int32_t p = r < R ? gpos[g * R + r] : -1;
             j[r] = p >= 0 ? rowptr[p] : 0;
             e[r] = p >= 0 ? rowptr[p + 1] : 0;
-            c[r] = j[r] < e[r] ? (cv[j[r]].x & 0x7fffffff) : INT_MAX;
+            c[r] = j[r] < e[r] ? cv[j[r]].x : INT_MAX;
             tot += e[r] - j[r];
             if (FILL && r < R) gdst[g * R + r] = p >= 0 ? perm[p] : NOSTORE;
         }
@@ -764,7 +749,7 @@ __global__ void k_union(const int32_t *gpos, int64_t n_groups, int32_t R, const 
                     mask |= 1 << r;
                     v[r] = cv[j[r]].y;
                     ++j[r];
-                    c[r] = j[r] < e[r] ? (cv[j[r]].x & 0x7fffffff) : INT_MAX;
+                    c[r] = j[r] < e[r] ? cv[j[r]].x : INT_MAX;
                 }
             }
             if (FILL) {
@@ -806,23 +791,6 @@ __global__ void k_fill_fused(const int32_t *gseg, int64_t n_groups, const int32_
         }
         const int64_t task = (int64_t)taskbase[k] + idx / rpw;
         units[task * rpw + idx % rpw] = make_int4(rbase[g], len, (int32_t)g, 1);
-    }
-}
-
-// ---- hot-column L2 hints (experiment, SPMM_HOT=H): the ~H most referenced columns' B rows are loaded with
-// L2::evict_last, the rest with evict_normal; the tag is bit 31 of the permuted CSR's column (N < 2^31) ----
-__global__ void k_col_count(const int2 *cv, int64_t nnz, int32_t *cnt) {
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&cnt[cv[j].x & 0x7fffffff], 1);
-}
-__global__ void k_count_hist(const int32_t *cnt, int64_t N, int32_t *hist) {
-    for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < N; c += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&hist[min(cnt[c], 65535)], 1);
-}
-__global__ void k_tag_hot(int2 *cv, int64_t nnz, const int32_t *cnt, int32_t t) {
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t c = cv[j].x & 0x7fffffff;
-        cv[j].x = cnt[c] >= t ? (c | (int32_t)0x80000000) : c;
     }
 }
 
@@ -1041,7 +1009,6 @@ int fuse_rows_for(int V, int G) {
 
 SpmmKernel pick_w8v(int var, int V, int G) {
     switch (var) {
-        case 64: return pick_w8<64>(V, G);
         case 1: return pick_w8<1>(V, G);
         case 4: return pick_w8<4>(V, G);
         case 8: return pick_w8<8>(V, G);
@@ -1072,7 +1039,7 @@ Config choose(int32_t K4, int sched, int var, bool w8ok) {
                     SpmmKernel k = pick_w8v(vu, V, G);
                     if (k) {
                         Config c{k, V, G, 1, 8};
-                        if ((vu & 3) == 0 && (vu & 64) == 0) {   // no fused kernel reads hot-tagged columns
+                        if ((vu & 3) == 0) {
                             c.R = fuse_rows_for(V, G);
                             c.kern_fused = c.R > 1 ? pick_w8_fused(var, V, G, c.R) : nullptr;
                         }
@@ -1197,30 +1164,6 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         const int aw = w8ok ? 8 : 4;
         if (K % (32 * av) == 0 && pick_aff(av, env_int("SPMM_AFF_LD", 2), aw))
             return launch_aff(h, B, K, C, s, av, aw, launches);
-    }
-    // hot-column tagging for the LD 3 kernel (SPMM_VARIANT=64, SPMM_HOT = number of hot B rows)
-    static const int hot_rows = env_int("SPMM_HOT", 0);
-    if (var == 64 && hot_rows > 0 && h->hot_tagged != hot_rows && h->nnz > 0) {
-        DevBuf cnt, hist;
-        SPMM_TRY(cnt.alloc(h->N * sizeof(int32_t), s));
-        SPMM_TRY(hist.alloc(65536 * sizeof(int32_t), s));
-        SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, h->N * sizeof(int32_t), s));
-        SPMM_CUDA(cudaMemsetAsync(hist.p, 0, 65536 * sizeof(int32_t), s));
-        k_col_count<<<g1(h->nnz), 256, 0, s>>>(h->cv_p.as<int2>(), h->nnz, cnt.as<int32_t>());
-        k_count_hist<<<g1(h->N), 256, 0, s>>>(cnt.as<int32_t>(), h->N, hist.as<int32_t>());
-        std::vector<int32_t> hh(65536);
-        SPMM_CUDA(cudaMemcpyAsync(hh.data(), hist.p, 65536 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-        SPMM_CUDA(cudaStreamSynchronize(s));
-        int64_t acc = 0;
-        int32_t t = 65536;
-        for (int32_t c = 65535; c >= 2; --c) {
-            if (acc + hh[c] > hot_rows) break;
-            acc += hh[c];
-            t = c;
-        }
-        k_tag_hot<<<g1(h->nnz), 256, 0, s>>>(h->cv_p.as<int2>(), h->nnz, cnt.as<int32_t>(), t);
-        SPMM_CUDA(cudaGetLastError());
-        h->hot_tagged = hot_rows;
     }
     const int32_t rpw = 32 / cfg.G;
     // row fusion: fuse_rows 1 = off; SPMM_FUSE=0 disables it process-wide (A/B knob)

@@ -368,7 +368,7 @@ print("OK")
                                  {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
                                  {"SPMM_W": "4", "SPMM_KERNEL": "3"}, {"SPMM_VARIANT": "4"}, {"SPMM_VARIANT": "8"},
                                  {"SPMM_VARIANT": "12"}, {"SPMM_FUSE_R": "2"}, {"SPMM_FUSE": "0"},
-                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}, {"SPMM_VARIANT": "64", "SPMM_HOT": "100"}])
+                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}])
 def test_kernel_variants_exact(env):
     """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4, 128-bit lane loads, schedule
     windows, SM-affine column tiles, 4 CTAs/SM, next-task L2 prefetch, row fusion R = 2 / off) are exact on
