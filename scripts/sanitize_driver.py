@@ -24,4 +24,21 @@ h2 = pkg.SpMM.from_csr(syn.blockcluster(3000, 5000, 32, 4, 12, 3))
 h2.permute("hybrid_2_2", window=512, preorder=1, seed=3)
 h2.run(torch.zeros((5000, 64), device="cuda"))
 torch.cuda.synchronize()
+# row fusion (forced, K = 64 -> R = 4, K = 128 -> R = 2) with a split row, the pipelined host API, B200 features
+st = syn.stencil27(10, 4)
+rows = [st.colidx[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
+rows[7] = list(range(0, st.N, 3))
+st = syn.from_lists(st.M, st.N, rows)
+h3 = pkg.SpMM.from_csr(st)
+for pol in ("identity", "cta_aware"):
+    h3.permute(pol, fuse_rows=2)
+    for K in (64, 128):
+        h3.run(torch.from_numpy(syn.dense(st.N, K, 2)).cuda())
+        Bs = [torch.from_numpy(syn.dense(st.N, K, 3 + i)).pin_memory() for i in range(3)]
+        Cs = [torch.empty((st.M, K)).pin_memory() for _ in range(3)]
+        h3.run_host_batch(Bs, Cs)
+    for K in (32, 128):
+        h3.features_b200(K, current_order=True)
+h.features_b200(64)
+torch.cuda.synchronize()
 print("sanitize driver done")
