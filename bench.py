@@ -288,9 +288,16 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # BENCH_GPU_INDEX / BENCH_DIST_BACKEND: test hooks only (dry-run of the N>1 path with several ranks on one
+    # GPU over gloo); the driver's runs use one GPU per rank and NCCL
+    local = int(os.environ.get("BENCH_GPU_INDEX", local))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     cfg = CONFIGS[args.config]

@@ -410,6 +410,7 @@ def test_select_policy_runs():
         assert pol in pkg.PREDICTOR_POLICIES
         pol4 = pkg.select_policy(h, K, paper_classes=True)
         assert pol4 in pkg.PAPER4_POLICIES
+        assert pkg.select_policy(h, K, b200=True) in pkg.PREDICTOR_POLICIES    # f4: 24 + 7 features
         h.permute(pol)
         assert np.array_equal(h.perm(), oracle.permute(a, pol, window=1024))
     h.close()
