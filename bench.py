@@ -39,16 +39,33 @@ CONFIGS = {
     "c3rl": dict(desc="configs[2] stress variant: power-law R-MAT S=22 random-label, M=N=4M, nnz~100M, K=128",
                  gen=("rmat", 22, 28, 3001, "random-label"), K=128),
     "c5": dict(desc="configs[4]: power-law R-MAT S=24 'local', M=N=16M, nnz~500M, K=128", gen=("rmat", 24, 38, 5000, "local"), K=128),
+    "c3sh": dict(desc="configs[2] with its rows randomly relabelled (seeded shuffle; columns unchanged): the original "
+                      "order has no locality, the column-similarity orders must recover the communities",
+                 gen=("rmat", 22, 28, 3000, "local"), shuffle=3002, K=128),
 }
-HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1"]
+HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1", "cta_aware+mh", "hybrid_2_1+mh"]
+# "+mh": the chain policy with its windows over the MinHash pre-order (spmm_params.preorder = 1)
 METRIC = "SpMM GFLOP/s and % HBM roofline per permutation policy at 1/2/4/8 B200"
 
 
 def make_matrix(cfg):
     g = cfg["gen"]
-    if g[0] == "rmat":
-        return syn.rmat(g[1], g[2], g[3], g[4])
-    return syn.stencil27(g[1], g[2])
+    a = syn.rmat(g[1], g[2], g[3], g[4]) if g[0] == "rmat" else syn.stencil27(g[1], g[2])
+    if cfg.get("shuffle") is not None:   # row relabel: new row r = old row q[r]
+        q = np.random.default_rng(cfg["shuffle"]).permutation(a.M)
+        lens = np.diff(a.rowidx)[q]
+        r = np.zeros(a.M + 1, dtype=np.int64)
+        np.cumsum(lens, out=r[1:])
+        idx = np.repeat(a.rowidx[q] - r[:-1], lens) + np.arange(a.nnz, dtype=np.int64)
+        a = syn.CSR(a.M, a.N, r, a.colidx[idx], a.value[idx])
+    return a
+
+
+def permute_spec(h, pol, window):
+    """A policy name, optionally with '+mh' (chain windows over the MinHash pre-order, preorder = 1)."""
+    if pol.endswith("+mh"):
+        return h.permute(pol[:-3], window=window, preorder=1, seed=1)
+    return h.permute(pol, window=window)
 
 
 def algorithmic_bytes(a, K):
@@ -365,7 +382,7 @@ def main():
     for pol in args.policies.split(","):
         torch.cuda.synchronize()
         tb = time.perf_counter()
-        h.permute(pol, window=args.window)
+        permute_spec(h, pol, args.window)
         build_ms = 1e3 * (time.perf_counter() - tb)
         for _ in range(args.warmup):
             h.run(Bd, Cd)
@@ -387,7 +404,7 @@ def main():
     if world > 1:
         dist.all_reduce(tvec, op=dist.ReduceOp.MAX)
     best = names[int(torch.argmin(tvec))]
-    h.permute(best, window=args.window)
+    permute_spec(h, best, args.window)
 
     # ---- the timed region: `steps` steps of the selected policy ----
     for _ in range(args.warmup):

@@ -60,6 +60,8 @@ def _load():
         lib.oracle_features_b200.argtypes = [i64, i64, vp, vp, vp, i64, vp]
         lib.oracle_mlp_forward_n.restype = i32
         lib.oracle_mlp_forward_n.argtypes = [vp, i32, vp, i32, vp]
+        lib.oracle_median_block_keys.restype = None
+        lib.oracle_median_block_keys.argtypes = [i64, vp, vp, i32, vp]
         lib.oracle_mlp_forward.restype = i32
         lib.oracle_mlp_forward.argtypes = [vp, vp, i32, vp]
         _lib = lib
@@ -152,6 +154,13 @@ def minhash_keys(csr, bw=32, seed=0) -> np.ndarray:
     r, c = _c(csr.rowidx, np.int64), _c(csr.colidx, np.int32)
     h = np.empty(csr.M, dtype=np.uint64)
     _load().oracle_minhash_keys(csr.M, r.ctypes.data, c.ctypes.data, bw, seed, h.ctypes.data)
+    return h
+
+
+def median_block_keys(csr, bw=32) -> np.ndarray:
+    r, c = _c(csr.rowidx, np.int64), _c(csr.colidx, np.int32)
+    h = np.empty(csr.M, dtype=np.uint64)
+    _load().oracle_median_block_keys(csr.M, r.ctypes.data, c.ctypes.data, bw, h.ctypes.data)
     return h
 
 

@@ -161,6 +161,22 @@ void oracle_minhash_keys(int64_t M, const int64_t *rowidx, const int32_t *colidx
         h[i] = m;
     }
 }
+/* Median-block pre-order key (preorder = 2; not in the paper, DESIGN.md §2 "pre-orders"): the lower median
+ * blocks_i[(|blocks_i| - 1) / 2] of the row's sorted distinct column blocks (a one-dimensional position of the
+ * row's column footprint, so rows over the same column range become neighbours); empty rows 2^64 - 1. */
+void oracle_median_block_keys(int64_t M, const int64_t *rowidx, const int32_t *colidx, int32_t bw, uint64_t *h) {
+    for (int64_t i = 0; i < M; ++i) {
+        int64_t nb = 0;   /* distinct blocks are where col/bw changes (columns strictly increasing, A15) */
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j)
+            if (j == rowidx[i] || colidx[j] / bw != colidx[j - 1] / bw) ++nb;
+        h[i] = ~(uint64_t)0;
+        if (nb == 0) continue;
+        int64_t want = (nb - 1) / 2, k = -1;
+        for (int64_t j = rowidx[i]; j < rowidx[i + 1]; ++j)
+            if (j == rowidx[i] || colidx[j] / bw != colidx[j - 1] / bw)
+                if (++k == want) { h[i] = (uint64_t)(colidx[j] / bw); break; }
+    }
+}
 typedef struct { uint64_t key; int64_t id; } ukeyed;
 static int cmp_u_asc(const void *pa, const void *pb) {
     const ukeyed *a = (const ukeyed *)pa, *b = (const ukeyed *)pb;
@@ -239,7 +255,8 @@ static void chain_window(int mode, const int32_t *om, int64_t n, const blocklist
 
 /* ------------------------------------------------------------------------------------
  * oracle_permute: perm[p] = original row placed at position p (gather form), a bijection.
- * window W (multiple of nw, 0 = whole matrix, reading A11); preorder 0 = original, 1 = MinHash.
+ * window W (multiple of nw, 0 = whole matrix, reading A11); preorder 0 = original, 1 = MinHash,
+ * 2 = median block.
  * Returns 0 on success, 1 on invalid arguments.
  * ---------------------------------------------------------------------------------- */
 int oracle_permute(int32_t policy, int64_t M, const int64_t *rowidx, const int32_t *colidx, int32_t nw,
@@ -307,7 +324,8 @@ int oracle_permute(int32_t policy, int64_t M, const int64_t *rowidx, const int32
         int32_t *pre = (int32_t *)malloc((size_t)(M ? M : 1) * sizeof(int32_t));
         if (preorder) {
             uint64_t *h = (uint64_t *)malloc((size_t)(M ? M : 1) * sizeof(uint64_t));
-            oracle_minhash_keys(M, rowidx, colidx, bw, seed, h);
+            if (preorder == 2) oracle_median_block_keys(M, rowidx, colidx, bw, h);
+            else oracle_minhash_keys(M, rowidx, colidx, bw, seed, h);
             ukeyed *t = (ukeyed *)malloc((size_t)(M ? M : 1) * sizeof(ukeyed));
             for (int64_t i = 0; i < M; ++i) { t[i].key = h[i]; t[i].id = i; }
             qsort(t, (size_t)M, sizeof(ukeyed), cmp_u_asc);

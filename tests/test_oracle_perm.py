@@ -153,6 +153,31 @@ def test_minhash_preorder_chain():
     ck.check_chain_local_optimality(perm, a, "cta", nw=8, W=64, pre=pre)
 
 
+def test_median_block_keys_by_hand(e1):
+    # E1 with bw = 2: blocks r0 {0,1,2} -> 1, r1 {3} -> 3, r2 {} -> 2^64-1, r3 {0,1} -> 0, r4 {2,3} -> 2,
+    # r5 {0} -> 0, r6 {2,3} -> 2, r7 {0,1,3} -> 1 (lower median of the sorted distinct blocks)
+    a = e1_csr(e1)
+    assert oracle.median_block_keys(a, bw=2).tolist() == [1, 3, 2 ** 64 - 1, 0, 2, 0, 2, 1]
+
+
+def test_median_block_keys_bruteforce():
+    a = syn.rmat(10, 9, 46, "local")
+    ref = []
+    for i in range(a.M):
+        b = sorted(set((a.colidx[a.rowidx[i]:a.rowidx[i + 1]] // 32).tolist()))
+        ref.append(b[(len(b) - 1) // 2] if b else 2 ** 64 - 1)
+    assert oracle.median_block_keys(a).tolist() == ref
+
+
+@pytest.mark.parametrize("policy,mode", [("cta_aware", "cta"), ("hybrid_2_1", "h21")])
+def test_median_preorder_chain(policy, mode):
+    """preorder = 2: windows over the stable (median block, id) order; every greedy step locally optimal."""
+    a = syn.rmat(10, 9, 47, "local")
+    pre = np.lexsort((np.arange(a.M), oracle.median_block_keys(a)))
+    perm = oracle.permute(a, policy, nw=8, window=64, preorder=2)
+    ck.check_chain_local_optimality(perm, a, mode, nw=8, W=64, pre=pre)
+
+
 def test_minhash_splitmix_vector():
     """splitmix64 test vector: the first output of the splitmix64 generator seeded with 0 is
     0xE220A8397B1DCDAF (= finaliser(0) with the golden-gamma pre-add).  A one-row matrix whose
