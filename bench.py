@@ -43,8 +43,9 @@ CONFIGS = {
                       "order has no locality, the column-similarity orders must recover the communities",
                  gen=("rmat", 22, 28, 3000, "local"), shuffle=3002, K=128),
 }
-HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1", "cta_aware+mh", "hybrid_2_1+mh"]
-# "+mh": the chain policy with its windows over the MinHash pre-order (spmm_params.preorder = 1)
+HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1", "cta_aware+mh", "cta_aware+md"]
+# "+mh" / "+md": the chain policy with its windows over the MinHash / median-block pre-order (spmm_params.preorder
+# = 1 / 2)
 METRIC = "SpMM GFLOP/s and % HBM roofline per permutation policy at 1/2/4/8 B200"
 
 
@@ -62,9 +63,12 @@ def make_matrix(cfg):
 
 
 def permute_spec(h, pol, window):
-    """A policy name, optionally with '+mh' (chain windows over the MinHash pre-order, preorder = 1)."""
+    """A policy name, optionally with '+mh' / '+md': chain windows over the MinHash / median-block pre-order
+    (spmm_params.preorder = 1 / 2)."""
     if pol.endswith("+mh"):
         return h.permute(pol[:-3], window=window, preorder=1, seed=1)
+    if pol.endswith("+md"):
+        return h.permute(pol[:-3], window=window, preorder=2)
     return h.permute(pol, window=window)
 
 

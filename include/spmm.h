@@ -71,7 +71,8 @@ typedef struct {
                                (bounds every fp32 accumulation chain, DESIGN.md §"Accuracy")         */
     int64_t window;         /* greedy-chain window W (multiple of nw); 0 = whole matrix (paper-exact,
                                supported up to 32768 rows); default 1024                               */
-    int32_t preorder;       /* chain policies: 0 = windows over the original order, 1 = MinHash key  */
+    int32_t preorder;       /* chain policies: windows over 0 = the original order, 1 = the MinHash key
+                               order, 2 = the median-column-block order (DESIGN.md §2 "pre-orders")    */
     int32_t fuse_rows;      /* row fusion in spmm_run (a7/a8): 0 = auto -- take the short rows R consecutive
                                positions at a time and walk the union of their columns once (each shared B
                                row loaded once) when the unions hold <= 3/4 of those rows' nnz; 1 = off;

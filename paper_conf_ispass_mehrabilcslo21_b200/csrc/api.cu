@@ -97,9 +97,9 @@ spmm_status check_device(spmm_ctx *h) {
 
 spmm_status check_params(const spmm_params &p) {
     if (p.nw <= 0 || p.nw > 1024 || p.nt <= 0 || p.bw <= 0 || p.split_nnz < 1 || p.window < 0 ||
-        (p.window % p.nw) != 0 || (p.preorder != 0 && p.preorder != 1) || p.fuse_rows < 0 || p.fuse_rows > 2)
+        (p.window % p.nw) != 0 || (p.preorder < 0 || p.preorder > 2) || p.fuse_rows < 0 || p.fuse_rows > 2)
         return fail(SPMM_ERR_INVALID_ARG, "invalid spmm_params (nw/nt/bw > 0, nw <= 1024, split_nnz >= 1, "
-                                          "window >= 0 and a multiple of nw, preorder in {0,1}, fuse_rows in {0,1,2})");
+                                          "window >= 0 and a multiple of nw, preorder in {0,1,2}, fuse_rows in {0,1,2})");
     return SPMM_OK;
 }
 

@@ -62,6 +62,15 @@ __global__ void k_minhash(const int32_t *sig_ptr, const int32_t *sig, int64_t M,
     }
 }
 
+// median-block pre-order key (preorder = 2): the lower median of the row's sorted distinct blocks; empty rows last
+__global__ void k_median_block(const int32_t *sig_ptr, const int32_t *sig, int64_t M, uint64_t *keys, uint32_t *vals) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t a = sig_ptr[i], n = sig_ptr[i + 1] - a;
+        keys[i] = n > 0 ? (uint64_t)(uint32_t)sig[a + (n - 1) / 2] : ~0ULL;
+        vals[i] = (uint32_t)i;
+    }
+}
+
 // ---- signatures: warp per row; distinct blocks are the positions where col/bw changes ---------
 __global__ void k_sig_count(const int32_t *rowidx, const int32_t *colidx, int64_t M, int32_t bw, int32_t *cnt) {
     const int lane = threadIdx.x & 31;
@@ -496,8 +505,12 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
             DevBuf keys, vals;
             SPMM_TRY(keys.alloc(M * sizeof(uint64_t), s));
             SPMM_TRY(vals.alloc(M * sizeof(uint32_t), s));
-            k_minhash<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M, p.seed,
-                                                        keys.as<uint64_t>(), vals.as<uint32_t>());
+            if (p.preorder == 2)
+                k_median_block<<<grid_for(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
+                                                                keys.as<uint64_t>(), vals.as<uint32_t>());
+            else
+                k_minhash<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M, p.seed,
+                                                            keys.as<uint64_t>(), vals.as<uint32_t>());
             SPMM_CUDA(cudaGetLastError());
             SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), vals.as<uint32_t>(), M, 0, 64, s));
             k_u32_to_i32<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, base.as<int32_t>());

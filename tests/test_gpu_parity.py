@@ -73,13 +73,15 @@ def test_perm_params(mats, params, policy):
     h.close()
 
 
+@pytest.mark.parametrize("preorder", [1, 2])
 @pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_2_2", "warp_aware", "hybrid_2_3"])
-def test_minhash_preorder(mats, policy):
-    a = mats["block"]
-    h = pkg.SpMM.from_csr(a)
-    h.permute(policy, window=256, preorder=1, seed=12345)
-    assert np.array_equal(h.perm(), oracle.permute(a, policy, window=256, preorder=1, seed=12345))
-    h.close()
+def test_minhash_preorder(mats, policy, preorder):
+    for gen in ("block", "rmat13_local"):
+        a = mats[gen]
+        h = pkg.SpMM.from_csr(a)
+        h.permute(policy, window=256, preorder=preorder, seed=12345)
+        assert np.array_equal(h.perm(), oracle.permute(a, policy, window=256, preorder=preorder, seed=12345)), gen
+        h.close()
 
 
 @pytest.mark.parametrize("gen", list(GENS))
