@@ -15,6 +15,7 @@
 // and bit-identical to the oracle (DESIGN.md §"Readings").
 #include "internal.cuh"
 #include <algorithm>
+#include <cstdlib>
 #include <vector>
 
 namespace spmm {
@@ -388,6 +389,386 @@ spmm_status launch_chain(int mode, const int32_t *base, const int32_t *seg, int6
     }
 }
 
+// ---- paper-exact chains over windows above 32768 rows, up to W = M (f3) -----------
+// The same definitions as k_chain (CTA_AWARE: next = argmin over the window's unplaced rows of
+// (ham(r, prev), r); HYBRID_2_1: (ham, |wl_r - wl_prev|, r)), evaluated through an
+// inverted index block -> rows instead of scoring every candidate each step:
+//   ham(r, prev) = |b_prev| + |b_r| - 2 |b_r ∩ b_prev|, and a row sharing no block with prev scores
+//   |b_prev| + |b_r|.  So the argmin lies in T ∪ {u*}: T = the unplaced rows of prev's posting lists
+//   (scored exactly, |b_r ∩ b_prev| counted by one atomic per list entry), u* = the best untouched-form
+//   candidate: the unplaced row of least (|b|, r) (CTA_AWARE) or, among the unplaced rows of the least
+//   |b| = b0, the least (|wl - wl_prev|, r) (HYBRID_2_1).  Any row outside T scores >= u* under the key
+//   (DESIGN.md §6 "exact chains"), so the result is the definition's, bit-identical to k_chain / oracle.
+// One CTA of 1024 threads per window; per step: count pass, barrier, score pass, block argmin.  The
+// counters are double-buffered by step parity and the previous step's lists are zeroed during the
+// count pass, so they need no pass of their own.
+constexpr int XCH_THREADS = 1024;
+constexpr int XCH_CACHE = XCH_THREADS;   // posting-list prefix of up to 1024 blocks kept in smem per step
+
+__global__ void k_win_of(const int32_t *base, int64_t M, int64_t W, int32_t *win) {
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < M; q += (int64_t)gridDim.x * blockDim.x)
+        win[base[q]] = (int32_t)(q / W);
+}
+__global__ void k_blk_count(const int32_t *blk, int64_t S, int32_t *bcnt) {
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < S; t += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&bcnt[blk[t]], 1);
+}
+__global__ void k_blk_fill(const int32_t *sig_ptr, const int32_t *blk, int64_t M, const int32_t *bptr, int32_t *bcur,
+                           int32_t *brow) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M;
+         r += ((int64_t)gridDim.x * blockDim.x) >> 5)
+        for (int32_t t = sig_ptr[r] + lane; t < sig_ptr[r + 1]; t += 32) {
+            const int32_t b = blk[t];
+            brow[bptr[b] + atomicAdd(&bcur[b], 1)] = (int32_t)r;
+        }
+}
+// multi-window: posting entries keyed by (block, window of the row), so each block's list holds every
+// window's rows contiguously and a window's CTA visits only its own (two binary searches per list)
+__global__ void k_blk_win_keys(const int32_t *sig_ptr, const int32_t *blk, int64_t M, const int32_t *win,
+                               uint64_t *keys, uint32_t *vals) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M;
+         r += ((int64_t)gridDim.x * blockDim.x) >> 5)
+        for (int32_t t = sig_ptr[r] + lane; t < sig_ptr[r + 1]; t += 32) {
+            keys[t] = ((uint64_t)(uint32_t)blk[t] << 32) | (uint32_t)win[r];
+            vals[t] = (uint32_t)r;
+        }
+}
+__global__ void k_xkeys(const int32_t *sig_ptr, const int32_t *nnz, int64_t M, int32_t nt, int with_wl, uint64_t *keys,
+                        uint32_t *vals) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < M; r += (int64_t)gridDim.x * blockDim.x) {
+        const uint64_t nb = (uint64_t)(sig_ptr[r + 1] - sig_ptr[r]);
+        const uint64_t wl = (uint64_t)((nnz[r] + nt - 1) / nt);
+        keys[r] = with_wl ? (nb << 26) | wl : nb;
+        vals[r] = (uint32_t)r;
+    }
+}
+__global__ void k_xkeys_win(const uint32_t *vals, const int32_t *win, int64_t M, uint64_t *keys) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x)
+        keys[i] = (uint64_t)win[vals[i]];
+}
+
+__device__ __forceinline__ bool is_placed(const uint32_t *placed, int32_t r) {
+    return (__ldcg(placed + (r >> 5)) >> (r & 31)) & 1u;
+}
+
+// block-wide argmin over XCH_THREADS threads; every thread returns the winner
+__device__ __forceinline__ Key xblock_argmin(Key k, Key *red) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        Key y = shfl_key(k, o);
+        if (key_less(y, k)) k = y;
+    }
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = k;
+    __syncthreads();
+    Key b = red[threadIdx.x & 31];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        Key y = shfl_key(b, o);
+        if (key_less(y, b)) b = y;
+    }
+    return b;
+}
+
+// prefix of the posting-list lengths of blocks sig_blk[c0 .. c0+nb) into pre[0..nb], list starts into bst[]
+// mwin >= 0: lists sorted by window; only window mwin's sub-range [first win >= mwin, first win > mwin)
+__device__ __forceinline__ int32_t lower_win(const int32_t *brow, const int32_t *win, int32_t lo, int32_t hi, int32_t w) {
+    while (lo < hi) {
+        const int32_t mid = (lo + hi) >> 1;
+        if (win[brow[mid]] < w) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+__device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *bptr, int32_t c0, int32_t nb,
+                                        int32_t *pre, int32_t *bst, int32_t *wsum, const int32_t *brow = nullptr,
+                                        const int32_t *win = nullptr, int32_t mwin = -1) {
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    int32_t len = 0;
+    if (tid < nb) {
+        const int32_t b = sig_blk[c0 + tid];
+        int32_t a = bptr[b], e = bptr[b + 1];
+        if (mwin >= 0) {
+            a = lower_win(brow, win, a, e, mwin);
+            e = lower_win(brow, win, a, e, mwin + 1);
+        }
+        len = e - a;
+        bst[tid] = a;
+    }
+    int32_t x = len;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) wsum[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+        int32_t w = wsum[lane];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int32_t y = __shfl_up_sync(0xffffffffu, w, o);
+            if (lane >= o) w += y;
+        }
+        wsum[lane] = w;
+    }
+    __syncthreads();
+    pre[tid + 1] = x + (wid ? wsum[wid - 1] : 0);
+    if (tid == 0) pre[0] = 0;
+    __syncthreads();
+}
+
+// visit every entry of the posting lists described by (pre, bst, nb): f(row)
+template <class F>
+__device__ __forceinline__ void xvisit(const int32_t *pre, const int32_t *bst, int32_t nb, const int32_t *brow, F f) {
+    const int32_t T = pre[nb];
+    for (int32_t e = threadIdx.x; e < T; e += XCH_THREADS) {
+        int lo = 0, hi = nb - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (pre[mid] <= e) lo = mid;
+            else hi = mid - 1;
+        }
+        f(__ldg(brow + bst[lo] + (e - pre[lo])));
+    }
+}
+
+// all entries of row r0's lists, chunked by XCH_THREADS blocks (re-derives the prefix; barriers inside)
+template <class F>
+__device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, const int32_t *sig_blk,
+                                           const int32_t *bptr, const int32_t *brow, int32_t *pre, int32_t *bst,
+                                           int32_t *wsum, const int32_t *win, int32_t mwin, F f) {
+    const int32_t bs = sig_ptr[r0], be = sig_ptr[r0 + 1];
+    for (int32_t c0 = bs; c0 < be; c0 += XCH_THREADS) {
+        const int32_t nb = min(XCH_THREADS, be - c0);
+        xprefix(sig_blk, bptr, c0, nb, pre, bst, wsum, brow, win, mwin);
+        xvisit(pre, bst, nb, brow, f);
+        __syncthreads();
+    }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base, int64_t W, int64_t M, int multiwin,
+                                                            const int32_t *sig_ptr, const int32_t *sig_blk,
+                                                            const int32_t *bptr, const int32_t *brow,
+                                                            const int32_t *win, const uint32_t *ord,
+                                                            const int32_t *nnz, int32_t nt, uint32_t *placed,
+                                                            int32_t *cnt0, int32_t *cnt1, int32_t *perm) {
+    __shared__ int32_t pre[2][XCH_CACHE + 1];
+    __shared__ int32_t bst[2][XCH_CACHE];
+    __shared__ int32_t wsum[32];
+    __shared__ Key red[2][XCH_THREADS / 32];
+    __shared__ int32_t s_ptr;
+    const int32_t w = (int32_t)blockIdx.x;
+    const int64_t s0 = (int64_t)w * W, s1 = min(s0 + W, M);
+    const int32_t n = (int32_t)(s1 - s0);
+    const uint32_t *o = ord + s0;            // the window's rows by (|b|, [wl,] r)
+    int32_t *out = perm + s0;
+    auto nb_of = [&](int32_t r) -> uint32_t { return (uint32_t)(sig_ptr[r + 1] - sig_ptr[r]); };
+    auto wl_of = [&](int32_t r) -> uint32_t { return (uint32_t)((nnz[r] + nt - 1) / nt); };
+    const int32_t mw = multiwin ? w : -1;    // lists sorted by window: visit only this window's rows
+    auto mine = [&](int32_t r) -> bool { return true; };
+    if (n <= 0) return;
+    // first row: least (wl, r) of the window (as k_chain)
+    Key best{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
+    for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
+        const int32_t r = base[s0 + a];
+        Key c{wl_of(r), 0u, (uint32_t)r, 0u};
+        if (key_less(c, best)) best = c;
+    }
+    Key win0 = xblock_argmin(best, red[0]);
+    int32_t prev = (int32_t)win0.r, pprev = -1;
+    if (threadIdx.x == 0) {
+        out[0] = prev;
+        atomicOr(placed + (prev >> 5), 1u << (prev & 31));
+        s_ptr = 0;
+    }
+    bool cached_pp = false;
+    for (int32_t q = 1; q < n; ++q) {
+        const int buf = q & 1;
+        int32_t *cc = buf ? cnt1 : cnt0, *co = buf ? cnt0 : cnt1;
+        const int32_t bs = sig_ptr[prev], be = sig_ptr[prev + 1];
+        const uint32_t cp = (uint32_t)(be - bs);
+        const bool cached = be - bs <= XCH_CACHE;
+        // prefix of prev's lists (kept for the score pass and for the next step's reset); the previous
+        // step's prefix lives in the other buffer
+        if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw);
+        // reset the previous step's counters (other buffer), then count |b_r ∩ b_prev|
+        // (only this window's rows: the other windows' CTAs count theirs in the same arrays)
+        if (pprev >= 0) {
+            auto reset = [&](int32_t r) { if (mine(r)) co[r] = 0; };
+            if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pprev + 1] - sig_ptr[pprev], brow, reset);
+            else xvisit_all(pprev, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, reset);
+        }
+        auto count = [&](int32_t r) {
+            if (r != prev && mine(r) && !is_placed(placed, r)) atomicAdd(cc + r, 1);
+        };
+        if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
+        else xvisit_all(prev, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
+        __syncthreads();
+        const uint32_t wlp = MODE == C_H21 ? wl_of(prev) : 0u;
+        auto keyof = [&](int32_t r) -> Key {
+            const uint32_t c = (uint32_t)__ldcg(cc + r);
+            Key k{cp + nb_of(r) - 2u * c, 0u, (uint32_t)r, 0u};
+            if (MODE == C_H21) {
+                const uint32_t x = wl_of(r);
+                k.k2 = x > wlp ? x - wlp : wlp - x;
+            }
+            return k;
+        };
+        best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
+        auto score = [&](int32_t r) {
+            if (r != prev && mine(r) && !is_placed(placed, r)) {
+                const Key k = keyof(r);
+                if (key_less(k, best)) best = k;
+            }
+        };
+        if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
+        else xvisit_all(prev, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, score);
+        // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
+        if (threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            int32_t ptr = s_ptr;
+            while (ptr < n) {   // warp-wide skip over placed entries, 32 at a time
+                const bool pl = ptr + lane < n ? is_placed(placed, (int32_t)o[ptr + lane]) : false;
+                const unsigned m = __ballot_sync(0xffffffffu, !pl && ptr + lane < n);
+                if (m) { ptr += __ffs(m) - 1; break; }
+                ptr = min(ptr + 32, n);
+            }
+            if (lane == 0) s_ptr = ptr;
+            if (ptr < n) {
+                if (MODE != C_H21) {
+                    if (lane == 0) {
+                        const Key k = keyof((int32_t)o[ptr]);
+                        if (key_less(k, best)) best = k;
+                    }
+                } else {
+                    // class b0 = |b| of o[ptr]; inside it rows are ordered by (wl, r)
+                    const uint32_t b0 = nb_of((int32_t)o[ptr]);
+                    int32_t lo = ptr, hi = n;                     // class end: first index with |b| > b0
+                    while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (nb_of((int32_t)o[mid]) > b0) hi = mid; else lo = mid + 1; }
+                    const int32_t cend = lo;
+                    lo = ptr; hi = cend;                          // lb: first index with wl >= wl_prev
+                    while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (wl_of((int32_t)o[mid]) >= wlp) hi = mid; else lo = mid + 1; }
+                    const int32_t lb = lo;
+                    // up: first unplaced in [lb, cend)
+                    for (int32_t i = lb; i < cend; i += 32) {
+                        const bool ok = i + lane < cend && !is_placed(placed, (int32_t)o[i + lane]);
+                        const unsigned m = __ballot_sync(0xffffffffu, ok);
+                        if (m) {
+                            if (lane == 0) {
+                                const Key k = keyof((int32_t)o[i + __ffs(m) - 1]);
+                                if (key_less(k, best)) best = k;
+                            }
+                            break;
+                        }
+                    }
+                    // down: last unplaced in [ptr, lb), then the first unplaced of its wl run
+                    int32_t d = -1;
+                    for (int32_t i = lb - 1; i >= ptr; i -= 32) {
+                        const bool ok = i - lane >= ptr && !is_placed(placed, (int32_t)o[i - lane]);
+                        const unsigned m = __ballot_sync(0xffffffffu, ok);
+                        if (m) { d = i - (__ffs(m) - 1); break; }
+                    }
+                    if (d >= 0) {
+                        const uint32_t wd = wl_of((int32_t)o[d]);
+                        lo = ptr; hi = d;
+                        while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (wl_of((int32_t)o[mid]) >= wd) hi = mid; else lo = mid + 1; }
+                        for (int32_t i = lo; i <= d; i += 32) {
+                            const bool ok = i + lane <= d && !is_placed(placed, (int32_t)o[i + lane]);
+                            const unsigned m = __ballot_sync(0xffffffffu, ok);
+                            if (m) {
+                                if (lane == 0) {
+                                    const Key k = keyof((int32_t)o[i + __ffs(m) - 1]);
+                                    if (key_less(k, best)) best = k;
+                                }
+                                break;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        const Key nx = xblock_argmin(best, red[buf]);
+        if (threadIdx.x == 0) {
+            out[q] = (int32_t)nx.r;
+            atomicOr(placed + (nx.r >> 5), 1u << (nx.r & 31));
+        }
+        pprev = prev;
+        cached_pp = cached;
+        prev = (int32_t)nx.r;
+    }
+}
+
+spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t M, const Signatures &sig,
+                               const int32_t *nnz, const spmm_params &p, int64_t N, int32_t *perm, cudaStream_t s) {
+    const int64_t nblk = ceil_div(N, p.bw);
+    const int64_t nwin = ceil_div(M, W);
+    DevBuf win, bcnt, bptr, bcur, brow, keys, ord, placed, cnt;
+    SPMM_TRY(win.alloc(M * sizeof(int32_t), s));
+    k_win_of<<<grid_for(M, 256), 256, 0, s>>>(base, M, W, win.as<int32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    // inverted index: block -> rows (CSR over blocks)
+    SPMM_TRY(bcnt.alloc((nblk + 1) * sizeof(int32_t), s));
+    SPMM_TRY(bptr.alloc((nblk + 1) * sizeof(int32_t), s));
+    SPMM_TRY(bcur.alloc((nblk + 1) * sizeof(int32_t), s));
+    SPMM_CUDA(cudaMemsetAsync(bcnt.p, 0, (nblk + 1) * sizeof(int32_t), s));
+    SPMM_CUDA(cudaMemsetAsync(bcur.p, 0, (nblk + 1) * sizeof(int32_t), s));
+    if (sig.S > 0) {
+        k_blk_count<<<grid_for(sig.S, 256), 256, 0, s>>>(sig.blk.as<int32_t>(), sig.S, bcnt.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    SPMM_TRY(exclusive_scan_i32(bcnt.as<int32_t>(), bptr.as<int32_t>(), nblk + 1, nullptr, s));
+    SPMM_TRY(brow.alloc(std::max<int64_t>(sig.S, 1) * sizeof(int32_t), s));
+    if (sig.S > 0 && nwin > 1) {
+        DevBuf ek;
+        SPMM_TRY(ek.alloc(sig.S * sizeof(uint64_t), s));
+        k_blk_win_keys<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
+                                                          win.as<int32_t>(), ek.as<uint64_t>(),
+                                                          reinterpret_cast<uint32_t *>(brow.as<int32_t>()));
+        SPMM_CUDA(cudaGetLastError());
+        int bb = 0;
+        while (bb < 32 && ((uint64_t)nblk >> bb) != 0) ++bb;
+        SPMM_TRY(radix_sort_pairs(ek.as<uint64_t>(), reinterpret_cast<uint32_t *>(brow.as<int32_t>()), sig.S, 0,
+                                  32 + bb, s));
+    } else if (sig.S > 0) {
+        k_blk_fill<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
+                                                      bptr.as<int32_t>(), bcur.as<int32_t>(), brow.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+    }
+    // rows by (window, |b|, [wl,] r): two stable radix sorts over row ids in ascending order
+    SPMM_TRY(keys.alloc(M * sizeof(uint64_t), s));
+    SPMM_TRY(ord.alloc(M * sizeof(uint32_t), s));
+    k_xkeys<<<grid_for(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), nnz, M, p.nt, mode == C_H21 ? 1 : 0,
+                                             keys.as<uint64_t>(), ord.as<uint32_t>());
+    SPMM_CUDA(cudaGetLastError());
+    SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), ord.as<uint32_t>(), M, 0, mode == C_H21 ? 56 : 32, s));
+    if (nwin > 1) {
+        k_xkeys_win<<<grid_for(M, 256), 256, 0, s>>>(ord.as<uint32_t>(), win.as<int32_t>(), M, keys.as<uint64_t>());
+        SPMM_CUDA(cudaGetLastError());
+        SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), ord.as<uint32_t>(), M, 0, 32, s));
+    }
+    SPMM_TRY(placed.alloc(ceil_div(M, 32) * sizeof(uint32_t), s));
+    SPMM_CUDA(cudaMemsetAsync(placed.p, 0, ceil_div(M, 32) * sizeof(uint32_t), s));
+    SPMM_TRY(cnt.alloc(2 * M * sizeof(int32_t), s));
+    SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, 2 * M * sizeof(int32_t), s));
+    auto kern = mode == C_H21 ? k_chain_x<C_H21> : k_chain_x<C_CTA>;
+    kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
+                                                sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
+                                                win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt,
+                                                placed.as<uint32_t>(), cnt.as<int32_t>(), cnt.as<int32_t>() + M, perm);
+    SPMM_CUDA(cudaGetLastError());
+    return SPMM_OK;
+}
+
+// SPMM_CHAIN_EXACT=1: use the inverted-index builder for every CTA_AWARE / HYBRID_2_1 window size (tests
+// compare it with k_chain and the oracle at small sizes)
+bool force_exact_ix() {
+    const char *e = getenv("SPMM_CHAIN_EXACT");   // read per call (once per spmm_permute)
+    return e && atoi(e) != 0;
+}
+
 // plain sort (by nnz or by warp load), result row ids in vals (uint32[M]); keys kept for H1
 spmm_status sort_rows(const int32_t *nnz, int64_t M, int32_t nt, bool by_wl, int32_t max_nnz, DevBuf &keys, DevBuf &vals,
                       cudaStream_t s) {
@@ -493,8 +874,11 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
     }
     default: {   // chain policies over windows of a pre-order
         const int64_t W = (p.window == 0 || p.window > M) ? M : p.window;
-        if (W > CHAIN_MAX_N)
-            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows (use window > 0)");
+        const bool exact_ix = W > CHAIN_MAX_N &&
+                              (policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1);
+        if (W > CHAIN_MAX_N && !exact_ix)
+            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows: only CTA_AWARE and HYBRID_2_1 "
+                                              "(inverted-index builder)");
         int mode = policy == SPMM_POLICY_CTA_AWARE ? C_CTA : policy == SPMM_POLICY_HYBRID_2_1 ? C_H21 :
                    policy == SPMM_POLICY_HYBRID_2_2 ? C_H22 : policy == SPMM_POLICY_WARP_AWARE ? C_WARP : C_H23;
         Signatures sig;
@@ -518,6 +902,8 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
             k_iota<<<grid_for(M, 256), 256, 0, s>>>(base.as<int32_t>(), M);
         }
         SPMM_CUDA(cudaGetLastError());
+        if (exact_ix || (force_exact_ix() && (mode == C_CTA || mode == C_H21)))
+            return launch_chain_exact(mode, base.as<int32_t>(), W, M, sig, nnz, p, h->N, perm, s);
         return launch_chain(mode, base.as<int32_t>(), nullptr, ceil_div(M, W), W, M, sig, nnz, p, h->N, perm, s);
     }
     }

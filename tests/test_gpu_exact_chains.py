@@ -1,0 +1,108 @@
+"""GPU parity of the inverted-index chain builder (k_chain_x): paper-exact greedy chains
+over windows above 32768 rows, up to the whole matrix (W = 0).
+
+Small sizes: forced onto the inverted-index builder (SPMM_CHAIN_EXACT=1) and compared bit-exact with the
+oracle (oracle.c, O(W^2) brute force of the definition) for CTA_AWARE and HYBRID_2_1, whole-matrix and
+multi-window, original and MinHash pre-orders.  Full size (C2 stencil, M = 1M, W = 0): a bijection whose
+sampled steps are locally optimal under the policy key, checked with scipy sparse products (independent of
+both the oracle and the kernel: DESIGN.md §3).
+"""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synthetic as syn
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
+
+GENS = {
+    "rmat12_natural": lambda: syn.rmat(12, 12, 2100, "natural"),
+    "rmat13_local": lambda: syn.rmat(13, 8, 2101, "local"),
+    "stencil14": lambda: syn.stencil27(14, 2102),
+    "block_planted": lambda: syn.blockcluster(3000, 6000, 30, 3, 12, 2103, planted=True),
+    "uniform_poisson": lambda: syn.uniform(3500, 5000, 3, 2104, poisson=True),   # many empty rows
+    "banded": lambda: syn.banded(4000, 9, 40, 2105),
+}
+
+
+@pytest.fixture
+def exact_builder(monkeypatch):
+    monkeypatch.setenv("SPMM_CHAIN_EXACT", "1")
+    yield
+
+
+@pytest.mark.parametrize("name", list(GENS))
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1"])
+@pytest.mark.parametrize("window,preorder", [(0, 0), (1024, 0), (1024, 1)])
+def test_exact_builder_matches_oracle(exact_builder, name, policy, window, preorder):
+    a = GENS[name]()
+    h = pkg.SpMM.from_csr(a)
+    h.permute(policy, window=window, preorder=preorder, seed=7)
+    got = h.perm()
+    h.close()
+    ref = oracle.permute(a, policy, window=window, preorder=preorder, seed=7)
+    assert np.array_equal(got, ref), (name, policy, window, int(np.argmax(got != ref)))
+
+
+def test_exact_builder_matches_k_chain():
+    """Same answer as the shared-memory bitmap builder k_chain on a window it can also take (32768 rows)."""
+    a = syn.rmat(15, 6, 2110, "local")
+    h = pkg.SpMM.from_csr(a)
+    outs = []
+    for force in ("0", "1"):
+        os.environ["SPMM_CHAIN_EXACT"] = force
+        try:
+            h.permute("hybrid_2_1", window=32768)
+            outs.append(h.perm())
+        finally:
+            os.environ.pop("SPMM_CHAIN_EXACT", None)
+    h.close()
+    assert np.array_equal(outs[0], outs[1])
+
+
+def _block_matrix(a, bw=32):
+    import scipy.sparse as sp
+    rows = np.repeat(np.arange(a.M), np.diff(a.rowidx))
+    m = sp.csr_matrix((np.ones(a.nnz, dtype=np.int32), (rows, np.asarray(a.colidx) // bw)),
+                      shape=(a.M, (a.N + bw - 1) // bw))
+    m = m.tocsr()
+    m.sum_duplicates()
+    m.data[:] = 1                                     # duplicate (row, block) pairs summed -> back to 1
+    return m
+
+
+def check_sampled_steps(a, perm, policy, samples, seed=0, nt=32):
+    """At sampled positions q >= 1 the row placed at q minimises (ham(r, perm[q-1]), [|wl_r - wl_prev|,] r)
+    over the rows not placed before q (W = 0: one window, P:L122 / P:L134)."""
+    Bm = _block_matrix(a)
+    nb = np.diff(Bm.indptr).astype(np.int64)
+    wl = (np.diff(np.asarray(a.rowidx)).astype(np.int64) + nt - 1) // nt
+    pos = np.empty(a.M, dtype=np.int64)
+    pos[perm] = np.arange(a.M)
+    rng = np.random.default_rng(seed)
+    qs = np.unique(np.concatenate([[1, a.M - 1], rng.integers(1, a.M, samples)]))
+    for q in qs:
+        p = int(perm[q - 1])
+        inter = np.asarray((Bm @ Bm[p].T).todense()).ravel().astype(np.int64)
+        ham = nb + nb[p] - 2 * inter
+        cand = np.nonzero(pos >= q)[0]
+        k2 = np.abs(wl[cand] - wl[p]) if policy == "hybrid_2_1" else np.zeros(len(cand), dtype=np.int64)
+        order = np.lexsort((cand, k2, ham[cand]))
+        assert int(cand[order[0]]) == int(perm[q]), (policy, int(q))
+
+
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1"])
+def test_exact_whole_matrix_c2(policy):
+    """C2 (27-point stencil 100^3, M = 1M): the paper's whole-matrix chain (W = 0)."""
+    a = syn.stencil27(100, 2000)
+    h = pkg.SpMM.from_csr(a)
+    h.permute(policy, window=0)
+    perm = h.perm()
+    h.close()
+    assert np.array_equal(np.sort(perm), np.arange(a.M))
+    check_sampled_steps(a, perm, policy, samples=40)
