@@ -636,6 +636,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                 if (m) { ptr += __ffs(m) - 1; break; }
                 ptr = min(ptr + 32, n);
             }
+            __syncwarp();
             if (lane == 0) s_ptr = ptr;
             if (ptr < n) {
                 if (MODE != C_H21) {
@@ -719,7 +720,7 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t
         k_blk_count<<<grid_for(sig.S, 256), 256, 0, s>>>(sig.blk.as<int32_t>(), sig.S, bcnt.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
     }
-    SPMM_TRY(exclusive_scan_i32(bcnt.as<int32_t>(), bptr.as<int32_t>(), nblk + 1, nullptr, s));
+    SPMM_TRY(exclusive_scan_i32(bcnt.as<int32_t>(), bptr.as<int32_t>(), nblk, nullptr, s));   // bptr[nblk] = S
     SPMM_TRY(brow.alloc(std::max<int64_t>(sig.S, 1) * sizeof(int32_t), s));
     if (sig.S > 0 && nwin > 1) {
         DevBuf ek;

@@ -41,4 +41,14 @@ for pol in ("identity", "cta_aware"):
         h3.features_b200(K, current_order=True)
 h.features_b200(64)
 torch.cuda.synchronize()
+# inverted-index exact chains (k_chain_x): whole matrix and multi-window, both modes, an empty-row-rich input
+os.environ["SPMM_CHAIN_EXACT"] = "1"
+for a4 in (syn.uniform(1500, 2000, 3, 5, poisson=True), syn.rmat(10, 8, 6, "local")):
+    h4 = pkg.SpMM.from_csr(a4)
+    for pol in ("cta_aware", "hybrid_2_1"):
+        for W in (0, 256):
+            h4.permute(pol, window=W)
+    h4.close()
+os.environ.pop("SPMM_CHAIN_EXACT")
+torch.cuda.synchronize()
 print("sanitize driver done")
