@@ -763,11 +763,11 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t
     return SPMM_OK;
 }
 
-// SPMM_CHAIN_EXACT=1: use the inverted-index builder for every CTA_AWARE / HYBRID_2_1 window size (tests
-// compare it with k_chain and the oracle at small sizes)
-bool force_exact_ix() {
-    const char *e = getenv("SPMM_CHAIN_EXACT");   // read per call (once per spmm_permute)
-    return e && atoi(e) != 0;
+// SPMM_CHAIN_EXACT=1 / 0: force the inverted-index builder / k_chain for CTA_AWARE and HYBRID_2_1 where both
+// apply (W <= 32768); unset: -1, the measured rule in build_permutation.  Read per spmm_permute call.
+int force_exact_ix() {
+    const char *e = getenv("SPMM_CHAIN_EXACT");
+    return e && *e ? (atoi(e) != 0 ? 1 : 0) : -1;
 }
 
 // plain sort (by nnz or by warp load), result row ids in vals (uint32[M]); keys kept for H1
@@ -875,9 +875,16 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
     }
     default: {   // chain policies over windows of a pre-order
         const int64_t W = (p.window == 0 || p.window > M) ? M : p.window;
-        const bool exact_ix = W > CHAIN_MAX_N &&
-                              (policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1);
-        if (W > CHAIN_MAX_N && !exact_ix)
+        // builder choice (identical results, tests/test_gpu_exact_chains.py): k_chain scores every candidate of the
+        // window each step (cost ~ W * sum of the window's signature lengths), k_chain_x walks prev's posting
+        // lists; measured (profiles/r1_chain_builders.jsonl) k_chain_x wins for W >= 8192 and on inputs with hub
+        // rows (C3 1024: 2.0 -> 0.55 s, C5 1024: 5.3 -> 1.9 s), k_chain on short-row inputs at small W (C2 1024:
+        // 0.012 vs 0.047 s).  SPMM_CHAIN_EXACT=0 / 1 forces one builder where both apply.
+        const bool ix_ok = policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1;
+        const int fx = force_exact_ix();
+        const bool exact_ix = ix_ok && (W > CHAIN_MAX_N || fx == 1 ||
+                                        (fx < 0 && (W >= 8192 || h->max_row_nnz > 1024)));
+        if (W > CHAIN_MAX_N && !ix_ok)
             return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows: only CTA_AWARE and HYBRID_2_1 "
                                               "(inverted-index builder)");
         int mode = policy == SPMM_POLICY_CTA_AWARE ? C_CTA : policy == SPMM_POLICY_HYBRID_2_1 ? C_H21 :
@@ -903,7 +910,7 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
             k_iota<<<grid_for(M, 256), 256, 0, s>>>(base.as<int32_t>(), M);
         }
         SPMM_CUDA(cudaGetLastError());
-        if (exact_ix || (force_exact_ix() && (mode == C_CTA || mode == C_H21)))
+        if (exact_ix)
             return launch_chain_exact(mode, base.as<int32_t>(), W, M, sig, nnz, p, h->N, perm, s);
         return launch_chain(mode, base.as<int32_t>(), nullptr, ceil_div(M, W), W, M, sig, nnz, p, h->N, perm, s);
     }
