@@ -409,6 +409,17 @@ __global__ void k_win_of(const int32_t *base, int64_t M, int64_t W, int32_t *win
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < M; q += (int64_t)gridDim.x * blockDim.x)
         win[base[q]] = (int32_t)(q / W);
 }
+__global__ void k_win_of_seg(const int32_t *base, const int32_t *seg, int64_t nseg, int64_t M, int32_t *win) {
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < M; q += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = 0, hi = nseg - 1;              // last segment with seg[k] <= q
+        while (lo < hi) {
+            const int64_t mid = (lo + hi + 1) >> 1;
+            if (seg[mid] <= q) lo = mid;
+            else hi = mid - 1;
+        }
+        win[base[q]] = (int32_t)lo;
+    }
+}
 __global__ void k_blk_count(const int32_t *blk, int64_t S, int32_t *bcnt) {
     for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < S; t += (int64_t)gridDim.x * blockDim.x)
         atomicAdd(&bcnt[blk[t]], 1);
@@ -549,19 +560,22 @@ __device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, c
 }
 
 template <int MODE>
-__global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base, int64_t W, int64_t M, int multiwin,
+__global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base, const int32_t *seg, int64_t W,
+                                                            int64_t M, int multiwin,
                                                             const int32_t *sig_ptr, const int32_t *sig_blk,
                                                             const int32_t *bptr, const int32_t *brow,
                                                             const int32_t *win, const uint32_t *ord,
-                                                            const int32_t *nnz, int32_t nt, uint32_t *placed,
-                                                            int32_t *cnt0, int32_t *cnt1, int32_t *perm) {
+                                                            const int32_t *nnz, int32_t nt, int32_t nw,
+                                                            uint32_t *placed, int32_t *cnt0, int32_t *cnt1,
+                                                            int32_t *perm) {
     __shared__ int32_t pre[2][XCH_CACHE + 1];
     __shared__ int32_t bst[2][XCH_CACHE];
     __shared__ int32_t wsum[32];
     __shared__ Key red[2][XCH_THREADS / 32];
     __shared__ int32_t s_ptr;
     const int32_t w = (int32_t)blockIdx.x;
-    const int64_t s0 = (int64_t)w * W, s1 = min(s0 + W, M);
+    // window w = positions [s0, s1) of the pre-order: fixed windows of W, or HYBRID_1's segments (seg)
+    const int64_t s0 = seg ? seg[w] : (int64_t)w * W, s1 = seg ? seg[w + 1] : min(s0 + W, M);
     const int32_t n = (int32_t)(s1 - s0);
     const uint32_t *o = ord + s0;            // the window's rows by (|b|, [wl,] r)
     int32_t *out = perm + s0;
@@ -570,48 +584,61 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     const int32_t mw = multiwin ? w : -1;    // lists sorted by window: visit only this window's rows
     auto mine = [&](int32_t r) -> bool { return true; };
     if (n <= 0) return;
-    // first row: least (wl, r) of the window (as k_chain)
-    Key best{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
-    for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
-        const int32_t r = base[s0 + a];
-        Key c{wl_of(r), 0u, (uint32_t)r, 0u};
-        if (key_less(c, best)) best = c;
-    }
-    Key win0 = xblock_argmin(best, red[0]);
-    int32_t prev = (int32_t)win0.r, pprev = -1;
-    if (threadIdx.x == 0) {
-        out[0] = prev;
-        atomicOr(placed + (prev >> 5), 1u << (prev & 31));
-        s_ptr = 0;
+    // first row(s): least (wl, r) of the window's unplaced rows -- 1 row (CTA_AWARE, HYBRID_2_1), nw rows
+    // (WARP_AWARE, HYBRID_2_3: "the first 32 rows are those ... with the lowest warp load"), as k_chain
+    // (HYBRID_1: every row of a segment has the same wl and the segment lists them in ascending id, so its
+    //  least (wl, r) is its first row -- the row P:L132 / reading A8 starts the segment with)
+    constexpr bool WARPREF = MODE == C_WARP || MODE == C_H23;   // Hamming reference out[q - nw], else prev
+    const int32_t nfirst = WARPREF ? min(n, nw) : 1;
+    Key best;
+    int32_t prev = -1, pprev = -1, pref = -1;
+    for (int32_t q = 0; q < nfirst; ++q) {
+        best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
+        for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
+            const int32_t r = base[s0 + a];
+            if (q > 0 && is_placed(placed, r)) continue;
+            Key c{wl_of(r), 0u, (uint32_t)r, 0u};
+            if (key_less(c, best)) best = c;
+        }
+        const Key w0 = xblock_argmin(best, red[q & 1]);
+        prev = (int32_t)w0.r;
+        if (threadIdx.x == 0) {
+            out[q] = prev;
+            atomicOr(placed + (prev >> 5), 1u << (prev & 31));
+            s_ptr = 0;
+        }
+        __syncthreads();
     }
     bool cached_pp = false;
-    for (int32_t q = 1; q < n; ++q) {
+    for (int32_t q = nfirst; q < n; ++q) {
         const int buf = q & 1;
         int32_t *cc = buf ? cnt1 : cnt0, *co = buf ? cnt0 : cnt1;
-        const int32_t bs = sig_ptr[prev], be = sig_ptr[prev + 1];
+        const int32_t ref = WARPREF ? out[q - nw] : prev;       // the row Hamming distances are taken to
+        const int32_t bs = sig_ptr[ref], be = sig_ptr[ref + 1];
         const uint32_t cp = (uint32_t)(be - bs);
         const bool cached = be - bs <= XCH_CACHE;
-        // prefix of prev's lists (kept for the score pass and for the next step's reset); the previous
+        // prefix of ref's lists (kept for the score pass and for the next step's reset); the previous
         // step's prefix lives in the other buffer
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw);
-        // reset the previous step's counters (other buffer), then count |b_r ∩ b_prev|
+        // reset the previous step's counters (other buffer), then count |b_r ∩ b_ref|
         // (only this window's rows: the other windows' CTAs count theirs in the same arrays)
-        if (pprev >= 0) {
+        if (pref >= 0) {
             auto reset = [&](int32_t r) { if (mine(r)) co[r] = 0; };
-            if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pprev + 1] - sig_ptr[pprev], brow, reset);
-            else xvisit_all(pprev, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, reset);
+            if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], brow, reset);
+            else xvisit_all(pref, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, reset);
         }
         auto count = [&](int32_t r) {
             if (r != prev && mine(r) && !is_placed(placed, r)) atomicAdd(cc + r, 1);
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
-        else xvisit_all(prev, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
         __syncthreads();
-        const uint32_t wlp = MODE == C_H21 ? wl_of(prev) : 0u;
+        constexpr bool WLTIE = MODE == C_H21 || MODE == C_H23;      // tie: |wl_r - wl_prev|
+        const uint32_t wlp = WLTIE ? wl_of(prev) : 0u;
         auto keyof = [&](int32_t r) -> Key {
             const uint32_t c = (uint32_t)__ldcg(cc + r);
             Key k{cp + nb_of(r) - 2u * c, 0u, (uint32_t)r, 0u};
-            if (MODE == C_H21) {
+            if (WLTIE) {
                 const uint32_t x = wl_of(r);
                 k.k2 = x > wlp ? x - wlp : wlp - x;
             }
@@ -625,7 +652,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
             }
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
-        else xvisit_all(prev, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, score);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, score);
         // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
         if (threadIdx.x < 32) {
             const int lane = threadIdx.x;
@@ -639,7 +666,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
             __syncwarp();
             if (lane == 0) s_ptr = ptr;
             if (ptr < n) {
-                if (MODE != C_H21) {
+                if (!WLTIE) {
                     if (lane == 0) {
                         const Key k = keyof((int32_t)o[ptr]);
                         if (key_less(k, best)) best = k;
@@ -697,18 +724,22 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
             atomicOr(placed + (nx.r >> 5), 1u << (nx.r & 31));
         }
         pprev = prev;
+        pref = ref;
         cached_pp = cached;
         prev = (int32_t)nx.r;
     }
 }
 
-spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t M, const Signatures &sig,
-                               const int32_t *nnz, const spmm_params &p, int64_t N, int32_t *perm, cudaStream_t s) {
+// seg != nullptr: HYBRID_1's nseg segments (positions seg[k] .. seg[k+1]) instead of windows of W
+spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg, int64_t nseg, int64_t W, int64_t M,
+                               const Signatures &sig, const int32_t *nnz, const spmm_params &p, int64_t N,
+                               int32_t *perm, cudaStream_t s) {
     const int64_t nblk = ceil_div(N, p.bw);
-    const int64_t nwin = ceil_div(M, W);
+    const int64_t nwin = seg ? nseg : ceil_div(M, W);
     DevBuf win, bcnt, bptr, bcur, brow, keys, ord, placed, cnt;
     SPMM_TRY(win.alloc(M * sizeof(int32_t), s));
-    k_win_of<<<grid_for(M, 256), 256, 0, s>>>(base, M, W, win.as<int32_t>());
+    if (seg) k_win_of_seg<<<grid_for(M, 256), 256, 0, s>>>(base, seg, nseg, M, win.as<int32_t>());
+    else k_win_of<<<grid_for(M, 256), 256, 0, s>>>(base, M, W, win.as<int32_t>());
     SPMM_CUDA(cudaGetLastError());
     // inverted index: block -> rows (CSR over blocks)
     SPMM_TRY(bcnt.alloc((nblk + 1) * sizeof(int32_t), s));
@@ -741,10 +772,11 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t
     // rows by (window, |b|, [wl,] r): two stable radix sorts over row ids in ascending order
     SPMM_TRY(keys.alloc(M * sizeof(uint64_t), s));
     SPMM_TRY(ord.alloc(M * sizeof(uint32_t), s));
-    k_xkeys<<<grid_for(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), nnz, M, p.nt, mode == C_H21 ? 1 : 0,
+    const bool with_wl = mode == C_H21 || mode == C_H23;
+    k_xkeys<<<grid_for(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), nnz, M, p.nt, with_wl ? 1 : 0,
                                              keys.as<uint64_t>(), ord.as<uint32_t>());
     SPMM_CUDA(cudaGetLastError());
-    SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), ord.as<uint32_t>(), M, 0, mode == C_H21 ? 56 : 32, s));
+    SPMM_TRY(radix_sort_pairs(keys.as<uint64_t>(), ord.as<uint32_t>(), M, 0, with_wl ? 56 : 32, s));
     if (nwin > 1) {
         k_xkeys_win<<<grid_for(M, 256), 256, 0, s>>>(ord.as<uint32_t>(), win.as<int32_t>(), M, keys.as<uint64_t>());
         SPMM_CUDA(cudaGetLastError());
@@ -754,10 +786,11 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, int64_t W, int64_t
     SPMM_CUDA(cudaMemsetAsync(placed.p, 0, ceil_div(M, 32) * sizeof(uint32_t), s));
     SPMM_TRY(cnt.alloc(2 * M * sizeof(int32_t), s));
     SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, 2 * M * sizeof(int32_t), s));
-    auto kern = mode == C_H21 ? k_chain_x<C_H21> : k_chain_x<C_CTA>;
-    kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
+    auto kern = mode == C_H21 ? k_chain_x<C_H21> : mode == C_WARP ? k_chain_x<C_WARP>
+              : mode == C_H23 ? k_chain_x<C_H23> : k_chain_x<C_CTA>;     // HYBRID_1 = C_CTA over segments
+    kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
-                                                win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt,
+                                                win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt, p.nw,
                                                 placed.as<uint32_t>(), cnt.as<int32_t>(), cnt.as<int32_t>() + M, perm);
     SPMM_CUDA(cudaGetLastError());
     return SPMM_OK;
@@ -865,12 +898,17 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
         k_compact_starts<<<grid_for(M, 256), 256, 0, s>>>(flag.as<int32_t>(), pos.as<int32_t>(), M, starts.as<int32_t>());
         k_set_last<<<1, 1, 0, s>>>(starts.as<int32_t>(), nseg, (int32_t)M);
         SPMM_CUDA(cudaGetLastError());
-        if (W > CHAIN_MAX_N) return fail(SPMM_ERR_UNSUPPORTED, "HYBRID_1: segment window above 32768 rows");
         SPMM_TRY(base.alloc(M * sizeof(int32_t), s));
         k_u32_to_i32<<<grid_for(M, 256), 256, 0, s>>>(vals.as<uint32_t>(), M, base.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
         Signatures sig;
         SPMM_TRY(build_signatures(h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), nullptr, M, h->nnz, p.bw, sig, s));
+        // segments above 32768 rows (or forced, or hub rows at large W): the inverted-index builder, HYBRID_1
+        // being CTA_AWARE's key over each segment (same rule as the chain policies below)
+        const int fx = force_exact_ix();
+        if (W > CHAIN_MAX_N || fx == 1 || (fx < 0 && (W >= 8192 || h->max_row_nnz > 1024)))
+            return launch_chain_exact(C_CTA, base.as<int32_t>(), starts.as<int32_t>(), nseg, 0, M, sig, nnz, p, h->N,
+                                      perm, s);
         return launch_chain(C_H1, base.as<int32_t>(), starts.as<int32_t>(), nseg, 0, M, sig, nnz, p, h->N, perm, s);
     }
     default: {   // chain policies over windows of a pre-order
@@ -880,13 +918,14 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
         // lists; measured (profiles/r1_chain_builders.jsonl) k_chain_x wins for W >= 8192 and on inputs with hub
         // rows (C3 1024: 2.0 -> 0.55 s, C5 1024: 5.3 -> 1.9 s), k_chain on short-row inputs at small W (C2 1024:
         // 0.012 vs 0.047 s).  SPMM_CHAIN_EXACT=0 / 1 forces one builder where both apply.
-        const bool ix_ok = policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1;
+        const bool ix_ok = policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1 ||
+                           policy == SPMM_POLICY_WARP_AWARE || policy == SPMM_POLICY_HYBRID_2_3;
         const int fx = force_exact_ix();
         const bool exact_ix = ix_ok && (W > CHAIN_MAX_N || fx == 1 ||
                                         (fx < 0 && (W >= 8192 || h->max_row_nnz > 1024)));
         if (W > CHAIN_MAX_N && !ix_ok)
-            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows: only CTA_AWARE and HYBRID_2_1 "
-                                              "(inverted-index builder)");
+            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows: only CTA_AWARE, HYBRID_2_1, "
+                                              "WARP_AWARE and HYBRID_2_3 (inverted-index builder)");
         int mode = policy == SPMM_POLICY_CTA_AWARE ? C_CTA : policy == SPMM_POLICY_HYBRID_2_1 ? C_H21 :
                    policy == SPMM_POLICY_HYBRID_2_2 ? C_H22 : policy == SPMM_POLICY_WARP_AWARE ? C_WARP : C_H23;
         Signatures sig;
@@ -911,7 +950,7 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
         }
         SPMM_CUDA(cudaGetLastError());
         if (exact_ix)
-            return launch_chain_exact(mode, base.as<int32_t>(), W, M, sig, nnz, p, h->N, perm, s);
+            return launch_chain_exact(mode, base.as<int32_t>(), nullptr, 0, W, M, sig, nnz, p, h->N, perm, s);
         return launch_chain(mode, base.as<int32_t>(), nullptr, ceil_div(M, W), W, M, sig, nnz, p, h->N, perm, s);
     }
     }

@@ -37,7 +37,7 @@ def exact_builder(monkeypatch):
 
 
 @pytest.mark.parametrize("name", list(GENS))
-@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1"])
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3", "hybrid_1"])
 @pytest.mark.parametrize("window,preorder", [(0, 0), (1024, 0), (1024, 1)])
 def test_exact_builder_matches_oracle(exact_builder, name, policy, window, preorder):
     a = GENS[name]()
@@ -76,27 +76,31 @@ def _block_matrix(a, bw=32):
     return m
 
 
-def check_sampled_steps(a, perm, policy, samples, seed=0, nt=32):
-    """At sampled positions q >= 1 the row placed at q minimises (ham(r, perm[q-1]), [|wl_r - wl_prev|,] r)
-    over the rows not placed before q (W = 0: one window, P:L122 / P:L134)."""
+def check_sampled_steps(a, perm, policy, samples, seed=0, nt=32, nw=32):
+    """At sampled positions q the row placed at q minimises (ham(r, ref), [|wl_r - wl_prev|,] r) over the rows not
+    placed before q; ref = perm[q-1] (CTA_AWARE, HYBRID_2_1: P:L122, L134) or perm[q-nw] for q >= nw (WARP_AWARE,
+    HYBRID_2_3: P:L118-120, L146); wl_prev = wl of perm[q-1].  W = 0: one window."""
     Bm = _block_matrix(a)
     nb = np.diff(Bm.indptr).astype(np.int64)
     wl = (np.diff(np.asarray(a.rowidx)).astype(np.int64) + nt - 1) // nt
     pos = np.empty(a.M, dtype=np.int64)
     pos[perm] = np.arange(a.M)
     rng = np.random.default_rng(seed)
-    qs = np.unique(np.concatenate([[1, a.M - 1], rng.integers(1, a.M, samples)]))
+    back = nw if policy in ("warp_aware", "hybrid_2_3") else 1
+    qs = np.unique(np.concatenate([[back, a.M - 1], rng.integers(back, a.M, samples)]))
     for q in qs:
-        p = int(perm[q - 1])
+        p = int(perm[q - back])
         inter = np.asarray((Bm @ Bm[p].T).todense()).ravel().astype(np.int64)
         ham = nb + nb[p] - 2 * inter
         cand = np.nonzero(pos >= q)[0]
-        k2 = np.abs(wl[cand] - wl[p]) if policy == "hybrid_2_1" else np.zeros(len(cand), dtype=np.int64)
+        wprev = wl[int(perm[q - 1])]
+        k2 = (np.abs(wl[cand] - wprev) if policy in ("hybrid_2_1", "hybrid_2_3")
+              else np.zeros(len(cand), dtype=np.int64))
         order = np.lexsort((cand, k2, ham[cand]))
         assert int(cand[order[0]]) == int(perm[q]), (policy, int(q))
 
 
-@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1"])
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3"])
 def test_exact_whole_matrix_c2(policy):
     """C2 (27-point stencil 100^3, M = 1M): the paper's whole-matrix chain (W = 0)."""
     a = syn.stencil27(100, 2000)
