@@ -39,8 +39,7 @@ typedef enum {
     SPMM_ERR_INVALID_ARG = 1,  /* NULL pointer, negative size, size >= 2^31, bad window/params   */
     SPMM_ERR_INVALID_CSR = 2,  /* rowidx[0]!=0, rowidx[M]!=nnz, decreasing offsets, column out of
                                   range, or columns not strictly increasing within a row         */
-    SPMM_ERR_UNSUPPORTED = 3,  /* K % 4 != 0, K > 1024, misaligned B/C, chain window > 32768 rows for
-                                  HYBRID_2_2                                                         */
+    SPMM_ERR_UNSUPPORTED = 3,  /* K % 4 != 0, K > 1024, misaligned B/C                            */
     SPMM_ERR_CUDA = 4,         /* a CUDA runtime error (text in spmm_last_error)                  */
     SPMM_ERR_OOM = 5,          /* device allocation failed                                        */
     SPMM_ERR_STATE = 6         /* handle used on a device other than the one it was created on    */
@@ -71,8 +70,8 @@ typedef struct {
                                partial sums are combined in a fixed pairwise order; default 128
                                (bounds every fp32 accumulation chain, DESIGN.md §"Accuracy")         */
     int64_t window;         /* greedy-chain window W (multiple of nw); 0 = whole matrix (paper-exact,
-                               P:L118-122).  W <= 32768: every chain policy; above (up to W = M):
-                               all but HYBRID_2_2 through the inverted-index builder (f3,
+                               P:L118-122).  Every chain policy at any W (up to W = M); above 32768
+                               rows through the inverted-index builder (f3,
                                DESIGN.md §8; cost grows with the posting lists of hub blocks).
                                Default 1024                                                            */
     int32_t preorder;       /* chain policies: windows over 0 = the original order, 1 = the MinHash key

@@ -567,7 +567,13 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                                                             const int32_t *win, const uint32_t *ord,
                                                             const int32_t *nnz, int32_t nt, int32_t nw,
                                                             uint32_t *placed, int32_t *cnt0, int32_t *cnt1,
-                                                            int32_t *perm) {
+                                                            int32_t *cnt2a, int32_t *cnt2b, int32_t *perm) {
+    // HYBRID_2_2: key (ham(r, prev), q >= nw ? ham(r, out[q - nw]) : 0, r) -- a second reference ref2
+    // with its own counters (cnt2a/b) and scratch; the argmin lies in T1 ∪ (T2 ∩ class b0) ∪ {u*}
+    constexpr bool TWOREF = MODE == C_H22;
+    constexpr int C2 = TWOREF ? XCH_CACHE : 1;
+    __shared__ int32_t pre2[C2 + 1];
+    __shared__ int32_t bst2[C2];
     __shared__ int32_t pre[2][XCH_CACHE + 1];
     __shared__ int32_t bst[2][XCH_CACHE];
     __shared__ int32_t wsum[32];
@@ -591,7 +597,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     constexpr bool WARPREF = MODE == C_WARP || MODE == C_H23;   // Hamming reference out[q - nw], else prev
     const int32_t nfirst = WARPREF ? min(n, nw) : 1;
     Key best;
-    int32_t prev = -1, pprev = -1, pref = -1;
+    int32_t prev = -1, pprev = -1, pref = -1, pref2 = -1;
     for (int32_t q = 0; q < nfirst; ++q) {
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
         for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
@@ -632,6 +638,21 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
+        int32_t ref2 = -1;
+        int32_t *cc2 = buf ? cnt2b : cnt2a;
+        uint32_t cp2 = 0;
+        if constexpr (TWOREF) {
+            int32_t *co2 = buf ? cnt2a : cnt2b;
+            if (pref2 >= 0)
+                xvisit_all(pref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) { co2[r] = 0; });
+            ref2 = q >= nw ? out[q - nw] : -1;
+            if (ref2 >= 0) {
+                cp2 = nb_of(ref2);
+                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {
+                    if (r != prev && !is_placed(placed, r)) atomicAdd(cc2 + r, 1);
+                });
+            }
+        }
         __syncthreads();
         constexpr bool WLTIE = MODE == C_H21 || MODE == C_H23;      // tie: |wl_r - wl_prev|
         const uint32_t wlp = WLTIE ? wl_of(prev) : 0u;
@@ -642,6 +663,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                 const uint32_t x = wl_of(r);
                 k.k2 = x > wlp ? x - wlp : wlp - x;
             }
+            if (TWOREF && ref2 >= 0) k.k2 = cp2 + nb_of(r) - 2u * (uint32_t)__ldcg(cc2 + r);
             return k;
         };
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
@@ -653,6 +675,32 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, score);
+        if constexpr (TWOREF) {
+            if (ref2 >= 0) {
+                // T2 ∩ class b0: b0 = |b| of the first unplaced row of the (|b|, r) order
+                if (threadIdx.x < 32) {
+                    const int lane = threadIdx.x;
+                    int32_t ptr = s_ptr;
+                    while (ptr < n) {
+                        const bool pl = ptr + lane < n ? is_placed(placed, (int32_t)o[ptr + lane]) : false;
+                        const unsigned m = __ballot_sync(0xffffffffu, !pl && ptr + lane < n);
+                        if (m) { ptr += __ffs(m) - 1; break; }
+                        ptr = min(ptr + 32, n);
+                    }
+                    __syncwarp();
+                    if (lane == 0) s_ptr = ptr;
+                }
+                __syncthreads();
+                const int32_t ptr = s_ptr;
+                const uint32_t b0 = ptr < n ? nb_of((int32_t)o[ptr]) : 0xffffffffu;
+                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {
+                    if (r != prev && !is_placed(placed, r) && nb_of(r) == b0) {
+                        const Key k = keyof(r);
+                        if (key_less(k, best)) best = k;
+                    }
+                });
+            }
+        }
         // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
         if (threadIdx.x < 32) {
             const int lane = threadIdx.x;
@@ -725,6 +773,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         }
         pprev = prev;
         pref = ref;
+        pref2 = ref2;
         cached_pp = cached;
         prev = (int32_t)nx.r;
     }
@@ -784,14 +833,18 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
     }
     SPMM_TRY(placed.alloc(ceil_div(M, 32) * sizeof(uint32_t), s));
     SPMM_CUDA(cudaMemsetAsync(placed.p, 0, ceil_div(M, 32) * sizeof(uint32_t), s));
-    SPMM_TRY(cnt.alloc(2 * M * sizeof(int32_t), s));
-    SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, 2 * M * sizeof(int32_t), s));
+    const int64_t ncnt = mode == C_H22 ? 4 : 2;
+    SPMM_TRY(cnt.alloc(ncnt * M * sizeof(int32_t), s));
+    SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, ncnt * M * sizeof(int32_t), s));
     auto kern = mode == C_H21 ? k_chain_x<C_H21> : mode == C_WARP ? k_chain_x<C_WARP>
-              : mode == C_H23 ? k_chain_x<C_H23> : k_chain_x<C_CTA>;     // HYBRID_1 = C_CTA over segments
+              : mode == C_H23 ? k_chain_x<C_H23> : mode == C_H22 ? k_chain_x<C_H22>
+              : k_chain_x<C_CTA>;                                       // HYBRID_1 = C_CTA over segments
     kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
                                                 win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt, p.nw,
-                                                placed.as<uint32_t>(), cnt.as<int32_t>(), cnt.as<int32_t>() + M, perm);
+                                                placed.as<uint32_t>(), cnt.as<int32_t>(), cnt.as<int32_t>() + M,
+                                                mode == C_H22 ? cnt.as<int32_t>() + 2 * M : nullptr,
+                                                mode == C_H22 ? cnt.as<int32_t>() + 3 * M : nullptr, perm);
     SPMM_CUDA(cudaGetLastError());
     return SPMM_OK;
 }
@@ -918,14 +971,8 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
         // lists; measured (profiles/r1_chain_builders.jsonl) k_chain_x wins for W >= 8192 and on inputs with hub
         // rows (C3 1024: 2.0 -> 0.55 s, C5 1024: 5.3 -> 1.9 s), k_chain on short-row inputs at small W (C2 1024:
         // 0.012 vs 0.047 s).  SPMM_CHAIN_EXACT=0 / 1 forces one builder where both apply.
-        const bool ix_ok = policy == SPMM_POLICY_CTA_AWARE || policy == SPMM_POLICY_HYBRID_2_1 ||
-                           policy == SPMM_POLICY_WARP_AWARE || policy == SPMM_POLICY_HYBRID_2_3;
         const int fx = force_exact_ix();
-        const bool exact_ix = ix_ok && (W > CHAIN_MAX_N || fx == 1 ||
-                                        (fx < 0 && (W >= 8192 || h->max_row_nnz > 1024)));
-        if (W > CHAIN_MAX_N && !ix_ok)
-            return fail(SPMM_ERR_UNSUPPORTED, "greedy chain window above 32768 rows: only CTA_AWARE, HYBRID_2_1, "
-                                              "WARP_AWARE and HYBRID_2_3 (inverted-index builder)");
+        const bool exact_ix = W > CHAIN_MAX_N || fx == 1 || (fx < 0 && (W >= 8192 || h->max_row_nnz > 1024));
         int mode = policy == SPMM_POLICY_CTA_AWARE ? C_CTA : policy == SPMM_POLICY_HYBRID_2_1 ? C_H21 :
                    policy == SPMM_POLICY_HYBRID_2_2 ? C_H22 : policy == SPMM_POLICY_WARP_AWARE ? C_WARP : C_H23;
         Signatures sig;

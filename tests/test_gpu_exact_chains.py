@@ -37,7 +37,7 @@ def exact_builder(monkeypatch):
 
 
 @pytest.mark.parametrize("name", list(GENS))
-@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3", "hybrid_1"])
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3", "hybrid_1", "hybrid_2_2"])
 @pytest.mark.parametrize("window,preorder", [(0, 0), (1024, 0), (1024, 1)])
 def test_exact_builder_matches_oracle(exact_builder, name, policy, window, preorder):
     a = GENS[name]()

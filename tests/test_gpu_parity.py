@@ -247,10 +247,7 @@ def test_errors():
     assert ex.value.status == 1
     big = syn.rmat(16, 2, 5)
     hb = pkg.SpMM.from_csr(big)
-    with pytest.raises(pkg.SpmmError) as ex:
-        hb.permute("hybrid_2_2", window=0)         # W=0 above 32768 rows: no inverted-index builder for 2.2
-    assert ex.value.status == 3
-    hb.permute("cta_aware", window=0)              # ... CTA-aware has one (k_chain_x, f3)
+    hb.permute("cta_aware", window=0)              # W=0 above 32768 rows: the inverted-index builder (f3)
     assert np.array_equal(np.sort(hb.perm()), np.arange(big.M))
     hb.close()
     h.close()
