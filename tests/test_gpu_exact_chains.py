@@ -79,7 +79,8 @@ def _block_matrix(a, bw=32):
 def check_sampled_steps(a, perm, policy, samples, seed=0, nt=32, nw=32):
     """At sampled positions q the row placed at q minimises (ham(r, ref), [|wl_r - wl_prev|,] r) over the rows not
     placed before q; ref = perm[q-1] (CTA_AWARE, HYBRID_2_1: P:L122, L134) or perm[q-nw] for q >= nw (WARP_AWARE,
-    HYBRID_2_3: P:L118-120, L146); wl_prev = wl of perm[q-1].  W = 0: one window."""
+    HYBRID_2_3: P:L118-120, L146); wl_prev = wl of perm[q-1]; HYBRID_2_2's second key is ham(r, perm[q-nw]) for
+    q >= nw.  W = 0: one window."""
     Bm = _block_matrix(a)
     nb = np.diff(Bm.indptr).astype(np.int64)
     wl = (np.diff(np.asarray(a.rowidx)).astype(np.int64) + nt - 1) // nt
@@ -94,13 +95,19 @@ def check_sampled_steps(a, perm, policy, samples, seed=0, nt=32, nw=32):
         ham = nb + nb[p] - 2 * inter
         cand = np.nonzero(pos >= q)[0]
         wprev = wl[int(perm[q - 1])]
-        k2 = (np.abs(wl[cand] - wprev) if policy in ("hybrid_2_1", "hybrid_2_3")
-              else np.zeros(len(cand), dtype=np.int64))
+        if policy in ("hybrid_2_1", "hybrid_2_3"):
+            k2 = np.abs(wl[cand] - wprev)
+        elif policy == "hybrid_2_2" and q >= nw:      # second key: Hamming to perm[q - nw]
+            p2 = int(perm[q - nw])
+            inter2 = np.asarray((Bm @ Bm[p2].T).todense()).ravel().astype(np.int64)
+            k2 = (nb + nb[p2] - 2 * inter2)[cand]
+        else:
+            k2 = np.zeros(len(cand), dtype=np.int64)
         order = np.lexsort((cand, k2, ham[cand]))
         assert int(cand[order[0]]) == int(perm[q]), (policy, int(q))
 
 
-@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3"])
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3", "hybrid_2_2"])
 def test_exact_whole_matrix_c2(policy):
     """C2 (27-point stencil 100^3, M = 1M): the paper's whole-matrix chain (W = 0)."""
     a = syn.stencil27(100, 2000)
