@@ -290,7 +290,7 @@ def main():
     ap.add_argument("--window", type=int, default=1024)
     ap.add_argument("--policy-steps", type=int, default=5, help="timed steps per policy for the exhaustive selection")
     ap.add_argument("--e2e-steps", type=int, default=5)
-    ap.add_argument("--ref-sample-nnz", type=int, default=400_000)
+    ap.add_argument("--ref-sample-nnz", type=int, default=10_000_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-ceiling", action="store_true", help="skip the host LRU model of L2 reuse")
