@@ -492,8 +492,9 @@ __device__ __forceinline__ int32_t lower_win(const int32_t *brow, const int32_t 
     }
     return lo;
 }
+template <class PT>
 __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *bptr, int32_t c0, int32_t nb,
-                                        int32_t *pre, int32_t *bst, int32_t *wsum, const int32_t *brow = nullptr,
+                                        PT *pre, int32_t *bst, PT *wsum, const int32_t *brow = nullptr,
                                         const int32_t *win = nullptr, int32_t mwin = -1) {
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     int32_t len = 0;
@@ -507,19 +508,19 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
         len = e - a;
         bst[tid] = a;
     }
-    int32_t x = len;
+    PT x = len;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        const int32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        const PT y = __shfl_up_sync(0xffffffffu, x, o);
         if (lane >= o) x += y;
     }
     if (lane == 31) wsum[wid] = x;
     __syncthreads();
     if (wid == 0) {
-        int32_t w = wsum[lane];
+        PT w = wsum[lane];
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const int32_t y = __shfl_up_sync(0xffffffffu, w, o);
+            const PT y = __shfl_up_sync(0xffffffffu, w, o);
             if (lane >= o) w += y;
         }
         wsum[lane] = w;
@@ -531,10 +532,11 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
 }
 
 // visit every entry of the posting lists described by (pre, bst, nb): f(row)
-template <class F>
-__device__ __forceinline__ void xvisit(const int32_t *pre, const int32_t *bst, int32_t nb, const int32_t *brow, F f) {
-    const int32_t T = pre[nb];
-    for (int32_t e = threadIdx.x; e < T; e += XCH_THREADS) {
+// PT: prefix type -- int32 when 1024 x the longest posting list fits (the host checks), else int64
+template <class PT, class F>
+__device__ __forceinline__ void xvisit(const PT *pre, const int32_t *bst, int32_t nb, const int32_t *brow, F f) {
+    const PT T = pre[nb];
+    for (PT e = threadIdx.x; e < T; e += XCH_THREADS) {
         int lo = 0, hi = nb - 1;
         while (lo < hi) {
             const int mid = (lo + hi + 1) >> 1;
@@ -546,10 +548,10 @@ __device__ __forceinline__ void xvisit(const int32_t *pre, const int32_t *bst, i
 }
 
 // all entries of row r0's lists, chunked by XCH_THREADS blocks (re-derives the prefix; barriers inside)
-template <class F>
+template <class PT, class F>
 __device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, const int32_t *sig_blk,
-                                           const int32_t *bptr, const int32_t *brow, int32_t *pre, int32_t *bst,
-                                           int32_t *wsum, const int32_t *win, int32_t mwin, F f) {
+                                           const int32_t *bptr, const int32_t *brow, PT *pre, int32_t *bst,
+                                           PT *wsum, const int32_t *win, int32_t mwin, F f) {
     const int32_t bs = sig_ptr[r0], be = sig_ptr[r0 + 1];
     for (int32_t c0 = bs; c0 < be; c0 += XCH_THREADS) {
         const int32_t nb = min(XCH_THREADS, be - c0);
@@ -559,7 +561,7 @@ __device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, c
     }
 }
 
-template <int MODE>
+template <int MODE, class PT>
 __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base, const int32_t *seg, int64_t W,
                                                             int64_t M, int multiwin,
                                                             const int32_t *sig_ptr, const int32_t *sig_blk,
@@ -572,11 +574,11 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     // with its own counters (cnt2a/b) and scratch; the argmin lies in T1 ∪ (T2 ∩ class b0) ∪ {u*}
     constexpr bool TWOREF = MODE == C_H22;
     constexpr int C2 = TWOREF ? XCH_CACHE : 1;
-    __shared__ int32_t pre2[C2 + 1];
+    __shared__ PT pre2[C2 + 1];
     __shared__ int32_t bst2[C2];
-    __shared__ int32_t pre[2][XCH_CACHE + 1];
+    __shared__ PT pre[2][XCH_CACHE + 1];
     __shared__ int32_t bst[2][XCH_CACHE];
-    __shared__ int32_t wsum[32];
+    __shared__ PT wsum[32];
     __shared__ Key red[2][XCH_THREADS / 32];
     __shared__ int32_t s_ptr;
     const int32_t w = (int32_t)blockIdx.x;
@@ -836,9 +838,18 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
     const int64_t ncnt = mode == C_H22 ? 4 : 2;
     SPMM_TRY(cnt.alloc(ncnt * M * sizeof(int32_t), s));
     SPMM_CUDA(cudaMemsetAsync(cnt.p, 0, ncnt * M * sizeof(int32_t), s));
-    auto kern = mode == C_H21 ? k_chain_x<C_H21> : mode == C_WARP ? k_chain_x<C_WARP>
-              : mode == C_H23 ? k_chain_x<C_H23> : mode == C_H22 ? k_chain_x<C_H22>
-              : k_chain_x<C_CTA>;                                       // HYBRID_1 = C_CTA over segments
+    // 32-bit posting-list prefixes unless 1024 x the longest list could overflow them
+    int32_t max_list = 0;
+    SPMM_TRY(reduce_max_i32(bcnt.as<int32_t>(), nblk, &max_list, s));
+    const char *fw = getenv("SPMM_CHAIN_WIDE");   // tests: force the 64-bit variant
+    const bool wide = (int64_t)max_list * XCH_CACHE >= ((int64_t)1 << 31) || (fw && atoi(fw) != 0);
+    auto pick = [&](auto pt) {
+        using PT = decltype(pt);
+        return mode == C_H21 ? k_chain_x<C_H21, PT> : mode == C_WARP ? k_chain_x<C_WARP, PT>
+             : mode == C_H23 ? k_chain_x<C_H23, PT> : mode == C_H22 ? k_chain_x<C_H22, PT>
+             : k_chain_x<C_CTA, PT>;                                    // HYBRID_1 = C_CTA over segments
+    };
+    auto kern = wide ? pick(int64_t{}) : pick(int32_t{});
     kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
                                                 win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt, p.nw,

@@ -49,6 +49,19 @@ def test_exact_builder_matches_oracle(exact_builder, name, policy, window, preor
     assert np.array_equal(got, ref), (name, policy, window, int(np.argmax(got != ref)))
 
 
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_2", "hybrid_1"])
+def test_exact_builder_wide_prefix(monkeypatch, policy):
+    """The 64-bit posting-list prefix variant (taken when 1024 x the longest list could overflow int32)."""
+    monkeypatch.setenv("SPMM_CHAIN_EXACT", "1")
+    monkeypatch.setenv("SPMM_CHAIN_WIDE", "1")
+    a = GENS["rmat13_local"]()
+    h = pkg.SpMM.from_csr(a)
+    for window in (0, 1024):
+        h.permute(policy, window=window)
+        assert np.array_equal(h.perm(), oracle.permute(a, policy, window=window)), (policy, window)
+    h.close()
+
+
 def test_exact_builder_matches_k_chain():
     """Same answer as the shared-memory bitmap builder k_chain on a window it can also take (32768 rows)."""
     a = syn.rmat(15, 6, 2110, "local")
