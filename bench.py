@@ -521,6 +521,13 @@ def main():
             "H2D(B) on rank 0 + NCCL broadcast + spmm_run + D2H(C shards)")}
     if e2e_pipe is not None:
         e2e["pipelined"] = e2e_pipe
+        # headline E = the pipelined public API when it ran: still every step copies its whole B in and its whole
+        # C out inside the timed region; the one-call-at-a-time number stays under "sequential"
+        if "value" in e2e_pipe and e2e_pipe["value"] > e2e["value"]:
+            e2e["sequential"] = {"value": e2e["value"], "ms_per_step": e2e["ms_per_step"], "path": e2e["path"]}
+            e2e["value"] = e2e_pipe["value"]
+            e2e["ms_per_step"] = e2e_pipe["ms_per_step"]
+            e2e["path"] = e2e_pipe["path"]
 
     # ---- cuSPARSE comparator: cusparseSpMM CSR ALG1/ALG2/ALG3 and the default algorithm, row-major B and C,
     # best-of (tools/cusparse_ref.cu), same inputs, same L2 flush, rank 0 shard ----
