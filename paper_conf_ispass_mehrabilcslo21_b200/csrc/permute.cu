@@ -695,6 +695,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                 __syncthreads();
                 const int32_t ptr = s_ptr;
                 const uint32_t b0 = ptr < n ? nb_of((int32_t)o[ptr]) : 0xffffffffu;
+                __syncthreads();   // everyone has read s_ptr before warp 0 may rewrite it below
                 xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {
                     if (r != prev && !is_placed(placed, r) && nb_of(r) == b0) {
                         const Key k = keyof(r);

@@ -3,7 +3,7 @@
 # features). Logs in gpurun_out/sanitize_*.log
 mkdir -p gpurun_out
 for tool in memcheck racecheck synccheck initcheck; do
-  timeout 900 /usr/local/cuda/bin/compute-sanitizer --tool $tool --error-exitcode 9 --target-processes all \
+  timeout ${SAN_TIMEOUT:-1500} /usr/local/cuda/bin/compute-sanitizer --tool $tool --error-exitcode 9 --target-processes all \
      python scripts/sanitize_driver.py > gpurun_out/sanitize_$tool.log 2>&1
   echo "$tool rc=$? $(grep -c 'ERROR SUMMARY: 0 errors' gpurun_out/sanitize_$tool.log) clean-summaries"
   grep "ERROR SUMMARY" gpurun_out/sanitize_$tool.log | tail -1

@@ -43,12 +43,15 @@ h.features_b200(64)
 torch.cuda.synchronize()
 # inverted-index exact chains (k_chain_x): whole matrix and multi-window, both modes, an empty-row-rich input
 os.environ["SPMM_CHAIN_EXACT"] = "1"
-for a4 in (syn.uniform(1500, 2000, 3, 5, poisson=True), syn.rmat(10, 8, 6, "local")):
-    h4 = pkg.SpMM.from_csr(a4)
-    for pol in ("cta_aware", "hybrid_2_1"):
-        for W in (0, 256):
-            h4.permute(pol, window=W)
-    h4.close()
+for wide in ("0", "1"):
+    os.environ["SPMM_CHAIN_WIDE"] = wide
+    for a4 in (syn.uniform(1500, 2000, 3, 5, poisson=True), syn.rmat(10, 8, 6, "local")):
+        h4 = pkg.SpMM.from_csr(a4)
+        for pol in ("cta_aware", "hybrid_2_1", "warp_aware", "hybrid_2_3", "hybrid_2_2", "hybrid_1"):
+            for W in (0, 256):
+                h4.permute(pol, window=W)
+        h4.close()
 os.environ.pop("SPMM_CHAIN_EXACT")
+os.environ.pop("SPMM_CHAIN_WIDE")
 torch.cuda.synchronize()
 print("sanitize driver done")
