@@ -238,6 +238,20 @@ def run_reference(args):
     }))
 
 
+def p2p_send(dist, t, dst):
+    """NCCL: send the device tensor.  gloo (one-GPU dry runs of the N>1 path only): via host memory."""
+    dist.send(t if dist.get_backend() == "nccl" else t.cpu(), dst=dst)
+
+
+def p2p_recv(torch, dist, t, src):
+    if dist.get_backend() == "nccl":
+        dist.recv(t, src=src)
+    else:
+        h = torch.empty(t.shape, dtype=t.dtype)
+        dist.recv(h, src=src)
+        t.copy_(h)
+
+
 def shard_inputs(torch, dist, a_full, world, rank, dev, pkg, compact=False):
     """Rank 0 holds the generated matrix; every rank gets its nnz-balanced row shard as CUDA tensors
     (NCCL send/recv for N>1).  Returns (M_r, lo, (rowidx, colidx, value), meta, cols) with rowidx rebased to 0.
@@ -265,7 +279,7 @@ def shard_inputs(torch, dist, a_full, world, rank, dev, pkg, compact=False):
                          + ((torch.from_numpy(cols_all[r]),) if compact else ()))
         for r in range(1, world):
             for t in parts[r]:
-                dist.send(t.to(dev), dst=r)
+                p2p_send(dist, t.to(dev), r)
         mine = tuple(t.to(dev) for t in parts[0])
     else:
         Mr, nnzr, nc = int(meta[rank, 0]), int(meta[rank, 1]), int(meta[rank, 3])
@@ -274,7 +288,7 @@ def shard_inputs(torch, dist, a_full, world, rank, dev, pkg, compact=False):
         if compact:
             mine = mine + (torch.empty(nc, dtype=torch.int64, device=dev),)
         for t in mine:
-            dist.recv(t, src=0)
+            p2p_recv(torch, dist, t, 0)
     cols = mine[3] if compact else None
     return int(meta[rank, 0]), int(meta[rank, 2]), mine[:3], meta, cols, (cols_all if rank == 0 else None)
 
@@ -354,12 +368,12 @@ def main():
         if rank == 0:
             Bfull = B_host.to(dev)
             for r in range(1, world):
-                dist.send(Bfull.index_select(0, torch.from_numpy(cols_all[r]).to(dev)).contiguous(), dst=r)
+                p2p_send(dist, Bfull.index_select(0, torch.from_numpy(cols_all[r]).to(dev)).contiguous(), r)
             Bd = Bfull.index_select(0, cols_d).contiguous()
             del Bfull
         else:
             Bd = torch.empty((N_loc, K), dtype=torch.float32, device=dev)
-            dist.recv(Bd, src=0)
+            p2p_recv(torch, dist, Bd, 0)
     else:
         Bd = B_host.to(dev) if rank == 0 else torch.empty((N, K), dtype=torch.float32, device=dev)
         if world > 1:
