@@ -148,6 +148,18 @@ spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, 
  * one handle must be ordered (same stream or external synchronisation). */
 spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream);
 
+/* spmm_run with the C all-gather fused into the epilogue (SURVEY §8(f) f2 ii): every row this handle computes
+ * (its shard, M rows) is stored to each of n_dsts (1..8) destinations at row row_offset + r, r = the handle's
+ * original row index -- C_dsts: HOST array of DEVICE pointers to [>= row_offset + M][K] float32 row-major
+ * buffers, typically this GPU's full-C buffer and its peers' (peer-mapped / symmetric-memory addresses on an
+ * NVLink/NVSwitch node: the SpMM's own stores carry the exchange, no separate collective).  When every rank
+ * calls it with all ranks' buffers and its shard's row offset, each buffer ends up holding the full C once all
+ * ranks are done (the caller orders that, e.g. a barrier).  Other rows are untouched.  Ordering and scratch
+ * as spmm_run.  Errors: INVALID_ARG (NULL, n_dsts out of range, negative row_offset), UNSUPPORTED (K, or a
+ * destination row not 16-byte aligned), STATE, CUDA. */
+spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
+                        int64_t row_offset, void *cuda_stream);
+
 /* End-to-end variant: B_host -> device, spmm_run, C -> C_host, all on cuda_stream with handle-owned
  * staging buffers (grown on demand).  Host buffers should be pinned for full copy bandwidth.
  * Synchronises cuda_stream before returning. */

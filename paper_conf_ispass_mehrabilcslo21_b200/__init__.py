@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_to", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -83,6 +83,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_features": (st, [vp, ctypes.c_int, vp, vp, vp]),
         "spmm_features_b200": (st, [vp, ctypes.c_int, i64, vp, vp]),
         "spmm_run": (st, [vp, vp, i64, vp, vp]),
+        "spmm_run_to": (st, [vp, vp, i64, vp, i32, i64, vp]),
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host_batch": (st, [vp, i64, vp, i64, vp, vp]),
         "spmm_predict": (st, [vp, vp, i64, i32, vp, vp]),
@@ -239,6 +240,17 @@ class SpMM:
             C = torch.empty((self.M, K), dtype=torch.float32, device=B.device)
         _check(load_library().spmm_run(self._h, B.data_ptr(), K, C.data_ptr(), _stream_ptr(stream)))
         return C
+
+    def run_to(self, B, dsts, row_offset=0, stream=None):
+        """spmm_run_to: this handle's C rows stored to every destination buffer (cuda float32 [>= row_offset + M, K]
+        tensors, or raw device / peer-mapped pointers as ints) at rows row_offset + r -- the C all-gather fused
+        into the SpMM epilogue."""
+        K = int(B.shape[1])
+        ptrs = [d if isinstance(d, int) else d.data_ptr() for d in dsts]
+        arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
+        _check(load_library().spmm_run_to(self._h, B.data_ptr(), K, arr, len(ptrs), int(row_offset),
+                                          _stream_ptr(stream)))
+        return dsts
 
     def run_host(self, B_host, C_host, stream=None):
         """End-to-end: host B -> device, SpMM, device -> host C (host buffers, ideally pinned)."""

@@ -313,6 +313,28 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
     return launch_spmm(h, B, K, C, (cudaStream_t)cuda_stream, &g_last_launches);
 }
 
+spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
+                        int64_t row_offset, void *cuda_stream) {
+    g_last_launches = 0;
+    if (!h || !C_dsts) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    if (n_dsts < 1 || n_dsts > SPMM_MAX_CDST) return fail(SPMM_ERR_INVALID_ARG, "n_dsts must be in [1, 8]");
+    if (row_offset < 0) return fail(SPMM_ERR_INVALID_ARG, "negative row_offset");
+    for (int32_t i = 0; i < n_dsts; ++i) {
+        SPMM_TRY(check_run_args(h, B, K, C_dsts[i], true));
+        if (((uintptr_t)(C_dsts[i] + row_offset * K)) & 15u)
+            return fail(SPMM_ERR_UNSUPPORTED, "destination rows must be 16-byte aligned");
+    }
+    SPMM_TRY(check_device(h));
+    CExtra cx{};
+    cx.n = n_dsts - 1;
+    for (int32_t i = 1; i < n_dsts; ++i) cx.p[i - 1] = reinterpret_cast<float4 *>(C_dsts[i] + row_offset * K);
+    h->cx = cx;
+    const spmm_status st = launch_spmm(h, B, K, C_dsts[0] + row_offset * K, (cudaStream_t)cuda_stream,
+                                       &g_last_launches);
+    h->cx = CExtra{};
+    return st;
+}
+
 spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *C_host, void *cuda_stream) {
     g_last_launches = 0;
     SPMM_TRY(check_run_args(h, B_host, K, C_host, false));

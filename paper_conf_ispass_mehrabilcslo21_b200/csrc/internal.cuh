@@ -93,6 +93,15 @@ struct Schedule {
 
 }  // namespace spmm
 
+// Extra C destinations of one spmm_run_to (f2 ii): every C row the run writes is also stored to p[0..n-1]
+// (device or peer-mapped pointers, already offset to this shard's first row) -- the all-gather of C fused into
+// the SpMM epilogue.  n = 0 for plain runs.
+constexpr int SPMM_MAX_CDST = 8;
+struct CExtra {
+    float4 *p[SPMM_MAX_CDST - 1];
+    int32_t n;
+};
+
 struct spmm_ctx {
     int device = 0;
     cudaStream_t create_stream = nullptr;
@@ -122,6 +131,7 @@ struct spmm_ctx {
     int num_sms = 148;
     // optional kernel timing (spmm_set_kernel_timing): events around the main SpMM kernel of spmm_run
     int timing = 0;
+    CExtra cx{};              // extra C destinations of the current spmm_run_to (n = 0 otherwise)
     bool timed = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     // side stream for the empty-row zero fill (SPMM_ZERO_SIDE=1)

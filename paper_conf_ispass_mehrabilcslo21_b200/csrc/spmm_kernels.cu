@@ -133,11 +133,11 @@ __device__ __forceinline__ int2 ld_cv(const int2 *ptr, uint64_t pol) {
 // count is warp-uniform (groups past their own length are predicated off), so the shuffles stay warp-wide.
 // Store: a whole row -> C[perm[p]] (streaming store); a chunk group of a long row -> the warp's groups
 // are reduced by a fixed xor butterfly and group 0 writes the partial.
-template <int V, int G, int U, int LD, class VT>
+template <int V, int G, int U, int LD, class VT, bool MD = false>
 __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int gl, const int col0, const bool (&colok)[V],
                                           const int2 *__restrict__ cv, const VT *__restrict__ BV,
                                           VT *__restrict__ CV, const int32_t KV, VT *__restrict__ PV,
-                                          const uint64_t pol_b, const uint64_t pol_a) {
+                                          const uint64_t pol_b, const uint64_t pol_a, const CExtra &cx) {
     constexpr int BATCH = (G >= 8 ? G : 8) >= U ? (G >= 8 ? G : 8) : U;   // (col, val) pairs per group per batch
     constexpr int PL = BATCH / G;                // pairs held per lane
     const int32_t start = u.x, len = u.y, dst = u.z;
@@ -200,10 +200,20 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
 #pragma unroll
         for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
     }
-    if (dst >= 0) {                                    // a whole row: C[perm[p]]
+    if (dst >= 0) {                                    // a whole row: C[perm[p]] (+ the extra destinations)
 #pragma unroll
         for (int v = 0; v < V; ++v)
             if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[v]);
+        if constexpr (MD) {   // spmm_run_to instantiations only (VAR bit 10): no cost for plain runs
+#pragma unroll
+            for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in parameter space
+                if (i >= cx.n) break;
+                VT *X = reinterpret_cast<VT *>(cx.p[i]);
+#pragma unroll
+                for (int v = 0; v < V; ++v)
+                    if (colok[v]) vstore_cs(X + (size_t)dst * KV + col0 + v * G, acc[v]);
+            }
+        }
     } else if (dst != NOSTORE) {                       // chunk group of a long row (warp-uniform)
 #pragma unroll
         for (int off = G; off < 32; off <<= 1) {       // fixed butterfly: ((c0+c1)+(c2+c3))...
@@ -238,11 +248,11 @@ __device__ __forceinline__ int rec_word(const RecT<4> &r, int i) {
 __device__ __forceinline__ RecT<2> rec_zero(RecT<2>) { return RecT<2>{make_int4(0, 0, 0, 0)}; }
 __device__ __forceinline__ RecT<4> rec_zero(RecT<4>) { return RecT<4>{make_int4(0, 0, 0, 0), make_int4(0, 0, 0, 0)}; }
 
-template <int V, int G, int R, int U, class VT>
+template <int V, int G, int R, int U, class VT, bool MD = false>
 __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const int gl, const int col0,
                                                 const bool (&colok)[V], const RecT<R> *__restrict__ recs,
                                                 const int32_t *__restrict__ gdst, const VT *__restrict__ BV,
-                                                VT *__restrict__ CV, const int32_t KV) {
+                                                VT *__restrict__ CV, const int32_t KV, const CExtra &cx) {
     constexpr int BATCH = G >= 8 ? G : 8;        // records per group per batch
     constexpr int PL = BATCH / G;                // records held per lane
     const int32_t start = u.x, len = u.y, gid = u.z;
@@ -312,6 +322,16 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
 #pragma unroll
                 for (int v = 0; v < V; ++v)
                     if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[r][v]);
+                if constexpr (MD) {   // spmm_run_to instantiations only (VAR bit 10): no cost for plain runs
+#pragma unroll
+                    for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in param space
+                        if (i >= cx.n) break;
+                        VT *X = reinterpret_cast<VT *>(cx.p[i]);
+#pragma unroll
+                        for (int v = 0; v < V; ++v)
+                            if (colok[v]) vstore_cs(X + (size_t)dst * KV + col0 + v * G, acc[r][v]);
+                    }
+                }
             }
         }
     }
@@ -376,7 +396,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter,
                                                        const int4 *__restrict__ recs,
-                                                       const int32_t *__restrict__ gdst) {
+                                                       const int32_t *__restrict__ gdst, const CExtra cx) {
     using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
     constexpr int CTV = V * G;
@@ -450,13 +470,14 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
         bool fused = false;
         if (FR > 1) fused = __shfl_sync(0xffffffffu, u.w, 0) == 1;
         if (FR > 1 && fused) {
-            spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU>(u, g, gl, col0, colok,
+            spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU, VT, (VAR & 1024) != 0>(u, g, gl, col0, colok,
                                                      reinterpret_cast<const RecT<(FR > 1 ? FR : 2)> *>(recs), gdst,
-                                                     reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV);
+                                                     reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV,
+                                                     cx);
         } else {
-            spmm_unit<V, G, U, LD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
+            spmm_unit<V, G, U, LD, VT, (VAR & 1024) != 0>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
                                                      reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), pol_b,
-                                                     pol_a);
+                                                     pol_a, cx);
         }
         t = t_next;
         u = u_next;
@@ -536,7 +557,7 @@ __global__ void __launch_bounds__(AFF_THREADS, 1) k_spmm_aff(const int4 *__restr
         const bool ok_next = aff_claim(&state, counter, n_tasks, ppt, T, n_items, lane, t_next, tile_next);
         const int4 u_next = ok_next ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
         spmm_unit<V, G, U, LD>(u, g, gl, tile * CTV + gl, colok, cv, reinterpret_cast<const VT *>(B4),
-                               reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), 0, 0);
+                               reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), 0, 0, CExtra{});
         ok = ok_next;
         t = t_next;
         tile = tile_next;
@@ -549,7 +570,7 @@ __global__ void __launch_bounds__(AFF_THREADS, 1) k_spmm_aff(const int4 *__restr
 // column of C.
 __global__ void __launch_bounds__(256) k_combine(const float4 *__restrict__ P4, const int32_t *__restrict__ pslot_ptr,
                                                  const int32_t *__restrict__ long_dst, int64_t n_long,
-                                                 float4 *__restrict__ C4, int32_t K4) {
+                                                 float4 *__restrict__ C4, int32_t K4, const CExtra cx) {
     const int lane = threadIdx.x & 31;
     for (int64_t l = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; l < n_long;
          l += ((int64_t)gridDim.x * blockDim.x) >> 5) {
@@ -572,15 +593,24 @@ __global__ void __launch_bounds__(256) k_combine(const float4 *__restrict__ P4, 
                 r = make_float4(y.x + r.x, y.y + r.y, y.z + r.z, y.w + r.w);
             }
             __stcs(dst + col, r);
+#pragma unroll
+            for (int i = 0; i < SPMM_MAX_CDST - 1; ++i)
+                if (i < cx.n) __stcs(cx.p[i] + (size_t)long_dst[l] * K4 + col, r);
         }
     }
 }
 
 // empty rows: zero-fill their C rows (thread per float4)
-__global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, float4 *__restrict__ C4) {
+__global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, float4 *__restrict__ C4,
+                            const CExtra cx) {
     const int64_t total = n * K4;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
-        __stcs(C4 + (size_t)rows[i / K4] * K4 + (i % K4), make_float4(0.f, 0.f, 0.f, 0.f));
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const size_t o = (size_t)rows[i / K4] * K4 + (i % K4);
+        __stcs(C4 + o, make_float4(0.f, 0.f, 0.f, 0.f));
+#pragma unroll
+        for (int j = 0; j < SPMM_MAX_CDST - 1; ++j)
+            if (j < cx.n) __stcs(cx.p[j] + o, make_float4(0.f, 0.f, 0.f, 0.f));
+    }
 }
 
 // ---- a7 schedule construction ------------------------------------------------------------------
@@ -926,7 +956,7 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s) 
 }
 
 using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
-                            unsigned int *, const int4 *, const int32_t *);
+                            unsigned int *, const int4 *, const int32_t *, const CExtra);
 
 template <int V, bool MASK, int SCHED, int VAR>
 SpmmKernel pick_g(int G) {
@@ -1115,7 +1145,7 @@ static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, 
         P4 = h->partials.as<float4>();
     }
     if (S.n_empty > 0) {
-        k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4);
+        k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4, h->cx);
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
@@ -1140,7 +1170,7 @@ static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, 
     }
     if (S.n_long > 0) {
         k_combine<<<(unsigned)std::min<int64_t>(ceil_div(S.n_long, 8), 148 * 64), 256, 0, s>>>(
-            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4);
+            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, h->cx);
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
@@ -1156,10 +1186,22 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     static const int sched = env_int("SPMM_SCHED", 0);
     static const int var = env_int("SPMM_VARIANT", 0);
     static const int wmax = env_int("SPMM_W", 8);
-    const bool w8ok = wmax >= 8 && K % 8 == 0 && ((uintptr_t)B % 32) == 0 && ((uintptr_t)C % 32) == 0;
-    const Config cfg = choose(K4, sched, var, w8ok);
+    uintptr_t align = (uintptr_t)B | (uintptr_t)C;
+    for (int i = 0; i < h->cx.n; ++i) align |= (uintptr_t)h->cx.p[i];
+    const bool w8ok = wmax >= 8 && K % 8 == 0 && (align % 32) == 0;
+    Config cfg = choose(K4, sched, var, w8ok);
+    bool copy_extra = false;      // spmm_run_to on a geometry without a multi-destination kernel: copy afterwards
+    if (h->cx.n > 0) {
+        SpmmKernel kmd = cfg.W == 8 ? pick_w8<1024>(cfg.V, cfg.G) : nullptr;
+        if (kmd && cfg.tiles == 1) {
+            cfg.kern = kmd;
+            if (cfg.kern_fused) cfg.kern_fused = pick_w8_fused_v<8 | 1024>(cfg.V, cfg.G, cfg.R);
+        } else {
+            copy_extra = true;
+        }
+    }
     static const int kmode = env_int("SPMM_KERNEL", 1);
-    if (kmode == 3) {
+    if (kmode == 3 && h->cx.n == 0) {   // (the experimental SM-affine mode has no extra C destinations)
         static const int av = env_int("SPMM_AFF_V", 1);
         const int aw = w8ok ? 8 : 4;
         if (K % (32 * av) == 0 && pick_aff(av, env_int("SPMM_AFF_LD", 2), aw))
@@ -1193,12 +1235,13 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
             }
             SPMM_CUDA(cudaEventRecord(h->ev_fork, s));
             SPMM_CUDA(cudaStreamWaitEvent(h->side, h->ev_fork, 0));
-            k_zero_rows<<<(unsigned)h->num_sms, 128, 0, h->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4);
+            k_zero_rows<<<(unsigned)h->num_sms, 128, 0, h->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4,
+                                                                   h->cx);
             SPMM_CUDA(cudaGetLastError());
             SPMM_CUDA(cudaEventRecord(h->ev_join, h->side));
             joined = false;
         } else {
-            k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4);
+            k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4, h->cx);
             SPMM_CUDA(cudaGetLastError());
         }
         ++*launches;
@@ -1216,7 +1259,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
                                            reinterpret_cast<const float4 *>(B), C4, K4, P4,
-                                           h->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>());
+                                           h->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>(),
+                                           h->cx);
         SPMM_CUDA(cudaGetLastError());
         if (h->timing) {
             SPMM_CUDA(cudaEventRecord(h->ev1, s));
@@ -1226,11 +1270,14 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     }
     if (S.n_long > 0) {
         k_combine<<<(unsigned)std::min<int64_t>(ceil_div(S.n_long, 8), 148 * 64), 256, 0, s>>>(
-            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4);
+            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, h->cx);
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
     if (!joined) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_join, 0));
+    if (copy_extra)
+        for (int i = 0; i < h->cx.n; ++i)
+            SPMM_CUDA(cudaMemcpyAsync(h->cx.p[i], C, (size_t)M * K * sizeof(float), cudaMemcpyDeviceToDevice, s));
     return SPMM_OK;
 }
 

@@ -128,6 +128,15 @@ class ShardedSpMM:
         """Local SpMM on this rank's row shard (B resident on every rank). Returns the C shard."""
         return self.local.run(B, C_local)
 
+    def run_allgather_fused(self, B, C_bufs, stream=None):
+        """the C all-gather fused into the SpMM epilogue.  This rank's SpMM stores its C rows
+        straight into every rank's full-C buffer (C_bufs[p]: cuda tensors [M, K] or device pointers addressable
+        from this GPU -- on an NVLink/NVSwitch node the peer views of a torch symmetric-memory allocation), at its
+        shard's row offset (spmm_run_to); no separate collective.  Every rank calls it; each buffer holds the
+        full C once all ranks' kernels are done (the caller's barrier)."""
+        self.local.run_to(B, C_bufs, row_offset=int(self.bounds[self.rank]), stream=stream)
+        return C_bufs
+
     def allgather_C(self, C_local):
         """Reassemble the full C (original row order) on every rank."""
         import torch

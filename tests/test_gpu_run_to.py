@@ -1,0 +1,97 @@
+"""spmm_run_to (SURVEY §8(f) f2 ii): the C all-gather fused into the SpMM epilogue -- every C row a handle computes is
+stored to n destination buffers at a row offset.  On one GPU the destinations are local buffers standing in for
+the peers' (the kernel's stores do not depend on where the pointers map).  Checks: every destination equals the
+plain spmm_run result bit for bit (whole rows, row-fusion records, long-row combine and empty-row zero fill all
+write every destination); two nnz-balanced shards writing into shared full-size buffers at their row offsets
+reassemble the unsharded C bit for bit and match the oracle; rows outside the shard are untouched; argument
+errors."""
+import numpy as np
+import pytest
+
+import oracle
+import synthetic as syn
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
+from paper_conf_ispass_mehrabilcslo21_b200.sharded import make_shard  # noqa: E402
+
+
+def _with_long_and_empty_rows(a):
+    rows = [a.colidx[a.rowidx[i]:a.rowidx[i + 1]].tolist() for i in range(a.M)]
+    rows[3] = list(range(0, a.N, 2))          # a long row (split into chunk groups + k_combine)
+    rows[5] = []                              # empty rows (k_zero_rows)
+    rows[6] = []
+    return syn.from_lists(a.M, a.N, rows)
+
+
+CASES = {
+    "rmat_long_empty_k128": (lambda: _with_long_and_empty_rows(syn.rmat(12, 10, 3100, "local")), 128, "cta_aware"),
+    "stencil_fused_k64": (lambda: syn.stencil27(18, 3101), 64, "identity"),      # row fusion R = 4
+    "uniform_k36": (lambda: syn.uniform(3000, 4000, 7, 3102, poisson=True), 36, "nnz_sort"),   # W = 4 path
+}
+
+
+@pytest.mark.parametrize("name", list(CASES))
+@pytest.mark.parametrize("n_dsts", [1, 3, 8])
+def test_run_to_every_destination(name, n_dsts):
+    gen, K, pol = CASES[name]
+    a = gen()
+    h = pkg.SpMM.from_csr(a)
+    h.permute(pol)
+    B = torch.from_numpy(syn.dense(a.N, K, 3103)).cuda()
+    ref = h.run(B).clone()
+    dsts = [torch.full((a.M, K), float("nan"), device="cuda") for _ in range(n_dsts)]
+    h.run_to(B, dsts)
+    torch.cuda.synchronize()
+    for d in dsts:
+        assert torch.equal(d.view(torch.int32), ref.view(torch.int32))
+    h.close()
+
+
+def test_run_to_shards_reassemble():
+    a = _with_long_and_empty_rows(syn.rmat(13, 8, 3104, "natural"))
+    K = 64
+    Bn = syn.dense(a.N, K, 3105)
+    B = torch.from_numpy(Bn).cuda()
+    whole = pkg.SpMM.from_csr(a)
+    whole.permute("hybrid_2_1")
+    ref = whole.run(B).clone()
+    whole.close()
+    bounds = pkg.spmm_partition_by_nnz(a.rowidx, 2)
+    bufs = [torch.full((a.M, K), float("nan"), device="cuda") for _ in range(2)]
+    for r in range(2):
+        sh = make_shard(a.M, a.N, a.rowidx, a.colidx, a.value, bounds, r)
+        hs = pkg.SpMM(sh.M, sh.N, sh.rowidx, sh.colidx, sh.value)
+        hs.permute("cta_aware")
+        hs.run_to(B, bufs, row_offset=int(bounds[r]))
+        torch.cuda.synchronize()
+        if r == 0:   # rows of the other shard untouched so far
+            assert torch.isnan(bufs[0][int(bounds[1]):]).all()
+        hs.close()
+    for d in bufs:
+        assert torch.equal(d.view(torch.int32), ref.view(torch.int32))
+    C_ref, bound = oracle.spmm(a, Bn)
+    err = np.abs(bufs[0].cpu().numpy().astype(np.float64) - C_ref)
+    assert np.all(err <= 1e-5 * bound + 1e-6)
+
+
+def test_run_to_errors():
+    a = syn.rmat(10, 6, 3106, "natural")
+    h = pkg.SpMM.from_csr(a)
+    B = torch.zeros((a.N, 32), device="cuda")
+    C = torch.zeros((a.M + 8, 32), device="cuda")
+    lib = pkg.load_library()
+    import ctypes
+    for n in (0, 9):
+        arr = (ctypes.c_void_p * max(n, 1))(*([C.data_ptr()] * max(n, 1)))
+        assert lib.spmm_run_to(h._h, B.data_ptr(), 32, arr, n, 0, None) == 1
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.run_to(B, [C.data_ptr() + 4])                 # destination rows not 16-byte aligned
+    assert ex.value.status == 3
+    with pytest.raises(pkg.SpmmError) as ex:
+        h.run_to(B, [C], row_offset=-1)
+    assert ex.value.status == 1
+    h.run_to(B, [C], row_offset=8)                      # in bounds: rows 8 .. 8 + M
+    h.close()
