@@ -32,6 +32,13 @@ class OracleLocal:
         out, _ = oracle.spmm(self.csr, B.numpy())
         return torch.from_numpy(out.astype(np.float32))
 
+    def run_to(self, B, dsts, row_offset=0, stream=None):
+        """spmm_run_to semantics: this shard's rows stored into every destination at row_offset + r."""
+        out = self.run(B)
+        for d in dsts:
+            d[row_offset:row_offset + out.shape[0]] = out
+        return dsts
+
 
 def _free_port():
     s = socket.socket()
@@ -63,6 +70,14 @@ def _worker(rank, world, port, K, results, compact=False):
             C_local = sh.run(B)
         C = sh.allgather_C(C_local)
         ref, _ = oracle.spmm(a, syn.dense(a.N, K, 5, int_values=True))
+        if not compact:
+            # fused all-gather (f2 ii): each rank stores its rows into "every rank's" full-C buffer at its row
+            # offset; here the peers' buffers are local stand-ins, so the disjoint writes are summed over ranks
+            bufs = [torch.zeros((a.M, K)) for _ in range(world)]
+            sh.run_allgather_fused(B, bufs)
+            for b in bufs:
+                dist.all_reduce(b)
+                assert np.array_equal(b.numpy().astype(np.float64), ref)
         nnz_local = sh.shard.nnz
         results[rank] = (bool(np.array_equal(C.numpy().astype(np.float64), ref)), nnz_local, a.nnz,
                          int(np.diff(a.rowidx).max()), sh.shard.lo, sh.shard.hi)
