@@ -589,8 +589,9 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     int32_t *out = perm + s0;
     auto nb_of = [&](int32_t r) -> uint32_t { return (uint32_t)(sig_ptr[r + 1] - sig_ptr[r]); };
     auto wl_of = [&](int32_t r) -> uint32_t { return (uint32_t)((nnz[r] + nt - 1) / nt); };
-    const int32_t mw = multiwin ? w : -1;    // lists sorted by window: visit only this window's rows
-    auto mine = [&](int32_t r) -> bool { return true; };
+    // multi-window: lists are sorted by window and only this window's sub-range is visited, so every row a
+    // pass sees belongs to this window (and only this CTA touches its counters)
+    const int32_t mw = multiwin ? w : -1;
     if (n <= 0) return;
     // first row(s): least (wl, r) of the window's unplaced rows -- 1 row (CTA_AWARE, HYBRID_2_1), nw rows
     // (WARP_AWARE, HYBRID_2_3: "the first 32 rows are those ... with the lowest warp load"), as k_chain
@@ -629,14 +630,13 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         // step's prefix lives in the other buffer
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw);
         // reset the previous step's counters (other buffer), then count |b_r ∩ b_ref|
-        // (only this window's rows: the other windows' CTAs count theirs in the same arrays)
         if (pref >= 0) {
-            auto reset = [&](int32_t r) { if (mine(r)) co[r] = 0; };
+            auto reset = [&](int32_t r) { co[r] = 0; };
             if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], brow, reset);
             else xvisit_all(pref, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, reset);
         }
         auto count = [&](int32_t r) {
-            if (r != prev && mine(r) && !is_placed(placed, r)) atomicAdd(cc + r, 1);
+            if (r != prev && !is_placed(placed, r)) atomicAdd(cc + r, 1);
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
@@ -670,7 +670,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         };
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
         auto score = [&](int32_t r) {
-            if (r != prev && mine(r) && !is_placed(placed, r)) {
+            if (r != prev && !is_placed(placed, r)) {
                 const Key k = keyof(r);
                 if (key_less(k, best)) best = k;
             }
