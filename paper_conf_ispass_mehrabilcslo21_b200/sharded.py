@@ -128,6 +128,17 @@ class ShardedSpMM:
         """Local SpMM on this rank's row shard (B resident on every rank). Returns the C shard."""
         return self.local.run(B, C_local)
 
+    def symmetric_C(self, K, dtype=None):
+        """A full-C buffer [M, K] in torch symmetric memory on this rank, plus every rank's view of it as device
+        pointers (the destinations for run_allgather_fused; peer addresses are NVLink-mapped on an NVSwitch
+        node).  Needs an NCCL process group."""
+        import torch
+        import torch.distributed._symmetric_memory as symm_mem
+        buf = symm_mem.empty((self.M, int(K)), dtype=dtype or torch.float32, device=torch.device("cuda"))
+        grp = self.group if self.group is not None else self.dist.group.WORLD
+        hdl = symm_mem.rendezvous(buf, grp.group_name)
+        return buf, [int(p) for p in hdl.buffer_ptrs], hdl
+
     def run_allgather_fused(self, B, C_bufs, stream=None):
         """the C all-gather fused into the SpMM epilogue.  This rank's SpMM stores its C rows
         straight into every rank's full-C buffer (C_bufs[p]: cuda tensors [M, K] or device pointers addressable

@@ -95,3 +95,40 @@ def test_run_to_errors():
     assert ex.value.status == 1
     h.run_to(B, [C], row_offset=8)                      # in bounds: rows 8 .. 8 + M
     h.close()
+
+
+def test_run_allgather_fused_symmetric_memory():
+    """ShardedSpMM.run_allgather_fused into a torch symmetric-memory full-C buffer (world 1 NCCL group on one GPU:
+    the destination is the symmetric allocation's own device pointer, the same address kind a peer would use)."""
+    import os
+    import socket
+    import torch.distributed as dist
+    from paper_conf_ispass_mehrabilcslo21_b200.sharded import ShardedSpMM
+
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        a = syn.rmat(12, 8, 3110, "local")
+        K = 64
+        Bn = syn.dense(a.N, K, 3111)
+        B = torch.from_numpy(Bn).cuda()
+        sh = ShardedSpMM(a.M, a.N, a.rowidx, a.colidx, a.value)
+        sh.permute("cta_aware")
+        buf, ptrs, _hdl = sh.symmetric_C(K)
+        assert len(ptrs) == 1
+        buf.fill_(float("nan"))
+        sh.run_allgather_fused(B, ptrs)
+        torch.cuda.synchronize()
+        ref = sh.run(B)
+        assert torch.equal(buf.view(torch.int32), ref.view(torch.int32))
+        C_ref, bound = oracle.spmm(a, Bn)
+        err = np.abs(buf.cpu().numpy().astype(np.float64) - C_ref)
+        assert np.all(err <= 1e-5 * bound + 1e-6)
+        sh.close()
+    finally:
+        dist.destroy_process_group()
