@@ -134,3 +134,25 @@ def test_bench_shard_inputs_gloo(compact):
     mp.spawn(_bench_worker, args=(2, _free_port(), compact, results), nprocs=2, join=True)
     assert all(results[r][0] for r in range(2)), dict(results)
     assert results[0][1] + results[1][1] == results[0][2]
+
+
+def test_bench_reference_arm_torchrun():
+    """bench.py --impl reference under torchrun N=2 (CPU): rank 0 alone times the oracle and prints ONE JSON
+    line with impl/cpu_baseline/e2e; the other rank exits 0 without work."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
+           os.path.join(root, "bench.py"), "--impl", "reference", "--config", "c1",
+           "--gpus", "2", "--steps", "2", "--warmup", "3"]
+    out = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["steps"] == 2 and d["warmup"] == 3
+    assert d["value"] > 0 and d["unit"] == "GFLOP/s" and d["higher_is_better"] is True
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] == d["value"]
+    assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
