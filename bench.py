@@ -42,6 +42,10 @@ CONFIGS = {
     "c3sh": dict(desc="configs[2] with its rows randomly relabelled (seeded shuffle; columns unchanged): the original "
                       "order has no locality, the column-similarity orders must recover the communities",
                  gen=("rmat", 22, 28, 3000, "local"), shuffle=3002, K=128),
+    "c5rl": dict(desc="configs[4] stress variant: power-law R-MAT S=24 random-label, M=N=16M, nnz~500M, K=128",
+                 gen=("rmat", 24, 38, 5001, "random-label"), K=128),
+    "c5sh": dict(desc="configs[4] with its rows randomly relabelled (seeded shuffle; columns unchanged)",
+                 gen=("rmat", 24, 38, 5000, "local"), shuffle=5002, K=128),
 }
 HOT = ["identity", "nnz_sort", "plain_sort", "cta_aware", "hybrid_1", "hybrid_2_1", "cta_aware+mh", "cta_aware+md"]
 # "+mh" / "+md": the chain policy with its windows over the MinHash / median-block pre-order (spmm_params.preorder

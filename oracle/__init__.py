@@ -72,9 +72,12 @@ def _c(a, dt):
     return np.ascontiguousarray(a, dtype=dt)
 
 
-def validate_csr(M, N, rowidx, colidx) -> int:
+def validate_csr(M, N, rowidx, colidx, nnz=None) -> int:
+    """0 if valid (nnz defaults to rowidx[M], i.e. only the other checks apply)."""
     r, c = _c(rowidx, np.int64), _c(colidx, np.int32)
-    return int(_load().oracle_validate_csr(M, N, int(r[-1]) if M >= 0 else 0, r.ctypes.data, c.ctypes.data))
+    if nnz is None:
+        nnz = int(r[-1]) if M >= 0 else 0
+    return int(_load().oracle_validate_csr(M, N, nnz, r.ctypes.data, c.ctypes.data))
 
 
 def spmm(csr, B: np.ndarray, rows=None):

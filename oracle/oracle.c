@@ -15,7 +15,11 @@
  * Pins (tests/test_oracle_*.py, -m "not gpu"): numpy dense matmul and scipy.sparse
  * for SpMM; hand-worked examples E1/E2 (tests/golden/); paper arithmetic P:L88,
  * P:L92; stencil closed forms; brute-force local-optimality
- * checkers for every greedy step; permutation invariants.
+ * checkers for every greedy step; permutation invariants; the MinHash key by the
+ * splitmix64 generator's published outputs (tests/golden/splitmix64.json, reached
+ * through the seed XOR) and a Python-int brute force of min-over-blocks with
+ * nonzero seeds (round 2: round 1 pinned it by one seed-0, one-block vector only,
+ * so a max-for-min or a dropped seed went undetected -- both mutations now fail).
  * Parity unpinned: none of the functions below (oracle_mlp_forward is pinned
  * against a torch forward; the predictor's TRAINING is not an oracle function).
  */

@@ -29,7 +29,7 @@ K = cfg["K"]
 B = torch.from_numpy(syn.dense(a.N, K, 1)).cuda()
 C = torch.empty((a.M, K), device="cuda")
 h = pkg.SpMM.from_csr(a)
-h.permute(args.policy, window=args.window, split_nnz=args.split)
+bench.permute_spec(h, args.policy, args.window)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 for _ in range(args.runs):
     flush.fill_(1.0)

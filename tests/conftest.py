@@ -34,3 +34,8 @@ def e2():
 @pytest.fixture(scope="session")
 def paper_arith():
     return load_golden("paper_arith.json")
+
+
+@pytest.fixture(scope="session")
+def golden():
+    return lambda name: load_golden(name + ".json")

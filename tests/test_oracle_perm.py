@@ -188,6 +188,74 @@ def test_minhash_splitmix_vector():
     assert int(h[1]) == 2 ** 64 - 1
 
 
+MASK64 = (1 << 64) - 1
+
+
+def _splitmix64_py(z):
+    """Python-int splitmix64 (z + golden gamma, then the two xor-shift-multiplies and a final xor-shift), pinned
+    below by the generator's published outputs -- independent of oracle.c's uint64 arithmetic."""
+    z = (z + 0x9E3779B97F4A7C15) & MASK64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & MASK64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & MASK64
+    return z ^ (z >> 31)
+
+
+def test_splitmix_python_matches_published_vectors(golden):
+    g = golden("splitmix64")
+    gamma = int(g["golden_gamma"], 16)
+    for k, v in enumerate(g["outputs_seed0"]):
+        assert _splitmix64_py((k * gamma) & MASK64) == int(v, 16)
+
+
+def test_minhash_published_vectors_through_seed(golden):
+    """One-block rows whose block id b XOR seed is (k-1)*gamma get the generator's k-th published output: pins the
+    seed XOR (a dropped seed gives finaliser(b) instead) and the hash itself against tests/golden/splitmix64.json."""
+    g = golden("splitmix64")
+    gamma = int(g["golden_gamma"], 16)
+    a = syn.from_lists(1, 256, [[3 * 32 + 5]])          # block 3 (bw = 32)
+    for k, v in enumerate(g["outputs_seed0"]):
+        seed = 3 ^ ((k * gamma) & MASK64)
+        assert int(oracle.minhash_keys(a, bw=32, seed=seed)[0]) == int(v, 16), k
+
+
+@pytest.mark.parametrize("seed", [0, 7, 0xDEADBEEF12345, 2 ** 64 - 3])
+def test_minhash_min_over_blocks_bruteforce(seed):
+    """h_i = min over b in blocks_i of splitmix64(b XOR seed), recomputed with Python ints over
+    multi-block rows (R-MAT rows touch up to hundreds of blocks): a max instead of the min, a dropped seed, a wrong
+    block width or a per-column (not per-block) hash all fail here."""
+    a = syn.rmat(10, 9, 48, "natural")
+    h = oracle.minhash_keys(a, bw=32, seed=seed)
+    nblk = 0
+    for i in range(a.M):
+        blocks = sorted(set((a.colidx[a.rowidx[i]:a.rowidx[i + 1]] // 32).tolist()))
+        nblk = max(nblk, len(blocks))
+        ref = min((_splitmix64_py(b ^ seed) for b in blocks), default=MASK64)
+        assert int(h[i]) == ref, (i, blocks)
+    assert nblk >= 3
+
+
+def test_minhash_invariants():
+    """Hash-value-free properties: a row's key is the min of the keys of its one-block sub-rows; the key of block b
+    under seed s is the seed-0 key of block b XOR s."""
+    rows = [[0, 33, 70, 100, 200], [5, 64 + 1], [230], []]
+    a = syn.from_lists(4, 256, rows)
+    for s in (0, 5, 6):
+        h = oracle.minhash_keys(a, bw=32, seed=s)
+        for i, r in enumerate(rows):
+            singles = syn.from_lists(len(r), 256, [[c] for c in r]) if r else None
+            hs = oracle.minhash_keys(singles, bw=32, seed=s) if r else np.array([MASK64], dtype=np.uint64)
+            assert int(h[i]) == int(hs.min())
+        for b in range(8):
+            one = syn.from_lists(1, 256, [[32 * b]])
+            x = syn.from_lists(1, 256, [[32 * (b ^ s)]])
+            assert int(oracle.minhash_keys(one, bw=32, seed=s)[0]) == int(oracle.minhash_keys(x, bw=32, seed=0)[0])
+    # a two-block row where the larger hash is not the min: max-instead-of-min changes the key
+    two = syn.from_lists(1, 256, [[0, 32]])
+    k0 = int(oracle.minhash_keys(syn.from_lists(1, 256, [[0]]), bw=32, seed=0)[0])
+    k1 = int(oracle.minhash_keys(syn.from_lists(1, 256, [[32]]), bw=32, seed=0)[0])
+    assert k0 != k1 and int(oracle.minhash_keys(two, bw=32, seed=0)[0]) == min(k0, k1)
+
+
 def test_planted_clusters_contiguous():
     """Planted block-clustered matrix (identical masks within a group, disjoint across groups):
     CTA-aware with W=0 keeps every group contiguous, so the chain crosses groups exactly G-1 times."""

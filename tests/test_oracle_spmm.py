@@ -100,3 +100,9 @@ def test_validate_csr():
     assert oracle.validate_csr(3, 4, ok.rowidx, np.array([0, 2, 3, 1], np.int32)) != 0   # unsorted row
     assert oracle.validate_csr(3, 4, ok.rowidx, np.array([0, 2, 1, 4], np.int32)) != 0   # out of range
     assert oracle.validate_csr(3, 4, np.array([0, 2, 1, 4]), ok.colidx) != 0             # non-monotone
+    assert oracle.validate_csr(3, 4, ok.rowidx, ok.colidx, nnz=4) == 0
+    assert oracle.validate_csr(3, 4, np.array([1, 2, 2, 4]), ok.colidx, nnz=4) != 0      # rowidx[0] != 0
+    assert oracle.validate_csr(3, 4, np.array([0, 2, 2, 3]), ok.colidx, nnz=4) != 0      # rowidx[M] != nnz
+    assert oracle.validate_csr(3, 4, ok.rowidx, ok.colidx, nnz=5) != 0                   # rowidx[M] != nnz
+    assert oracle.validate_csr(3, 4, ok.rowidx, np.array([0, 2, -1, 3], np.int32)) != 0  # negative column
+    assert oracle.validate_csr(3, 4, ok.rowidx, np.array([0, 0, 1, 3], np.int32)) != 0   # duplicate column
