@@ -192,8 +192,9 @@ def oracle_sample_rows(a, target_nnz, seed=7):
 def cpu_baseline(a, B, K, budget_s=15.0):
     """The oracle (oracle.c, float64, OpenMP) as it stands, on a bounded row sample, on this host's cores."""
     import oracle
-    cores = len(os.sched_getaffinity(0))
-    os.environ.setdefault("OMP_NUM_THREADS", str(cores))
+    # every core of this process's affinity set, replacing any inherited OMP_NUM_THREADS (torchrun sets 1);
+    # `cores` is the thread count OpenMP reports in effect
+    cores = oracle.set_threads(len(os.sched_getaffinity(0)))
     rows, snnz = oracle_sample_rows(a, 200_000)
     t0 = time.perf_counter()
     oracle.spmm(a, B, rows=rows)
@@ -220,7 +221,7 @@ def run_reference(args):
     K = cfg["K"]
     B = syn.dense(a.N, K, cfg["gen"][-2] + 1 if cfg["gen"][0] == "rmat" else cfg["gen"][2] + 1)
     import oracle
-    cores = len(os.sched_getaffinity(0))
+    cores = oracle.set_threads(len(os.sched_getaffinity(0)))   # overrides torchrun's OMP_NUM_THREADS=1
     rows, snnz = oracle_sample_rows(a, args.ref_sample_nnz)
     for _ in range(args.warmup):
         oracle.spmm(a, B, rows=rows[: max(1, len(rows) // 10)])

@@ -62,6 +62,8 @@ def _load():
         lib.oracle_mlp_forward_n.argtypes = [vp, i32, vp, i32, vp]
         lib.oracle_median_block_keys.restype = None
         lib.oracle_median_block_keys.argtypes = [i64, vp, vp, i32, vp]
+        lib.oracle_threads.restype = ctypes.c_int
+        lib.oracle_threads.argtypes = [ctypes.c_int]
         lib.oracle_mlp_forward.restype = i32
         lib.oracle_mlp_forward.argtypes = [vp, vp, i32, vp]
         _lib = lib
@@ -70,6 +72,12 @@ def _load():
 
 def _c(a, dt):
     return np.ascontiguousarray(a, dtype=dt)
+
+
+def set_threads(n: int = 0) -> int:
+    """OpenMP threads of the oracle's parallel loops: n > 0 sets them (overriding an inherited OMP_NUM_THREADS,
+    e.g. torchrun's 1); returns the count actually in effect."""
+    return int(_load().oracle_threads(int(n)))
 
 
 def validate_csr(M, N, rowidx, colidx, nnz=None) -> int:

@@ -27,12 +27,20 @@
 #include <stdlib.h>
 #include <string.h>
 #include <math.h>
+#include <omp.h>
 
 /* policy ids: same numbering as the C-ABI enum (an integer protocol, not shared code) */
 enum {
     P_IDENTITY = 0, P_NNZ_SORT = 1, P_PLAIN_SORT = 2, P_CTA_AWARE = 3, P_HYBRID_1 = 4, P_HYBRID_2_1 = 5,
     P_FLIPPED = 6, P_LPT = 7, P_WARP_AWARE = 8, P_HYBRID_2_2 = 9, P_HYBRID_2_3 = 10, P_DCSR = 11
 };
+
+/* Thread count of the OpenMP loops (infrastructure, no method arithmetic): n > 0 sets it (replacing whatever
+ * OMP_NUM_THREADS the process inherited, e.g. torchrun's 1); returns the count the next parallel loop uses. */
+int oracle_threads(int n) {
+    if (n > 0) omp_set_num_threads(n);
+    return omp_get_max_threads();
+}
 
 /* ------------------------------------------------------------------------------------
  * CSR validity (§II.A): rowidx[0]=0, rowidx[M]=nnz, non-decreasing; 0<=col<N;

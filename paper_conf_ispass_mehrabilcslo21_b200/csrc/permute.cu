@@ -622,7 +622,9 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     for (int32_t q = nfirst; q < n; ++q) {
         const int buf = q & 1;
         int32_t *cc = buf ? cnt1 : cnt0, *co = buf ? cnt0 : cnt1;
-        const int32_t ref = WARPREF ? out[q - nw] : prev;       // the row Hamming distances are taken to
+        // the row Hamming distances are taken to; out[q - 1] is written by thread 0 after the previous step's
+        // last barrier, so nw == 1 reads it from the register copy prev (as k_chain does)
+        const int32_t ref = WARPREF ? (nw == 1 ? prev : out[q - nw]) : prev;
         const int32_t bs = sig_ptr[ref], be = sig_ptr[ref + 1];
         const uint32_t cp = (uint32_t)(be - bs);
         const bool cached = be - bs <= XCH_CACHE;
@@ -647,7 +649,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
             int32_t *co2 = buf ? cnt2a : cnt2b;
             if (pref2 >= 0)
                 xvisit_all(pref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) { co2[r] = 0; });
-            ref2 = q >= nw ? out[q - nw] : -1;
+            ref2 = q >= nw ? (nw == 1 ? prev : out[q - nw]) : -1;
             if (ref2 >= 0) {
                 cp2 = nb_of(ref2);
                 xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {

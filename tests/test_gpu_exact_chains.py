@@ -62,6 +62,21 @@ def test_exact_builder_wide_prefix(monkeypatch, policy):
     h.close()
 
 
+@pytest.mark.parametrize("policy", ["warp_aware", "hybrid_2_3", "hybrid_2_2"])
+@pytest.mark.parametrize("nw", [1, 2])
+def test_exact_builder_small_nw(exact_builder, policy, nw):
+    """nw = 1: the reference row out[q - nw] is the previous position, written by thread 0 after the previous
+    step's last barrier -- the builder must take it from its register copy (a read of out[q - 1] raced
+    that write).  Bit-exact against the oracle at nw = 1 and 2, whole matrix and windows."""
+    a = GENS["rmat12_natural"]()
+    h = pkg.SpMM.from_csr(a)
+    for window in (0, 512):
+        h.permute(policy, window=window, nw=nw)
+        ref = oracle.permute(a, policy, nw=nw, window=window)
+        assert np.array_equal(h.perm(), ref), (policy, nw, window)
+    h.close()
+
+
 def test_exact_builder_matches_k_chain():
     """Same answer as the shared-memory bitmap builder k_chain on a window it can also take (32768 rows)."""
     a = syn.rmat(15, 6, 2110, "local")

@@ -156,3 +156,5 @@ def test_bench_reference_arm_torchrun():
     assert d["value"] > 0 and d["unit"] == "GFLOP/s" and d["higher_is_better"] is True
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] == d["value"]
     assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+    # torchrun exports OMP_NUM_THREADS=1; the oracle must still run on every core of the affinity set
+    assert d["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
