@@ -101,13 +101,23 @@ spmm_status spmm_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, con
                         const int32_t *colidx, const float *value, int inputs_on_device, void *cuda_stream);
 
 /* Build permutation `policy` (params NULL = defaults), the permuted CSR it implies and its row-class
- * counts, all on the device (offline / amortised).  Replaces the previous permutation.  The
- * K-dependent run schedule (a7: empty / whole / split rows packed into warp tasks) is built by the next
- * spmm_run (once per permutation and lanes-per-row geometry; that call synchronises its stream).
- * Needs external synchronisation against spmm_run on the same handle. */
+ * counts, all on the device (offline / amortised), then replace the current permutation with it.
+ * Atomic: everything is built into new buffers first; on any failure (e.g. SPMM_ERR_OOM) the handle keeps
+ * its previous permutation, permuted CSR and schedules and stays usable.  Synchronises cuda_stream, and waits
+ * for this handle's runs still in flight (they read the arrays being replaced).  Drops the cached run
+ * schedules (rebuild: spmm_prepare).  Must not be called concurrently with other calls on the same handle. */
 spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *params, void *cuda_stream);
 
-/* Copy the current permutation (M int32, HOST buffer).  Synchronises. */
+/* Build the K-dependent run schedule of the current permutation (a7: empty / whole / split rows packed into
+ * warp tasks for the lane geometry of K, row-fusion unions where they pay) so that spmm_run with this K is
+ * fully asynchronous.  B / C (device, may be NULL) only select the lane geometry: 32-byte aligned (or NULL)
+ * -> 256-bit lane loads, else 128-bit; pass the buffers the runs will use.  Up to 4 geometries are cached per
+ * permutation.  A run whose geometry was not prepared builds it itself (and then synchronises its stream).
+ * Synchronises cuda_stream.  Errors: INVALID_ARG (NULL h, K <= 0), UNSUPPORTED (K), STATE, OOM, CUDA. */
+spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *C, void *cuda_stream);
+
+/* Copy the current permutation (M int32, HOST buffer).  Reads it back on the handle's own non-blocking
+ * stream (the permutation is complete when spmm_permute returns); no device-wide synchronisation. */
 spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out);
 
 /* Copy the current permuted CSR to HOST buffers: rowidx int64[M+1], colidx int32[nnz], value f32[nnz]. */
@@ -118,7 +128,7 @@ spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colid
  * rows, out[4]=max row nnz. */
 spmm_status spmm_get_info(spmm_handle h, int64_t out[5]);
 
-/* Run schedule (a7) built by the most recent spmm_run on h: out[0] = rows per warp task (lane groups; 0 = no
+/* Run schedule (a7) used by the most recent spmm_run on h: out[0] = rows per warp task (lane groups; 0 = no
  * schedule yet), out[1] = row-fusion factor R in use (1 = none), out[2] = warp tasks, out[3] = fusion groups,
  * out[4] = union records of those groups, out[5] = nnz of the fused rows (out[4] / out[5] = B-row loads per
  * nnz on the fused rows).  Errors: INVALID_ARG (NULL). */
@@ -144,8 +154,11 @@ spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, 
 
 /* C = A . B on the device (beta = 0: C is fully overwritten; empty rows get zeros).
  * B: device, float32 row-major [N][K]; C: device, float32 row-major [M][K] in ORIGINAL row order.
- * Asynchronous on cuda_stream; reads the handle only, but shares its long-row scratch, so calls on
- * one handle must be ordered (same stream or external synchronisation). */
+ * Asynchronous on cuda_stream once the schedule of K's geometry exists (spmm_prepare, or an earlier run
+ * with this K): no host synchronisation, and runs on one handle may be issued concurrently from several
+ * streams / host threads -- each run takes one of 4 handle-owned scratch slots (task counter, split-row
+ * partials, zero-fill side stream) round-robin and waits, on its own stream, for that slot's previous run.
+ * (The kernel-timing aid, spmm_set_kernel_timing, is the exception: its events belong to the handle.) */
 spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream);
 
 /* spmm_run with the C all-gather fused into the epilogue (SURVEY §8(f) f2 ii): every row this handle computes
@@ -154,8 +167,8 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
  * buffers, typically this GPU's full-C buffer and its peers' (peer-mapped / symmetric-memory addresses on an
  * NVLink/NVSwitch node: the SpMM's own stores carry the exchange, no separate collective).  When every rank
  * calls it with all ranks' buffers and its shard's row offset, each buffer ends up holding the full C once all
- * ranks are done (the caller orders that, e.g. a barrier).  Other rows are untouched.  Ordering and scratch
- * as spmm_run.  Errors: INVALID_ARG (NULL, n_dsts out of range, negative row_offset), UNSUPPORTED (K, or a
+ * ranks are done (the caller orders that, e.g. a barrier).  Other rows are untouched.  Asynchrony and
+ * concurrency as spmm_run.  Errors: INVALID_ARG (NULL, n_dsts out of range, negative row_offset), UNSUPPORTED (K, or a
  * destination row not 16-byte aligned), STATE, CUDA. */
 spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
                         int64_t row_offset, void *cuda_stream);
@@ -194,7 +207,8 @@ spmm_status spmm_predict_n(const double *features, int32_t n_features, const flo
  * bounds[p] = min{ r : rowidx[r] >= ceil(p*nnz/P) }.  rowidx: HOST int64[M+1]; bounds: HOST int64[P+1]. */
 spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, int64_t *bounds);
 
-/* Release the handle and all its device memory (stream-ordered on the creation stream). */
+/* Release the handle and all its device memory (stream-ordered frees).  Waits for the handle's own runs and
+ * copies (their slot events and streams) -- not for other work on the device. */
 spmm_status spmm_destroy(spmm_handle h);
 
 const char *spmm_status_string(spmm_status s);

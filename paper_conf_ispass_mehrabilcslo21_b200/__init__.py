@@ -55,7 +55,7 @@ _lib = None
 _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
-EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_get_perm",
+EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_prepare", "spmm_get_perm",
            "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_to", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
@@ -76,6 +76,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_set_allocator": (st, [_ALLOC_T, _FREE_T, vp]),
         "spmm_create": (st, [vp, i64, i64, i64, vp, vp, vp, ctypes.c_int, vp]),
         "spmm_permute": (st, [vp, ctypes.c_int, vp, vp]),
+        "spmm_prepare": (st, [vp, i64, vp, vp, vp]),
         "spmm_get_perm": (st, [vp, vp]),
         "spmm_get_permuted_csr": (st, [vp, vp, vp, vp]),
         "spmm_get_info": (st, [vp, vp]),
@@ -159,6 +160,37 @@ def _ptr(a):
     return a.data_ptr(), bool(a.is_cuda), a
 
 
+def _need(cond, msg):
+    if not cond:
+        raise ValueError(msg)
+
+
+def _check_dense(t, name, rows, K=None, device=True, min_rows=None):
+    """The C ABI takes raw pointers and cannot check buffer sizes or layouts: this is the one place they are
+    checked (a transposed / non-contiguous / too small tensor would otherwise give a wrong C or write out of
+    bounds).  rows: exact row count, or min_rows: at least that many."""
+    import torch
+    _need(isinstance(t, torch.Tensor), f"{name} must be a torch tensor")
+    _need(t.is_cuda == device, f"{name} must be a {'CUDA' if device else 'host (CPU)'} tensor")
+    _need(t.dtype == torch.float32, f"{name} must be float32, got {t.dtype}")
+    _need(t.dim() == 2 and t.is_contiguous(), f"{name} must be a contiguous (row-major) 2-D tensor")
+    if rows is not None:
+        _need(t.shape[0] == rows, f"{name} must have {rows} rows, got {t.shape[0]}")
+    if min_rows is not None:
+        _need(t.shape[0] >= min_rows, f"{name} must have at least {min_rows} rows, got {t.shape[0]}")
+    if K is not None:
+        _need(t.shape[1] == K, f"{name} must have {K} columns, got {t.shape[1]}")
+
+
+def _check_host(a, name, rows, K):
+    """Host buffers of the end-to-end calls: numpy arrays or CPU tensors, float32, C-contiguous [rows, K]."""
+    if isinstance(a, np.ndarray):
+        _need(a.dtype == np.float32 and a.ndim == 2 and a.flags.c_contiguous, f"{name} must be C-contiguous float32 2-D")
+        _need(a.shape == (rows, K), f"{name} must be [{rows}, {K}], got {list(a.shape)}")
+    else:
+        _check_dense(a, name, rows, K, device=False)
+
+
 _live = weakref.WeakSet()
 
 
@@ -172,6 +204,16 @@ class SpMM:
             rowidx = np.ascontiguousarray(rowidx, dtype=np.int64)
             colidx = np.ascontiguousarray(colidx, dtype=np.int32)
             value = np.ascontiguousarray(value, dtype=np.float32)
+        else:   # torch tensors: the library reads raw int64 / int32 / float32 arrays of these lengths
+            import torch
+            _need(rowidx.dtype == torch.int64 and colidx.dtype == torch.int32 and value.dtype == torch.float32,
+                  "rowidx / colidx / value must be int64 / int32 / float32")
+            _need(all(t.is_contiguous() and t.dim() == 1 for t in (rowidx, colidx, value)),
+                  "rowidx / colidx / value must be contiguous 1-D tensors")
+            _need(rowidx.is_cuda == colidx.is_cuda == value.is_cuda, "CSR arrays must all be on the same side")
+        _need(len(rowidx) == int(M) + 1, f"rowidx must have M + 1 = {int(M) + 1} entries")
+        _need(len(colidx) >= (int(rowidx[-1]) if M > 0 else 0) and len(value) == len(colidx),
+              "colidx / value must hold rowidx[M] entries")
         r, on_dev, _k1 = _ptr(rowidx)
         c, _, _k2 = _ptr(colidx)
         v, _, _k3 = _ptr(value)
@@ -191,6 +233,13 @@ class SpMM:
         p = make_params(**params)
         _check(load_library().spmm_permute(self._h, pid, ctypes.byref(p), _stream_ptr(stream)))
         self.policy = POLICY_NAMES[pid]
+        return self
+
+    def prepare(self, K, B=None, C=None, stream=None):
+        """spmm_prepare: build the run schedule of K's lane geometry now, so spmm_run with this K is asynchronous
+        (B / C: the buffers the runs will use -- only their alignment matters; None = aligned)."""
+        _check(load_library().spmm_prepare(self._h, int(K), None if B is None else B.data_ptr(),
+                                           None if C is None else C.data_ptr(), _stream_ptr(stream)))
         return self
 
     def perm(self) -> np.ndarray:
@@ -235,9 +284,12 @@ class SpMM:
     def run(self, B, C=None, stream=None):
         """C = A.B on the device (B: cuda float32 [N, K] row-major). Returns C (cuda float32 [M, K])."""
         import torch
+        _check_dense(B, "B", self.N)
         K = int(B.shape[1])
         if C is None:
             C = torch.empty((self.M, K), dtype=torch.float32, device=B.device)
+        _check_dense(C, "C", self.M, K)
+        _need(C.device == B.device, "B and C must be on the same device")
         _check(load_library().spmm_run(self._h, B.data_ptr(), K, C.data_ptr(), _stream_ptr(stream)))
         return C
 
@@ -245,7 +297,11 @@ class SpMM:
         """spmm_run_to: this handle's C rows stored to every destination buffer (cuda float32 [>= row_offset + M, K]
         tensors, or raw device / peer-mapped pointers as ints) at rows row_offset + r -- the C all-gather fused
         into the SpMM epilogue."""
+        _check_dense(B, "B", self.N)
         K = int(B.shape[1])
+        for d in dsts:
+            if not isinstance(d, int):   # raw (peer) pointers are the caller's responsibility
+                _check_dense(d, "destination", None, K, min_rows=int(row_offset) + self.M)
         ptrs = [d if isinstance(d, int) else d.data_ptr() for d in dsts]
         arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
         _check(load_library().spmm_run_to(self._h, B.data_ptr(), K, arr, len(ptrs), int(row_offset),
@@ -255,6 +311,8 @@ class SpMM:
     def run_host(self, B_host, C_host, stream=None):
         """End-to-end: host B -> device, SpMM, device -> host C (host buffers, ideally pinned)."""
         K = int(B_host.shape[1])
+        _check_host(B_host, "B_host", self.N, K)
+        _check_host(C_host, "C_host", self.M, K)
         b, _, _ = _ptr(B_host)
         c, _, _ = _ptr(C_host)
         _check(load_library().spmm_run_host(self._h, b, K, c, _stream_ptr(stream)))
@@ -268,6 +326,9 @@ class SpMM:
         if n == 0:
             return Cs
         K = int(Bs[0].shape[1])
+        for b, c in zip(Bs, Cs):
+            _check_host(b, "B_host", self.N, K)
+            _check_host(c, "C_host", self.M, K)
         bp = (ctypes.c_void_p * n)(*[_ptr(b)[0] for b in Bs])
         cp = (ctypes.c_void_p * n)(*[_ptr(c)[0] for c in Cs])
         _check(load_library().spmm_run_host_batch(self._h, n, bp, K, cp, _stream_ptr(stream)))

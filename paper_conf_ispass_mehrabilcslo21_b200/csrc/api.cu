@@ -117,6 +117,7 @@ spmm_status do_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, const
     SPMM_CUDA(cudaGetDevice(&h->device));
     SPMM_CUDA(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
     h->create_stream = s;
+    SPMM_CUDA(cudaStreamCreateWithFlags(&h->aux, cudaStreamNonBlocking));
     h->M = M; h->N = N; h->nnz = nnz;
     spmm_default_params(&h->params);
     const cudaMemcpyKind kind = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
@@ -158,8 +159,8 @@ spmm_status do_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, const
     flags.release();
     // current policy: IDENTITY
     h->policy = SPMM_POLICY_IDENTITY;
-    SPMM_TRY(build_permutation(h, SPMM_POLICY_IDENTITY, h->params, s));
-    SPMM_TRY(build_permuted_csr(h, s));
+    SPMM_TRY(build_permutation(h, SPMM_POLICY_IDENTITY, h->params, h->perm, s));
+    SPMM_TRY(build_permuted_csr(h, h->params.split_nnz, h->perm, h->rowptr_p, h->cv_p, h->rc, s));
     SPMM_CUDA(cudaStreamSynchronize(s));
     *out = guard.release();
     return SPMM_OK;
@@ -212,11 +213,24 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
     SPMM_TRY(check_params(p));
     cudaStream_t s = (cudaStream_t)cuda_stream;
     try {
-        h->params = p;
-        SPMM_TRY(build_permutation(h, policy, p, s));
-        SPMM_TRY(build_permuted_csr(h, s));
-        h->policy = policy;
+        // build into temporaries; the handle keeps its current permutation, permuted CSR and schedules unless
+        // every step succeeds (a failed permute -- e.g. SPMM_ERR_OOM -- leaves a usable handle)
+        DevBuf perm, rowptr_p, cv_p;
+        RowClasses rc;
+        SPMM_TRY(build_permutation(h, policy, p, perm, s));
+        SPMM_TRY(build_permuted_csr(h, p.split_nnz, perm, rowptr_p, cv_p, rc, s));
         SPMM_CUDA(cudaStreamSynchronize(s));
+        std::lock_guard<std::mutex> lk(h->mu);
+        for (int i = 0; i < RUN_SLOTS; ++i)        // runs still in flight read the old arrays
+            if (h->slots[i].used) SPMM_CUDA(cudaEventSynchronize(h->slots[i].done));
+        h->perm.swap(perm);
+        h->rowptr_p.swap(rowptr_p);
+        h->cv_p.swap(cv_p);
+        h->rc = rc;
+        h->params = p;
+        h->policy = policy;
+        for (int i = 0; i < SCHED_CACHE; ++i) h->sched[i].built = 0;
+        h->last_sched.store(-1);
     } catch (const std::exception &e) {
         return fail(SPMM_ERR_OOM, e.what());
     }
@@ -227,21 +241,24 @@ spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out) {
     if (!h || (!perm_out && h->M > 0)) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     SPMM_TRY(check_device(h));
     if (h->M == 0) return SPMM_OK;
-    SPMM_CUDA(cudaDeviceSynchronize());
-    SPMM_CUDA(cudaMemcpy(perm_out, h->perm.p, h->M * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    // the permutation is complete (spmm_create / spmm_permute synchronise their stream); read it back on the
+    // handle's own non-blocking stream -- no device-wide synchronisation
+    SPMM_CUDA(cudaMemcpyAsync(perm_out, h->perm.p, h->M * sizeof(int32_t), cudaMemcpyDeviceToHost, h->aux));
+    SPMM_CUDA(cudaStreamSynchronize(h->aux));
     return SPMM_OK;
 }
 
 spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colidx, float *value) {
     if (!h || !rowidx || (h->nnz > 0 && (!colidx || !value))) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     SPMM_TRY(check_device(h));
-    SPMM_CUDA(cudaDeviceSynchronize());
     std::vector<int32_t> r32(h->M + 1);
-    SPMM_CUDA(cudaMemcpy(r32.data(), h->rowptr_p.p, (h->M + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    SPMM_CUDA(cudaMemcpyAsync(r32.data(), h->rowptr_p.p, (h->M + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, h->aux));
+    SPMM_CUDA(cudaStreamSynchronize(h->aux));
     for (int64_t i = 0; i <= h->M; ++i) rowidx[i] = r32[i];
     if (h->nnz > 0) {
         std::vector<int2> cv(h->nnz);
-        SPMM_CUDA(cudaMemcpy(cv.data(), h->cv_p.p, h->nnz * sizeof(int2), cudaMemcpyDeviceToHost));
+        SPMM_CUDA(cudaMemcpyAsync(cv.data(), h->cv_p.p, h->nnz * sizeof(int2), cudaMemcpyDeviceToHost, h->aux));
+        SPMM_CUDA(cudaStreamSynchronize(h->aux));
         for (int64_t j = 0; j < h->nnz; ++j) {
             colidx[j] = cv[j].x;
             std::memcpy(&value[j], &cv[j].y, sizeof(float));
@@ -262,13 +279,15 @@ spmm_status spmm_get_info(spmm_handle h, int64_t out[5]) {
 
 spmm_status spmm_get_schedule_info(spmm_handle h, int64_t out[6]) {
     if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
-    const Schedule &S = h->sched;
-    out[0] = S.rpw;
-    out[1] = S.rpw ? S.fuse : 1;
-    out[2] = S.rpw ? S.n_tasks : 0;
-    out[3] = S.rpw ? S.n_groups : 0;
-    out[4] = S.rpw ? S.n_records : 0;
-    out[5] = S.rpw ? S.fused_nnz : 0;
+    const int i = h->last_sched.load();
+    const bool ok = i >= 0 && h->sched[i].built;
+    const Schedule &S = h->sched[ok ? i : 0];
+    out[0] = ok ? S.rpw : 0;
+    out[1] = ok ? S.fuse : 1;
+    out[2] = ok ? S.n_tasks : 0;
+    out[3] = ok ? S.n_groups : 0;
+    out[4] = ok ? S.n_records : 0;
+    out[5] = ok ? S.fused_nnz : 0;
     return SPMM_OK;
 }
 
@@ -310,7 +329,26 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
     g_last_launches = 0;
     SPMM_TRY(check_run_args(h, B, K, C, true));
     SPMM_TRY(check_device(h));
-    return launch_spmm(h, B, K, C, (cudaStream_t)cuda_stream, &g_last_launches);
+    try {
+        return launch_spmm(h, B, K, C, (cudaStream_t)cuda_stream, &g_last_launches, CExtra{});
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
+}
+
+spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *C, void *cuda_stream) {
+    if (!h) return fail(SPMM_ERR_INVALID_ARG, "handle is NULL");
+    if (K <= 0) return fail(SPMM_ERR_INVALID_ARG, "K must be positive");
+    if (K % 4 != 0 || K > 1024) return fail(SPMM_ERR_UNSUPPORTED, "K must be a multiple of 4 and <= 1024");
+    SPMM_TRY(check_device(h));
+    if (h->M == 0) return SPMM_OK;
+    // B / C only decide the lane geometry (32-byte alignment); NULL = the aligned (256-bit load) geometry
+    static const float kAligned[8] __attribute__((aligned(32))) = {0};
+    try {
+        return prepare_schedule(h, K, B ? B : kAligned, C ? C : kAligned, (cudaStream_t)cuda_stream);
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
 }
 
 spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
@@ -328,11 +366,11 @@ spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *
     CExtra cx{};
     cx.n = n_dsts - 1;
     for (int32_t i = 1; i < n_dsts; ++i) cx.p[i - 1] = reinterpret_cast<float4 *>(C_dsts[i] + row_offset * K);
-    h->cx = cx;
-    const spmm_status st = launch_spmm(h, B, K, C_dsts[0] + row_offset * K, (cudaStream_t)cuda_stream,
-                                       &g_last_launches);
-    h->cx = CExtra{};
-    return st;
+    try {
+        return launch_spmm(h, B, K, C_dsts[0] + row_offset * K, (cudaStream_t)cuda_stream, &g_last_launches, cx);
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
 }
 
 spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *C_host, void *cuda_stream) {
@@ -344,7 +382,7 @@ spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *
     if (h->stage_B.bytes < bB) SPMM_TRY(h->stage_B.alloc(bB, s));
     if (h->stage_C.bytes < bC) SPMM_TRY(h->stage_C.alloc(bC, s));
     if (bB) SPMM_CUDA(cudaMemcpyAsync(h->stage_B.p, B_host, bB, cudaMemcpyHostToDevice, s));
-    SPMM_TRY(launch_spmm(h, h->stage_B.as<float>(), K, h->stage_C.as<float>(), s, &g_last_launches));
+    SPMM_TRY(launch_spmm(h, h->stage_B.as<float>(), K, h->stage_C.as<float>(), s, &g_last_launches, CExtra{}));
     if (bC) SPMM_CUDA(cudaMemcpyAsync(C_host, h->stage_C.p, bC, cudaMemcpyDeviceToHost, s));
     SPMM_CUDA(cudaStreamSynchronize(s));
     return SPMM_OK;
@@ -390,7 +428,7 @@ spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_
         SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_in[k], 0));
         if (i >= 2) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_out[k], 0));
         int32_t l = 0;
-        SPMM_TRY(launch_spmm(h, Bs, K, Cs, s, &l));
+        SPMM_TRY(launch_spmm(h, Bs, K, Cs, s, &l, CExtra{}));
         launches += l;
         SPMM_CUDA(cudaEventRecord(h->ev_comp[k], s));
         // D2H of C_i (overlaps the H2D of B_{i+1}: PCIe is full duplex)
@@ -455,13 +493,13 @@ spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, i
 
 spmm_status spmm_destroy(spmm_handle h) {
     if (!h) return SPMM_OK;
-    cudaStreamSynchronize(h->create_stream);
-    cudaDeviceSynchronize();
+    // wait for this handle's own work only (its runs' slot events, its copy streams), not the whole device
+    release_run_slots(h);
+    if (h->cin) cudaStreamSynchronize(h->cin);
+    if (h->cout) cudaStreamSynchronize(h->cout);
+    if (h->aux) cudaStreamSynchronize(h->aux);   // (destroyed with the handle)
     if (h->ev0) cudaEventDestroy(h->ev0);
     if (h->ev1) cudaEventDestroy(h->ev1);
-    if (h->ev_fork) cudaEventDestroy(h->ev_fork);
-    if (h->ev_join) cudaEventDestroy(h->ev_join);
-    if (h->side) cudaStreamDestroy(h->side);
     if (h->ev_start) cudaEventDestroy(h->ev_start);
     for (int k = 0; k < 2; ++k) {
         if (h->ev_in[k]) cudaEventDestroy(h->ev_in[k]);

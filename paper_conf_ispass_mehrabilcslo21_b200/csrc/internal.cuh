@@ -3,7 +3,10 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stddef.h>
+#include <atomic>
+#include <mutex>
 #include <string>
+#include <utility>
 #include "../../include/spmm.h"
 
 namespace spmm {
@@ -51,6 +54,11 @@ struct DevBuf {
         p = nullptr;
         bytes = 0;
     }
+    void swap(DevBuf &o) {
+        std::swap(p, o.p);
+        std::swap(bytes, o.bytes);
+        std::swap(s, o.s);
+    }
     template <class T> T *as() const { return reinterpret_cast<T *>(p); }
 };
 
@@ -61,8 +69,8 @@ struct RowClasses {
     int64_t n_chunks = 0;     // split_nnz-chunks over those rows
 };
 
-// a7 run schedule for one lanes-per-row geometry (rows per warp RPW), built on the first spmm_run after
-// a permute with that RPW.  Warp task t owns units [t*RPW, (t+1)*RPW): either up to RPW consecutive
+// a7 run schedule for one lanes-per-row geometry (rows per warp RPW), built by spmm_prepare (or the first
+// spmm_run of that geometry) after a permute; up to SCHED_CACHE geometries are kept per permutation.  Warp task t owns units [t*RPW, (t+1)*RPW): either up to RPW consecutive
 // non-empty short rows of the permuted order, or RPW consecutive chunks of one long row (a chunk group,
 // reduced across the warp into one partial).  Units: int4 (start, len, dst, 0); dst >= 0: C row,
 // dst == INT_MIN: padding, dst < 0: chunk group -> partial slot -(dst+1).
@@ -89,7 +97,22 @@ struct Schedule {
     int64_t n_pslots = 0;
     int64_t n_empty = 0;
     DevBuf empty_dst;         // int32[n_empty]     C rows of empty rows (zero-filled)
+    uint64_t built = 0;       // build sequence number (0 = free slot): the oldest slot is rebuilt first
 };
+constexpr int SCHED_CACHE = 4;
+
+// Per-run scratch (the task counter, split-row partials and the side stream of the empty-row zero fill).  A run
+// takes the next of RUN_SLOTS slots round-robin and waits (on its own stream, no host sync) for the slot's
+// previous user to finish, so runs on one handle may be issued concurrently from several streams / threads.
+struct RunSlot {
+    DevBuf counters;          // unsigned[64]: dynamic warp-task counters, one per column tile
+    DevBuf partials;          // float[n_pslots * K]: split-row chunk-group partials
+    cudaEvent_t done = nullptr;        // recorded on the run's stream after its last launch
+    bool used = false;
+    cudaStream_t side = nullptr;       // empty-row zero fill (forked from / joined to the run's stream)
+    cudaEvent_t fork = nullptr, join = nullptr;
+};
+constexpr int RUN_SLOTS = 4;
 
 }  // namespace spmm
 
@@ -119,10 +142,13 @@ struct spmm_ctx {
     spmm::DevBuf rowptr_p; // int32[M+1]
     spmm::DevBuf cv_p;     // int2[nnz]: (colidx', bits(value'))
     spmm::RowClasses rc;
-    spmm::Schedule sched;
-    // run scratch (partials of split rows), grown on demand
-    spmm::DevBuf partials;
-    spmm::DevBuf counters;  // dynamic warp-task counters, one per column tile
+    spmm::Schedule sched[spmm::SCHED_CACHE];
+    uint64_t sched_seq = 0;                 // build counter of the schedule slots
+    std::atomic<int> last_sched{-1};        // slot of the most recent run (spmm_get_schedule_info)
+    std::mutex mu;                          // schedule builds and run-slot hand-out
+    spmm::RunSlot slots[spmm::RUN_SLOTS];
+    uint32_t next_slot = 0;
+    cudaStream_t aux = nullptr;             // non-blocking stream of host read-backs (no device-wide sync)
     // host-run staging (spmm_run_host: one slot; spmm_run_host_batch: two slots each, double-buffered)
     spmm::DevBuf stage_B, stage_C;
     cudaStream_t cin = nullptr, cout = nullptr;          // spmm_run_host_batch copy streams
@@ -130,13 +156,13 @@ struct spmm_ctx {
                 ev_out[2] = {nullptr, nullptr};
     int num_sms = 148;
     // optional kernel timing (spmm_set_kernel_timing): events around the main SpMM kernel of spmm_run
+    // (a measurement aid: the events belong to the handle, so timed runs must not overlap)
     int timing = 0;
-    CExtra cx{};              // extra C destinations of the current spmm_run_to (n = 0 otherwise)
     bool timed = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-    // side stream for the empty-row zero fill (SPMM_ZERO_SIDE=1)
-    cudaStream_t side = nullptr;
-    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    ~spmm_ctx() {
+        if (aux) cudaStreamDestroy(aux);
+    }
 };
 
 namespace spmm {
@@ -149,12 +175,19 @@ spmm_status reduce_max_i32(const int32_t *in, int64_t n, int32_t *result_host, c
 spmm_status radix_sort_pairs(uint64_t *keys, uint32_t *vals, int64_t n, int begin_bit, int end_bit,
                              cudaStream_t s);     // stable, ascending, in place (uses scratch)
 
-spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, cudaStream_t s);
-spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s);
+// permutation `policy` into perm (int32[M]); the permuted CSR of perm into rowptr_p / cv_p and its row classes
+// (the handle's current permutation is untouched: spmm_permute swaps the results in only on success)
+spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, DevBuf &perm, cudaStream_t s);
+spmm_status build_permuted_csr(spmm_ctx *h, int32_t split, const DevBuf &perm, DevBuf &rowptr_p, DevBuf &cv_p,
+                               RowClasses &rc, cudaStream_t s);
+// a7 schedule for the K geometry (built if no cached slot matches; synchronises s when it builds)
+spmm_status prepare_schedule(spmm_ctx *h, int64_t K, const float *B, const float *C, cudaStream_t s);
 spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24],
                              cudaStream_t s);
 spmm_status compute_features_b200(spmm_ctx *h, bool current_order, int64_t K, double out[7], cudaStream_t s);
-spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches);
+spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches,
+                        const CExtra &cx);
+void release_run_slots(spmm_ctx *h);   // waits for the slots' last runs, frees their scratch and streams
 
 // signatures of the rows (sorted unique col/bw), used by chains and features
 struct Signatures {

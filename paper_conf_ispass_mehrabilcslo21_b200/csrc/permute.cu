@@ -906,10 +906,10 @@ spmm_status build_signatures(const int32_t *rowidx, const int32_t *colidx, const
     return SPMM_OK;
 }
 
-spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, cudaStream_t s) {
+spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params &p, DevBuf &perm_out, cudaStream_t s) {
     const int64_t M = h->M;
-    SPMM_TRY(h->perm.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
-    int32_t *perm = h->perm.as<int32_t>();
+    SPMM_TRY(perm_out.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
+    int32_t *perm = perm_out.as<int32_t>();
     if (M == 0) return SPMM_OK;
     DevBuf nnzb;
     SPMM_TRY(nnzb.alloc(M * sizeof(int32_t), s));
@@ -1017,38 +1017,37 @@ spmm_status build_permutation(spmm_ctx *h, spmm_policy policy, const spmm_params
     }
 }
 
-spmm_status build_permuted_csr(spmm_ctx *h, cudaStream_t s) {
+spmm_status build_permuted_csr(spmm_ctx *h, int32_t split, const DevBuf &perm, DevBuf &rowptr_p, DevBuf &cv_p,
+                               RowClasses &rc, cudaStream_t s) {
     const int64_t M = h->M;
-    const int32_t split = h->params.split_nnz;
-    SPMM_TRY(h->rowptr_p.alloc((M + 1) * sizeof(int32_t), s));
-    SPMM_TRY(h->cv_p.alloc(std::max<int64_t>(h->nnz, 1) * sizeof(int2), s));
+    SPMM_TRY(rowptr_p.alloc((M + 1) * sizeof(int32_t), s));
+    SPMM_TRY(cv_p.alloc(std::max<int64_t>(h->nnz, 1) * sizeof(int2), s));
     DevBuf len;
     SPMM_TRY(len.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
     if (M > 0) {
-        k_perm_len<<<grid_for(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), h->perm.as<int32_t>(), M, len.as<int32_t>());
+        k_perm_len<<<grid_for(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), perm.as<int32_t>(), M, len.as<int32_t>());
         SPMM_CUDA(cudaGetLastError());
     }
-    SPMM_TRY(exclusive_scan_i32(len.as<int32_t>(), h->rowptr_p.as<int32_t>(), M, nullptr, s));
+    SPMM_TRY(exclusive_scan_i32(len.as<int32_t>(), rowptr_p.as<int32_t>(), M, nullptr, s));
     if (M > 0 && h->nnz > 0) {
         k_gather<<<grid_warps(M, 256), 256, 0, s>>>(h->rowidx.as<int32_t>(), h->colidx.as<int32_t>(), h->value.as<float>(),
-                                                   h->perm.as<int32_t>(), h->rowptr_p.as<int32_t>(), M, h->cv_p.as<int2>());
+                                                   perm.as<int32_t>(), rowptr_p.as<int32_t>(), M, cv_p.as<int2>());
         SPMM_CUDA(cudaGetLastError());
     }
-    // a7 row-class counts (the K-dependent run schedule is built by the first spmm_run)
-    h->sched.rpw = 0;
-    h->rc.n_long = h->rc.n_chunks = 0;
+    // a7 row-class counts (the K-dependent run schedule is built by spmm_prepare / the first spmm_run)
+    rc.n_long = rc.n_chunks = 0;
     if (M == 0 || h->max_row_nnz <= split) return SPMM_OK;
     DevBuf flag, nch, tmp;
     SPMM_TRY(flag.alloc(M * sizeof(int32_t), s));
     SPMM_TRY(nch.alloc(M * sizeof(int32_t), s));
     SPMM_TRY(tmp.alloc((M + 1) * sizeof(int32_t), s));
-    k_long_flags<<<grid_for(M, 256), 256, 0, s>>>(h->rowptr_p.as<int32_t>(), M, split, flag.as<int32_t>(), nch.as<int32_t>());
+    k_long_flags<<<grid_for(M, 256), 256, 0, s>>>(rowptr_p.as<int32_t>(), M, split, flag.as<int32_t>(), nch.as<int32_t>());
     SPMM_CUDA(cudaGetLastError());
     int32_t nlong = 0, nchunks = 0;
     SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), tmp.as<int32_t>(), M, &nlong, s));
     SPMM_TRY(exclusive_scan_i32(nch.as<int32_t>(), tmp.as<int32_t>(), M, &nchunks, s));
-    h->rc.n_long = nlong;
-    h->rc.n_chunks = nchunks;
+    rc.n_long = nlong;
+    rc.n_chunks = nchunks;
     return SPMM_OK;
 }
 

@@ -32,6 +32,7 @@ namespace {
 
 constexpr int SPMM_THREADS = 256;
 constexpr int32_t NOSTORE = INT_MIN;
+constexpr int SORT_WIN = 32;          // a7: short rows sorted by length within windows of this many positions
 
 // ---- per-lane vectors: W = 4 floats (LDG.128) or W = 8 floats (sm_100 LDG.E.ENL2.256) ---------------
 struct float8 {
@@ -71,57 +72,18 @@ __device__ __forceinline__ void vstore(float8 *p, const float8 &v) {
                  "f"(v.lo.z), "f"(v.lo.w), "f"(v.hi.x), "f"(v.hi.y), "f"(v.hi.z), "f"(v.hi.w) : "memory");
 }
 
-// Load flavours of the inner loop (LD template parameter; defaults are the measured best):
-//   LD 0: plain read-only loads (ld.global.nc) of (col, val) and of B rows;
-//   LD 1: L2 cache-policy hints: B rows, the reused operand -> L2::evict_last; the streamed (col, val)
-//         pairs -> L2::evict_first and no L1 allocation;
-//   LD 2: (col, val) pairs bypass L1 (L1::no_allocate), B rows plain (L1 keeps only B).
-__device__ __forceinline__ uint64_t policy_evict_last() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ uint64_t policy_evict_first() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-#define SPMM_V4_OUT "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
-#define SPMM_V8_OUT "=f"(r.lo.x), "=f"(r.lo.y), "=f"(r.lo.z), "=f"(r.lo.w), "=f"(r.hi.x), "=f"(r.hi.y), "=f"(r.hi.z), "=f"(r.hi.w)
-template <int LD>
-__device__ __forceinline__ float4 ld_b(const float4 *ptr, uint64_t pol) {
-    float4 r;
-    if (LD == 1) {
-        asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;" : SPMM_V4_OUT : "l"(ptr), "l"(pol));
-    } else {
-        r = __ldg(ptr);
-    }
-    return r;
-}
-template <int LD>
-__device__ __forceinline__ float8 ld_b(const float8 *ptr, uint64_t pol) {
+// Loads of the inner loop: read-only (ld.global.nc) B vectors -- W = 8: one 256-bit load per lane (sm_100
+// LDG.E.ENL2.256, which tools/ldpathprobe.cu measures at twice the bytes per SM clock of 128-bit loads for the same
+// gather), W = 4: LDG.128 -- and 8-byte (col, val) pairs.
+__device__ __forceinline__ float4 ld_b(const float4 *ptr) { return __ldg(ptr); }
+__device__ __forceinline__ float8 ld_b(const float8 *ptr) {
     float8 r;
-    if (LD == 1) {
-        asm("ld.global.nc.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;" : SPMM_V8_OUT : "l"(ptr), "l"(pol));
-    } else {
-        asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];" : SPMM_V8_OUT : "l"(ptr));
-    }
+    asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(r.lo.x), "=f"(r.lo.y), "=f"(r.lo.z), "=f"(r.lo.w), "=f"(r.hi.x), "=f"(r.hi.y), "=f"(r.hi.z), "=f"(r.hi.w)
+        : "l"(ptr));
     return r;
 }
-#undef SPMM_V4_OUT
-#undef SPMM_V8_OUT
-template <int LD>
-__device__ __forceinline__ int2 ld_cv(const int2 *ptr, uint64_t pol) {
-    int2 r;
-    if (LD == 1) {
-        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(ptr), "l"(pol));
-    } else if (LD == 2) {
-        asm("ld.global.nc.L1::no_allocate.v2.s32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(ptr));
-    } else {
-        r = __ldg(ptr);
-    }
-    return r;
-}
+__device__ __forceinline__ int2 ld_cv(const int2 *ptr) { return __ldg(ptr); }
 
 // One work unit per lane group: the G lanes of group g own the unit u = (start, len, dst) and the V vectors
 // (VT = W floats each) col0 + v*G of its C row (colok: inside K; indices in VT units, KV = K / W per row).
@@ -133,11 +95,11 @@ __device__ __forceinline__ int2 ld_cv(const int2 *ptr, uint64_t pol) {
 // count is warp-uniform (groups past their own length are predicated off), so the shuffles stay warp-wide.
 // Store: a whole row -> C[perm[p]] (streaming store); a chunk group of a long row -> the warp's groups
 // are reduced by a fixed xor butterfly and group 0 writes the partial.
-template <int V, int G, int U, int LD, class VT, bool MD = false>
+template <int V, int G, int U, class VT, bool MD = false>
 __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int gl, const int col0, const bool (&colok)[V],
                                           const int2 *__restrict__ cv, const VT *__restrict__ BV,
                                           VT *__restrict__ CV, const int32_t KV, VT *__restrict__ PV,
-                                          const uint64_t pol_b, const uint64_t pol_a, const CExtra &cx) {
+                                          const CExtra &cx) {
     constexpr int BATCH = (G >= 8 ? G : 8) >= U ? (G >= 8 ? G : 8) : U;   // (col, val) pairs per group per batch
     constexpr int PL = BATCH / G;                // pairs held per lane
     const int32_t start = u.x, len = u.y, dst = u.z;
@@ -149,14 +111,14 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
 #pragma unroll
     for (int p = 0; p < PL; ++p) {
         const int32_t o = p * G + gl;
-        cur[p] = o < len ? ld_cv<LD>(cv + start + o, pol_a) : make_int2(0, 0);
+        cur[p] = o < len ? ld_cv(cv + start + o) : make_int2(0, 0);
     }
     for (int32_t b0 = 0; b0 < maxlen; b0 += BATCH) {
         int2 nxt[PL];
 #pragma unroll
         for (int p = 0; p < PL; ++p) {
             const int32_t o = b0 + BATCH + p * G + gl;
-            nxt[p] = o < len ? ld_cv<LD>(cv + start + o, pol_a) : make_int2(0, 0);
+            nxt[p] = o < len ? ld_cv(cv + start + o) : make_int2(0, 0);
         }
 #pragma unroll
         for (int q0 = 0; q0 < BATCH; q0 += U) {
@@ -177,7 +139,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                     const VT *b = BV + (size_t)col[w] * KV + col0;
 #pragma unroll
                     for (int v = 0; v < V; ++v) {
-                        if (colok[v]) x[w][v] = ld_b<LD>(b + v * G, pol_b);
+                        if (colok[v]) x[w][v] = ld_b(b + v * G);
                         else vzero(x[w][v]);
                     }
                 }
@@ -192,7 +154,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                         const VT *b = BV + (size_t)col[w] * KV + col0;
 #pragma unroll
                         for (int v = 0; v < V; ++v)
-                            if (colok[v]) vfma(a[w], ld_b<LD>(b + v * G, pol_b), acc[v]);
+                            if (colok[v]) vfma(a[w], ld_b(b + v * G), acc[v]);
                     }
                 }
             }
@@ -204,7 +166,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
 #pragma unroll
         for (int v = 0; v < V; ++v)
             if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[v]);
-        if constexpr (MD) {   // spmm_run_to instantiations only (VAR bit 10): no cost for plain runs
+        if constexpr (MD) {   // spmm_run_to instantiations only: no cost for plain runs
 #pragma unroll
             for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in parameter space
                 if (i >= cx.n) break;
@@ -298,7 +260,7 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
                     const VT *b = BV + (size_t)col[w] * KV + col0;
 #pragma unroll
                     for (int v = 0; v < V; ++v) {
-                        if (colok[v] && w < rem) x[w][v] = ld_b<0>(b + v * G, 0);
+                        if (colok[v] && w < rem) x[w][v] = ld_b(b + v * G);
                         else vzero(x[w][v]);
                     }
                 }
@@ -322,7 +284,7 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
 #pragma unroll
                 for (int v = 0; v < V; ++v)
                     if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[r][v]);
-                if constexpr (MD) {   // spmm_run_to instantiations only (VAR bit 10): no cost for plain runs
+                if constexpr (MD) {   // spmm_run_to instantiations only: no cost for plain runs
 #pragma unroll
                     for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in param space
                         if (i >= cx.n) break;
@@ -337,61 +299,18 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
     }
 }
 
-// Kernel mode 1 (default): row-group SpMM over the a7 warp-task list.
-// V float4 per lane, G lanes per unit, MASK: column tail present (K not a multiple of 4*V*G).
-// VAR bit 0: L2 cache-policy hints (LD 1); bit 1: U = 4 nnz per step for V = 4.
-// Warp tasks are claimed dynamically (one atomicAdd per task on a per-column-tile counter), so the set
-// of tasks in flight stays a narrow window of the permuted order whatever the task costs: the order's
-// B-row locality survives into L2 and no warp is left with a long static tail.
-// CTA-contiguous task claiming (SCHED = 1): the CTA takes chunks of CTA_CHUNK consecutive warp tasks
-// from the global counter, so the consecutive rows of a chunk run concurrently on one SM (the paper's
-// "clusters of N_w consecutive rows ... processed in parallel" by a CTA) and their shared B rows
-// can hit in L1.  Warps draw tickets from a shared-memory counter; ticket k belongs to local chunk
-// k / CTA_CHUNK, whose global id is published in a ring slot by the warp holding its first ticket.  A
-// slot is republished only after all readers of its previous chunk have read it (no ABA, no barrier).
-constexpr int CTA_CHUNK = SPMM_THREADS / 32;
-constexpr int RING = 4;
-
-struct TaskQueue {
-    unsigned int ticket;
-    unsigned int gid[RING];
-    int tag[RING];
-    int pending[RING];
-};
-
-__device__ __forceinline__ unsigned int claim_task(TaskQueue *q, unsigned int *gcounter, int lane) {
-    unsigned int task = 0;
-    if (lane == 0) {
-        const unsigned int k = atomicAdd(&q->ticket, 1u);
-        const int c = (int)(k / CTA_CHUNK), w = (int)(k % CTA_CHUNK), s = c % RING;
-        volatile int *vtag = q->tag;
-        volatile int *vpend = q->pending;
-        volatile unsigned int *vgid = q->gid;
-        unsigned int g;
-        if (w == 0) {
-            while (vpend[s] != 0) { }
-            g = atomicAdd(gcounter, 1u);
-            vgid[s] = g;
-            vpend[s] = CTA_CHUNK - 1;
-            __threadfence_block();
-            vtag[s] = c;
-        } else {
-            while (vtag[s] != c) { }
-            __threadfence_block();
-            g = vgid[s];
-            atomicSub(&q->pending[s], 1);
-        }
-        task = g * CTA_CHUNK + (unsigned int)w;
-    }
-    return __shfl_sync(0xffffffffu, task, 0);
-}
-
-// FR > 1: the kernel also runs fused tasks (row fusion, Schedule) -- a task's type is its first unit's w
-// field (1 = fused), uniform over the warp by construction.
-// VAR bit 2: __launch_bounds__ minimum of 4 CTAs per SM (<= 64 registers); bit 3: two-deep task pipeline
-// with an L2 prefetch of the next task's (col, val) / record range (prefetch.global.L2) issued one task ahead.
-template <int V, int G, bool MASK, int SCHED, int VAR, int W, int FR = 1, int FU = 2>
-__global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 3 : 2) : ((VAR & 4) ? 4 : 3)) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
+// The row-group SpMM over the a7 warp-task list.  V vectors of W floats per lane, G lanes per unit, MASK: column
+// tail present (K not a multiple of W*V*G, several column tiles).  Warp tasks are claimed dynamically (one atomicAdd
+// per task on a per-column-tile counter), so the set of tasks in flight stays a narrow window of the permuted
+// order whatever the task costs: the order's B-row locality survives into L2 and no warp is left with a long
+// static tail.
+// FR > 1: the kernel also runs fused tasks (row fusion, Schedule) -- a task's type is its first unit's w field
+// (1 = fused), uniform over the warp by construction.  The fused kernel needs > 80 registers (2 CTAs/SM), so it
+// takes a two-deep task pipeline with an L2 prefetch (prefetch.global.L2) of the next task's record range issued
+// one task ahead (measured 0.336 -> 0.321 ms at C2, K = 64; the unfused kernel at 3 CTAs/SM gains nothing from it).
+// MD: spmm_run_to instantiations (extra C destinations), so plain runs carry no extra code.
+template <int V, int G, bool MASK, int W, int FR, bool MD>
+__global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? 2 : 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
                                                        float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
                                                        unsigned int *__restrict__ counter,
@@ -400,8 +319,9 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
     using VT = typename VecT<W>::T;
     constexpr int RPW = 32 / G;
     constexpr int CTV = V * G;
-    constexpr int LD = (VAR & 1) ? 1 : 0;
-    constexpr int U = (V * W >= 12 && !(VAR & 2)) ? 2 : 4;   // nnz per inner step (B loads in flight per lane: U*V)
+    constexpr int U = V * W >= 12 ? 2 : 4;        // nnz per inner step (B loads in flight per lane: U*V)
+    constexpr int FU = V == 1 ? 4 : 2;            // union records per inner step of a fused unit
+    constexpr bool PF = FR > 1;
     const int32_t KV = K4 * 4 / W;
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
@@ -409,22 +329,10 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
     bool colok[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) colok[v] = !MASK || (col0 + v * G < KV);
-    const uint64_t pol_b = LD == 1 ? policy_evict_last() : 0, pol_a = LD == 1 ? policy_evict_first() : 0;
 
-    __shared__ TaskQueue q;
     unsigned int tk = 0;
-    if (SCHED == 1) {
-        if (threadIdx.x == 0) {
-            q.ticket = 0;
-            for (int r = 0; r < RING; ++r) { q.tag[r] = -1; q.pending[r] = 0; q.gid[r] = 0; }
-        }
-        __syncthreads();
-        tk = claim_task(&q, counter + blockIdx.y, lane);
-    } else {
-        if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
-        tk = __shfl_sync(0xffffffffu, tk, 0);
-    }
-    constexpr bool PF = (VAR & 8) != 0 && SCHED == 0;
+    if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+    tk = __shfl_sync(0xffffffffu, tk, 0);
     int64_t t = tk;
     int4 u = t < n_tasks ? __ldg(units + t * RPW + g) : make_int4(0, 0, NOSTORE, 0);
     int64_t t1 = 0;
@@ -459,108 +367,22 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? ((V == 1 && FU == 2) ? 
             t1 = t2;
             u1 = u2;
         } else {
-            if (SCHED == 1) {
-                t_next = claim_task(&q, counter + blockIdx.y, lane);
-            } else {
-                if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
-                t_next = __shfl_sync(0xffffffffu, tk, 0);
-            }
+            if (lane == 0) tk = atomicAdd(counter + blockIdx.y, 1u);
+            t_next = __shfl_sync(0xffffffffu, tk, 0);
             u_next = t_next < n_tasks ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
         }
         bool fused = false;
         if (FR > 1) fused = __shfl_sync(0xffffffffu, u.w, 0) == 1;
         if (FR > 1 && fused) {
-            spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU, VT, (VAR & 1024) != 0>(u, g, gl, col0, colok,
+            spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU, VT, MD>(u, g, gl, col0, colok,
                                                      reinterpret_cast<const RecT<(FR > 1 ? FR : 2)> *>(recs), gdst,
                                                      reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV,
                                                      cx);
         } else {
-            spmm_unit<V, G, U, LD, VT, (VAR & 1024) != 0>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
-                                                     reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), pol_b,
-                                                     pol_a, cx);
+            spmm_unit<V, G, U, VT, MD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
+                                       reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), cx);
         }
         t = t_next;
-        u = u_next;
-    }
-}
-
-// ---- kernel mode 3: SM-affine column-tiled SpMM ---------------------------------------------------
-// One persistent CTA per SM.  Work items are (panel, column tile) pairs, panel = `ppt` consecutive warp
-// tasks of the a7 schedule (so a panel is a run of consecutive rows of the permuted order), column tile =
-// 4*V*G columns of C.  A CTA owns one item at a time and its warps claim the item's tasks from a
-// shared-memory counter, so every B row the panel's rows share is requested by ONE SM within a short time
-// and can be served by that SM's L1 (the B-row reuse the paper's CTA-aware order aims at, made
-// SM-local; the column tile keeps a panel's working set L1-sized).  The T tiles of a panel are consecutive
-// items, claimed by different SMs at about the same time, so the panel's (col, val) stream is read from
-// HBM once and from L2 by the other tiles.
-// Item hand-over without a barrier: state = (item << 32) | next task offset, advanced by atomicAdd; the
-// one warp that draws offset == #tasks claims the next item from the global counter and publishes it with
-// atomicExch; warps that overshoot spin until the item changes and retry.
-constexpr int AFF_THREADS = 768;
-
-// claim the next (item, task) of this CTA; returns false when the work is exhausted
-__device__ __forceinline__ bool aff_claim(unsigned long long *state, unsigned int *counter, int64_t n_tasks,
-                                          int32_t ppt, int32_t T, int64_t n_items, int lane, int64_t &task,
-                                          int32_t &tile) {
-    for (;;) {
-        unsigned long long old = 0;
-        if (lane == 0) old = atomicAdd(state, 1ull);
-        old = __shfl_sync(0xffffffffu, old, 0);
-        const int64_t item = (int64_t)(old >> 32);
-        if (item >= n_items) return false;
-        const int64_t off = (int64_t)(old & 0xffffffffull);
-        const int64_t panel = item / T;
-        const int64_t t0 = panel * ppt;
-        const int64_t nt = n_tasks - t0 < ppt ? n_tasks - t0 : ppt;
-        if (off < nt) {
-            task = t0 + off;
-            tile = (int32_t)(item - panel * T);
-            return true;
-        }
-        if (off == nt) {
-            if (lane == 0) atomicExch(state, (unsigned long long)atomicAdd(counter, 1u) << 32);
-        } else if (lane == 0) {
-            volatile unsigned long long *vs = state;
-            while ((int64_t)(*vs >> 32) == item) { }
-        }
-        __syncwarp();
-    }
-}
-
-template <int V, int G, int LD, int W>
-__global__ void __launch_bounds__(AFF_THREADS, 1) k_spmm_aff(const int4 *__restrict__ units, int64_t n_tasks,
-                                                          int32_t ppt, int32_t T, int64_t n_items,
-                                                          const int2 *__restrict__ cv, const float4 *__restrict__ B4,
-                                                          float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
-                                                          unsigned int *__restrict__ counter) {
-    using VT = typename VecT<W>::T;
-    constexpr int RPW = 32 / G;
-    constexpr int CTV = V * G;
-    constexpr int U = V * W == 4 ? 8 : V * W == 8 ? 4 : 2;
-    const int32_t KV = K4 * 4 / W;
-    __shared__ unsigned long long state;
-    const int lane = threadIdx.x & 31;
-    const int g = lane / G, gl = lane % G;
-    bool colok[V];
-#pragma unroll
-    for (int v = 0; v < V; ++v) colok[v] = true;
-    if (threadIdx.x == 0) state = (unsigned long long)atomicAdd(counter, 1u) << 32;
-    __syncthreads();
-    int64_t t = 0;
-    int32_t tile = 0;
-    bool ok = aff_claim(&state, counter, n_tasks, ppt, T, n_items, lane, t, tile);
-    int4 u = ok ? __ldg(units + t * RPW + g) : make_int4(0, 0, NOSTORE, 0);
-    while (ok) {
-        // claim and fetch the next task first, so its latency hides behind this one
-        int64_t t_next = 0;
-        int32_t tile_next = 0;
-        const bool ok_next = aff_claim(&state, counter, n_tasks, ppt, T, n_items, lane, t_next, tile_next);
-        const int4 u_next = ok_next ? __ldg(units + t_next * RPW + g) : make_int4(0, 0, NOSTORE, 0);
-        spmm_unit<V, G, U, LD>(u, g, gl, tile * CTV + gl, colok, cv, reinterpret_cast<const VT *>(B4),
-                               reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), 0, 0, CExtra{});
-        ok = ok_next;
-        t = t_next;
-        tile = tile_next;
         u = u_next;
     }
 }
@@ -828,8 +650,7 @@ inline unsigned g1(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<i
 
 // R > 1: row fusion requested (fuse_rows 0 = auto: keep it only when the unions hold <= 3/4 of the fused
 // rows' nnz; 2 = always).  Falls back to R = 1 (plain row units) otherwise.
-spmm_status build_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s) {
-    Schedule &S = h->sched;
+spmm_status build_schedule(spmm_ctx *h, Schedule &S, int32_t rpw, int32_t R, cudaStream_t s) {
     S.rpw = 0;
     S.fuse_req = R;
     S.fuse = 1;
@@ -866,8 +687,9 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s) 
     SPMM_TRY(groups.alloc((n_long + 1) * sizeof(int32_t), s));
     SPMM_TRY(taskbase.alloc((n_long + 2) * sizeof(int32_t), s));
     SPMM_TRY(S.pslot_ptr.alloc((n_long + 2) * sizeof(int32_t), s));
-    static const int win_env = [] { const char *e = getenv("SPMM_SORT_WIN"); return e ? atoi(e) : 32; }();
-    const int32_t win = win_env <= 0 ? 0 : (int32_t)ceil_div(win_env, rpw) * rpw;
+    // short rows are sorted by length inside windows of 32 positions (measured: no window costs 5 % on C3 identity,
+    // 32..1024 are within run-to-run noise for the locality orders -- profiles/HISTORY.md r1e)
+    const int32_t win = (int32_t)ceil_div(SORT_WIN, rpw) * rpw;
     // row fusion: groups of R consecutive short rows of each run, their column unions
     DevBuf ngroups, gbase, gpos, gseg, ucnt, gnnz, rbase;
     int32_t n_fgroups = 0;
@@ -958,92 +780,48 @@ spmm_status build_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s) 
 using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
                             unsigned int *, const int4 *, const int32_t *, const CExtra);
 
-template <int V, bool MASK, int SCHED, int VAR>
-SpmmKernel pick_g(int G) {
+// W = 4 (LDG.128) geometries: any power-of-two G <= 32, V in 1..4 (no extra-destination variants: spmm_run_to
+// copies C to the extra destinations after the run on these geometries)
+template <int V, bool MASK, bool MD>
+SpmmKernel pick_w4(int G) {
     switch (G) {
-        case 1: return k_spmm<V, 1, MASK, SCHED, VAR, 4>;
-        case 2: return k_spmm<V, 2, MASK, SCHED, VAR, 4>;
-        case 4: return k_spmm<V, 4, MASK, SCHED, VAR, 4>;
-        case 8: return k_spmm<V, 8, MASK, SCHED, VAR, 4>;
-        case 16: return k_spmm<V, 16, MASK, SCHED, VAR, 4>;
-        default: return k_spmm<V, 32, MASK, SCHED, VAR, 4>;
+        case 1: return k_spmm<V, 1, MASK, 4, 1, MD>;
+        case 2: return k_spmm<V, 2, MASK, 4, 1, MD>;
+        case 4: return k_spmm<V, 4, MASK, 4, 1, MD>;
+        case 8: return k_spmm<V, 8, MASK, 4, 1, MD>;
+        case 16: return k_spmm<V, 16, MASK, 4, 1, MD>;
+        default: return k_spmm<V, 32, MASK, 4, 1, MD>;
     }
 }
-// run-time knobs (tuning experiments; defaults are the measured best): SPMM_SCHED (0 per-warp claiming,
-// 1 CTA-contiguous queue), SPMM_VARIANT (bit 0 L2 cache hints, bit 1 U=4), SPMM_W (4: LDG.128 only)
-template <int V, bool MASK>
-SpmmKernel pick_gs(int G, int sched, int var) {
-    if (sched) return pick_g<V, MASK, 1, 0>(G);
-    switch (var) {
-        case 1: return pick_g<V, MASK, 0, 1>(G);
-        case 2: return pick_g<V, MASK, 0, 2>(G);
-        case 3: return pick_g<V, MASK, 0, 3>(G);
-        default: return pick_g<V, MASK, 0, 0>(G);
-    }
+template <bool MASK, bool MD>
+SpmmKernel pick_w4v(int V, int G) {
+    return V == 4 ? pick_w4<4, MASK, MD>(G) : V == 3 ? pick_w4<3, MASK, MD>(G) : V == 2 ? pick_w4<2, MASK, MD>(G)
+                  : pick_w4<1, MASK, MD>(G);
 }
-// 256-bit lane loads (W = 8), exact fits only, per-warp claiming, VAR 0 or 1
-template <int VAR>
+// 256-bit lane loads (W = 8), exact fits only
+template <bool MD>
 SpmmKernel pick_w8(int V, int G) {
     switch (V * 100 + G) {
-        case 104: return k_spmm<1, 4, false, 0, VAR, 8>;
-        case 108: return k_spmm<1, 8, false, 0, VAR, 8>;
-        case 204: return k_spmm<2, 4, false, 0, VAR, 8>;
-        case 208: return k_spmm<2, 8, false, 0, VAR, 8>;
-        case 408: return k_spmm<4, 8, false, 0, VAR, 8>;
-        case 416: return k_spmm<4, 16, false, 0, VAR, 8>;
-        case 432: return k_spmm<4, 32, false, 0, VAR, 8>;
+        case 104: return k_spmm<1, 4, false, 8, 1, MD>;
+        case 108: return k_spmm<1, 8, false, 8, 1, MD>;
+        case 204: return k_spmm<2, 4, false, 8, 1, MD>;
+        case 208: return k_spmm<2, 8, false, 8, 1, MD>;
+        case 408: return k_spmm<4, 8, false, 8, 1, MD>;
+        case 416: return k_spmm<4, 16, false, 8, 1, MD>;
+        case 432: return k_spmm<4, 32, false, 8, 1, MD>;
         default: return nullptr;
     }
 }
-
-// fused-capable variants (row fusion, W = 8, per-warp claiming, VAR 0): R rows per group, U records per
-// inner step (U*V B loads in flight per lane, as in the unfused kernel).  R = 4 at V = 1 (SPMM_FUSE_R=2: R = 2).
-int fuse_r_env() {
-    static const int r = [] { const char *e = getenv("SPMM_FUSE_R"); return e ? atoi(e) : 4; }();
-    return r == 2 ? 2 : 4;
-}
-int fuse_u_env() {
-    static const int u = [] { const char *e = getenv("SPMM_FUSE_U"); return e ? atoi(e) : 4; }();
-    return u == 2 ? 2 : 4;
-}
-template <int VAR>
-SpmmKernel pick_w8_fused_v(int V, int G, int R) {
-    if (V == 1 && fuse_u_env() == 2) {     // U = 2 records per step at 3 CTAs/SM (A/B: SPMM_FUSE_U=2)
-        switch (R * 10 + G) {
-            case 28: return k_spmm<1, 8, false, 0, VAR, 8, 2, 2>;
-            case 48: return k_spmm<1, 8, false, 0, VAR, 8, 4, 2>;
-            default: return nullptr;
-        }
-    }
-    switch (R * 1000 + V * 100 + G) {
-        case 2108: return k_spmm<1, 8, false, 0, VAR, 8, 2, 4>;
-        case 2208: return k_spmm<2, 8, false, 0, VAR, 8, 2, 2>;
-        case 4108: return k_spmm<1, 8, false, 0, VAR, 8, 4, 4>;
+// Row fusion only where it measured faster: G = 8 lanes per row, K = 64 (V = 1): R = 4 rows per
+// group, 4 union records per inner step; K = 128 (V = 2): R = 2, 2 records per step.  At K = 32 (G = 4) a B row is
+// one 128-byte line and the 32-byte records cost as much as they save (0.199 -> 0.197 ms at C2, 0.229 ms with the
+// prefetch pipeline); at K = 256 the R*V accumulators do not fit.
+template <bool MD>
+SpmmKernel pick_w8_fused(int V, int G) {
+    switch (V * 100 + G) {
+        case 108: return k_spmm<1, 8, false, 8, 4, MD>;
+        case 208: return k_spmm<2, 8, false, 8, 2, MD>;
         default: return nullptr;
-    }
-}
-// The fused kernel runs at 2 CTAs/SM (its R*V accumulators need > 80 registers), so it always takes the
-// next-task L2 prefetch (VAR bit 3): measured 0.336 -> 0.321 ms at C2, K = 64 (the unfused kernel at 3
-// CTAs/SM gains nothing from it).  SPMM_VARIANT=16 turns it off (A/B).
-SpmmKernel pick_w8_fused(int var, int V, int G, int R) {
-    return (var & 16) ? pick_w8_fused_v<0>(V, G, R) : pick_w8_fused_v<8>(V, G, R);
-}
-// Row fusion only where it measured faster: G = 8 lanes per row (K = 64: R = 4, K = 128: R = 2).
-// At K = 32 (G = 4) a B row is one 128-byte line and the 32-byte records cost as much as they save (0.199 ->
-// 0.197 ms at C2, 0.229 ms with the prefetch pipeline).
-int fuse_rows_for(int V, int G) {
-    if (G != 8) return 1;
-    const int R = V == 1 ? fuse_r_env() : 2;
-    return pick_w8_fused(0, V, G, R) ? R : 1;
-}
-
-SpmmKernel pick_w8v(int var, int V, int G) {
-    switch (var) {
-        case 1: return pick_w8<1>(V, G);
-        case 4: return pick_w8<4>(V, G);
-        case 8: return pick_w8<8>(V, G);
-        case 12: return pick_w8<12>(V, G);
-        default: return pick_w8<0>(V, G);
     }
 }
 
@@ -1059,191 +837,157 @@ struct Config {
 // warp at K >= 64), else G in {16, 32} with V = 4.  Otherwise W = 4: exact fit 4*V*G == K with V in
 // {4,3,2,1} and G a power of two <= 32, preferring G >= 8 (G*16 B >= 128 B: an L1 wavefront per line,
 // measured to halve L1 data-pipe load at K=64); else V=4 with a masked column tail.
-Config choose(int32_t K4, int sched, int var, bool w8ok) {
-    if (w8ok && sched == 0 && (var & 2) == 0 && K4 % 2 == 0) {
-        const int vu = var & ~16;  // bit 4 only selects the fused kernel's prefetch
+template <bool MD>
+Config choose(int32_t K4, bool w8ok) {
+    if (w8ok && K4 % 2 == 0) {
         const int32_t K8 = K4 / 2;
         for (int G : {8, 4})
             for (int V : {1, 2, 4})
                 if (V * G == K8) {
-                    SpmmKernel k = pick_w8v(vu, V, G);
+                    SpmmKernel k = pick_w8<MD>(V, G);
                     if (k) {
                         Config c{k, V, G, 1, 8};
-                        if ((vu & 3) == 0) {
-                            c.R = fuse_rows_for(V, G);
-                            c.kern_fused = c.R > 1 ? pick_w8_fused(var, V, G, c.R) : nullptr;
-                        }
+                        c.kern_fused = pick_w8_fused<MD>(V, G);
+                        c.R = c.kern_fused ? (V == 1 ? 4 : 2) : 1;
                         return c;
                     }
                 }
         for (int G : {16, 32})
-            if (4 * G == K8) return {pick_w8v(vu, 4, G), 4, G, 1, 8};
+            if (4 * G == K8) return {pick_w8<MD>(4, G), 4, G, 1, 8};
     }
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
-        int G = K4 / V;
-        if (G >= 8 && G <= 32 && (G & (G - 1)) == 0) {
-            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
-                         : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
-            return {k, V, G, 1, 4};
-        }
+        const int G = K4 / V;
+        if (G >= 8 && G <= 32 && (G & (G - 1)) == 0) return {pick_w4v<false, false>(V, G), V, G, 1, 4};
     }
     for (int V = 4; V >= 1; --V) {
         if (K4 % V) continue;
-        int G = K4 / V;
-        if (G >= 1 && G <= 32 && (G & (G - 1)) == 0) {
-            SpmmKernel k = V == 4 ? pick_gs<4, false>(G, sched, var) : V == 3 ? pick_gs<3, false>(G, sched, var)
-                         : V == 2 ? pick_gs<2, false>(G, sched, var) : pick_gs<1, false>(G, sched, var);
-            return {k, V, G, 1, 4};
-        }
+        const int G = K4 / V;
+        if (G >= 1 && G <= 32 && (G & (G - 1)) == 0) return {pick_w4v<false, false>(V, G), V, G, 1, 4};
     }
     int G = 1;
     while (G < 32 && 4 * G < K4) G <<= 1;
-    int tiles = (int)ceil_div(K4, 4 * G);
-    return {pick_gs<4, true>(G, sched, var), 4, G, tiles, 4};
+    return {pick_w4<4, true, false>(G), 4, G, (int)ceil_div(K4, 4 * G), 4};
+}
+
+Config choose_for(spmm_ctx *h, int64_t K, const float *B, const float *C, const CExtra &cx) {
+    uintptr_t align = (uintptr_t)B | (uintptr_t)C;
+    for (int i = 0; i < cx.n; ++i) align |= (uintptr_t)cx.p[i];
+    const bool w8ok = K % 8 == 0 && (align % 32) == 0;
+    Config cfg = cx.n > 0 ? choose<true>((int32_t)(K / 4), w8ok) : choose<false>((int32_t)(K / 4), w8ok);
+    if (h->params.fuse_rows == 1) {    // row fusion off (spmm_params.fuse_rows)
+        cfg.kern_fused = nullptr;
+        cfg.R = 1;
+    }
+    return cfg;
 }
 
 }  // namespace
 
-using AffKernel = void (*)(const int4 *, int64_t, int32_t, int32_t, int64_t, const int2 *, const float4 *, float4 *,
-                          int32_t, float4 *, unsigned int *);
-// mode 3 geometry: column tile of 32*V floats; W = 8: G = 4 lanes x 32 B per 128-byte line, else W = 4: G = 8
-static AffKernel pick_aff(int V, int ld, int W) {
-    switch (W * 100 + V * 10 + ld) {
-        case 410: return k_spmm_aff<1, 8, 0, 4>;
-        case 412: return k_spmm_aff<1, 8, 2, 4>;
-        case 810: return k_spmm_aff<1, 4, 0, 8>;
-        case 812: return k_spmm_aff<1, 4, 2, 8>;
-        case 820: return k_spmm_aff<2, 4, 0, 8>;
-        case 822: return k_spmm_aff<2, 4, 2, 8>;
-        case 840: return k_spmm_aff<4, 4, 0, 8>;
-        case 842: return k_spmm_aff<4, 4, 2, 8>;
-        default: return nullptr;
-    }
-}
-
-static int env_int(const char *name, int dflt) {
-    const char *e = getenv(name);
-    return e ? atoi(e) : dflt;
-}
-
-// Kernel mode 3 (SM-affine, column tiles of 32*V columns, G = 8 lanes per row): needs K % (32*V) == 0.
-static spmm_status launch_aff(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int V, int W,
-                              int32_t *launches) {
-    const int32_t K4 = (int32_t)(K / 4);
-    static const int ppt = std::max(1, env_int("SPMM_AFF_PPT", 256));
-    static const int ld = env_int("SPMM_AFF_LD", 2);
-    const int32_t rpw = W == 8 ? 8 : 4;                    // G = 4 (W = 8) or 8 (W = 4)
-    if (h->sched.rpw != rpw || h->sched.fuse_req != 1) SPMM_TRY(build_schedule(h, rpw, 1, s));
-    const Schedule &S = h->sched;
-    const int2 *cv = h->cv_p.as<int2>();
-    float4 *C4 = reinterpret_cast<float4 *>(C);
-    float4 *P4 = nullptr;
-    if (S.n_pslots > 0) {
-        const size_t need = (size_t)S.n_pslots * K * sizeof(float);
-        if (h->partials.bytes < need) SPMM_TRY(h->partials.alloc(need, s));
-        P4 = h->partials.as<float4>();
-    }
-    if (S.n_empty > 0) {
-        k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4, h->cx);
-        SPMM_CUDA(cudaGetLastError());
-        ++*launches;
-    }
-    if (S.n_tasks > 0) {
-        AffKernel kern = pick_aff(V, ld, W);
-        if (!kern) return fail(SPMM_ERR_INVALID_ARG, "unsupported SPMM_AFF_V / SPMM_AFF_LD combination");
-        const int32_t T = (int32_t)(K / (32 * V));
-        const int64_t n_items = ceil_div(S.n_tasks, ppt) * T;
-        SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 0));
-        if (h->counters.bytes < sizeof(unsigned int)) SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
-        SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, sizeof(unsigned int), s));
-        if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
-        kern<<<(unsigned)std::min<int64_t>(h->num_sms, n_items), AFF_THREADS, 0, s>>>(
-            S.units.as<int4>(), S.n_tasks, ppt, T, n_items, cv, reinterpret_cast<const float4 *>(B), C4, K4, P4,
-            h->counters.as<unsigned int>());
-        SPMM_CUDA(cudaGetLastError());
-        if (h->timing) {
-            SPMM_CUDA(cudaEventRecord(h->ev1, s));
-            h->timed = true;
+// The schedule for (rpw, R): a cached slot, else built into the oldest slot (waiting for this handle's runs in
+// flight first, since they may read the slot being replaced).  Called with h->mu held.
+static spmm_status get_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s, int *slot_out) {
+    int oldest = 0;
+    for (int i = 0; i < SCHED_CACHE; ++i) {
+        const Schedule &S = h->sched[i];
+        if (S.built && S.rpw == rpw && S.fuse_req == R) {
+            *slot_out = i;
+            return SPMM_OK;
         }
-        ++*launches;
+        if (S.built < h->sched[oldest].built) oldest = i;
     }
-    if (S.n_long > 0) {
-        k_combine<<<(unsigned)std::min<int64_t>(ceil_div(S.n_long, 8), 148 * 64), 256, 0, s>>>(
-            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, h->cx);
-        SPMM_CUDA(cudaGetLastError());
-        ++*launches;
-    }
+    for (int i = 0; i < RUN_SLOTS; ++i)
+        if (h->slots[i].used) SPMM_CUDA(cudaEventSynchronize(h->slots[i].done));
+    Schedule &S = h->sched[oldest];
+    S.built = 0;
+    SPMM_TRY(build_schedule(h, S, rpw, R, s));
+    SPMM_CUDA(cudaStreamSynchronize(s));
+    S.built = ++h->sched_seq;
+    *slot_out = oldest;
     return SPMM_OK;
 }
 
-spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches) {
+spmm_status prepare_schedule(spmm_ctx *h, int64_t K, const float *B, const float *C, cudaStream_t s) {
+    const Config cfg = choose_for(h, K, B, C, CExtra{});
+    std::lock_guard<std::mutex> lk(h->mu);
+    int slot = 0;
+    SPMM_TRY(get_schedule(h, 32 / cfg.G, cfg.R, s, &slot));
+    // the fused kernel's schedule falls back to R = 1 when the unions do not pay; the W = 4 geometry of the same K
+    // (misaligned B / C) shares rpw only when G matches, so it is prepared on first use
+    return SPMM_OK;
+}
+
+void release_run_slots(spmm_ctx *h) {
+    for (int i = 0; i < RUN_SLOTS; ++i) {
+        RunSlot &r = h->slots[i];
+        if (r.done) {
+            cudaEventSynchronize(r.done);
+            cudaEventDestroy(r.done);
+        }
+        if (r.side) {
+            cudaStreamSynchronize(r.side);
+            cudaStreamDestroy(r.side);
+        }
+        if (r.fork) cudaEventDestroy(r.fork);
+        if (r.join) cudaEventDestroy(r.join);
+        r.counters.release();
+        r.partials.release();
+        r.done = r.fork = r.join = nullptr;
+        r.side = nullptr;
+        r.used = false;
+    }
+}
+
+spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches,
+                        const CExtra &cx) {
     *launches = 0;
-    h->timed = false;
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
     const int32_t K4 = (int32_t)(K / 4);
-    static const int sched = env_int("SPMM_SCHED", 0);
-    static const int var = env_int("SPMM_VARIANT", 0);
-    static const int wmax = env_int("SPMM_W", 8);
-    uintptr_t align = (uintptr_t)B | (uintptr_t)C;
-    for (int i = 0; i < h->cx.n; ++i) align |= (uintptr_t)h->cx.p[i];
-    const bool w8ok = wmax >= 8 && K % 8 == 0 && (align % 32) == 0;
-    Config cfg = choose(K4, sched, var, w8ok);
+    Config cfg = choose_for(h, K, B, C, cx);
     bool copy_extra = false;      // spmm_run_to on a geometry without a multi-destination kernel: copy afterwards
-    if (h->cx.n > 0) {
-        SpmmKernel kmd = cfg.W == 8 ? pick_w8<1024>(cfg.V, cfg.G) : nullptr;
-        if (kmd && cfg.tiles == 1) {
-            cfg.kern = kmd;
-            if (cfg.kern_fused) cfg.kern_fused = pick_w8_fused_v<8 | 1024>(cfg.V, cfg.G, cfg.R);
-        } else {
-            copy_extra = true;
-        }
-    }
-    static const int kmode = env_int("SPMM_KERNEL", 1);
-    if (kmode == 3 && h->cx.n == 0) {   // (the experimental SM-affine mode has no extra C destinations)
-        static const int av = env_int("SPMM_AFF_V", 1);
-        const int aw = w8ok ? 8 : 4;
-        if (K % (32 * av) == 0 && pick_aff(av, env_int("SPMM_AFF_LD", 2), aw))
-            return launch_aff(h, B, K, C, s, av, aw, launches);
+    if (cx.n > 0 && !(cfg.W == 8 && cfg.tiles == 1)) {
+        cfg = choose_for(h, K, B, C, CExtra{});
+        copy_extra = true;
     }
     const int32_t rpw = 32 / cfg.G;
-    // row fusion: fuse_rows 1 = off; SPMM_FUSE=0 disables it process-wide (A/B knob)
-    static const int fuse_env = env_int("SPMM_FUSE", 1);
-    const int32_t R = (h->params.fuse_rows != 1 && fuse_env != 0 && cfg.kern_fused) ? cfg.R : 1;
-    if (h->sched.rpw != rpw || h->sched.fuse_req != R) SPMM_TRY(build_schedule(h, rpw, R, s));
-    const Schedule &S = h->sched;
+    RunSlot *rs = nullptr;
+    int sidx = 0;
+    {
+        std::lock_guard<std::mutex> lk(h->mu);
+        SPMM_TRY(get_schedule(h, rpw, cfg.R, s, &sidx));
+        rs = &h->slots[h->next_slot++ % RUN_SLOTS];
+        if (!rs->done) {
+            SPMM_CUDA(cudaEventCreateWithFlags(&rs->done, cudaEventDisableTiming));
+            SPMM_CUDA(cudaStreamCreateWithFlags(&rs->side, cudaStreamNonBlocking));
+            SPMM_CUDA(cudaEventCreateWithFlags(&rs->fork, cudaEventDisableTiming));
+            SPMM_CUDA(cudaEventCreateWithFlags(&rs->join, cudaEventDisableTiming));
+        }
+        // the slot's previous run (maybe on another stream) must be done with its scratch
+        if (rs->used) SPMM_CUDA(cudaStreamWaitEvent(s, rs->done, 0));
+        rs->used = true;
+        h->last_sched.store(sidx);
+    }
+    const Schedule &S = h->sched[sidx];
     const SpmmKernel kern = S.fuse > 1 ? cfg.kern_fused : cfg.kern;
     float4 *C4 = reinterpret_cast<float4 *>(C);
     float4 *P4 = nullptr;
     if (S.n_pslots > 0) {
         const size_t need = (size_t)S.n_pslots * K * sizeof(float);
-        if (h->partials.bytes < need) SPMM_TRY(h->partials.alloc(need, s));
-        P4 = h->partials.as<float4>();
+        if (rs->partials.bytes < need) SPMM_TRY(rs->partials.alloc(need, s));
+        P4 = rs->partials.as<float4>();
     }
-    // empty rows: zero fill on a side stream forked from / joined to `s`, one small CTA per SM, so its HBM
-    // writes run alongside the L2-bound SpMM kernel (measured 2-4 % faster steps than a preceding launch;
-    // SPMM_ZERO_SIDE=0 keeps it in `s` before the SpMM)
-    static const int zside = env_int("SPMM_ZERO_SIDE", 1);
+    // empty rows: zero fill on the slot's side stream forked from / joined to `s`, one small CTA per SM, so its HBM
+    // writes run alongside the L2-bound SpMM kernel (measured 2-4 % faster steps than a preceding launch)
     bool joined = true;
     if (S.n_empty > 0) {
-        if (zside) {
-            if (!h->side) {
-                SPMM_CUDA(cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking));
-                SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming));
-                SPMM_CUDA(cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming));
-            }
-            SPMM_CUDA(cudaEventRecord(h->ev_fork, s));
-            SPMM_CUDA(cudaStreamWaitEvent(h->side, h->ev_fork, 0));
-            k_zero_rows<<<(unsigned)h->num_sms, 128, 0, h->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4,
-                                                                   h->cx);
-            SPMM_CUDA(cudaGetLastError());
-            SPMM_CUDA(cudaEventRecord(h->ev_join, h->side));
-            joined = false;
-        } else {
-            k_zero_rows<<<g1(S.n_empty * K4), 256, 0, s>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4, h->cx);
-            SPMM_CUDA(cudaGetLastError());
-        }
+        SPMM_CUDA(cudaEventRecord(rs->fork, s));
+        SPMM_CUDA(cudaStreamWaitEvent(rs->side, rs->fork, 0));
+        k_zero_rows<<<(unsigned)h->num_sms, 128, 0, rs->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4,
+                                                                copy_extra ? CExtra{} : cx);
+        SPMM_CUDA(cudaGetLastError());
+        SPMM_CUDA(cudaEventRecord(rs->join, rs->side));
+        joined = false;
         ++*launches;
     }
     if (S.n_tasks > 0) {
@@ -1253,14 +997,14 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(S.n_tasks, SPMM_THREADS / 32),
                                                                       (int64_t)h->num_sms * occ));
         const dim3 grid((unsigned)blocks, (unsigned)cfg.tiles);
-        if (h->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int))
-            SPMM_TRY(h->counters.alloc(64 * sizeof(unsigned int), s));
-        SPMM_CUDA(cudaMemsetAsync(h->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
+        if (rs->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int))
+            SPMM_TRY(rs->counters.alloc(64 * sizeof(unsigned int), s));
+        SPMM_CUDA(cudaMemsetAsync(rs->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
         if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
                                            reinterpret_cast<const float4 *>(B), C4, K4, P4,
-                                           h->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>(),
-                                           h->cx);
+                                           rs->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>(),
+                                           copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
         if (h->timing) {
             SPMM_CUDA(cudaEventRecord(h->ev1, s));
@@ -1270,14 +1014,15 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     }
     if (S.n_long > 0) {
         k_combine<<<(unsigned)std::min<int64_t>(ceil_div(S.n_long, 8), 148 * 64), 256, 0, s>>>(
-            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, h->cx);
+            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }
-    if (!joined) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_join, 0));
+    if (!joined) SPMM_CUDA(cudaStreamWaitEvent(s, rs->join, 0));
     if (copy_extra)
-        for (int i = 0; i < h->cx.n; ++i)
-            SPMM_CUDA(cudaMemcpyAsync(h->cx.p[i], C, (size_t)M * K * sizeof(float), cudaMemcpyDeviceToDevice, s));
+        for (int i = 0; i < cx.n; ++i)
+            SPMM_CUDA(cudaMemcpyAsync(cx.p[i], C, (size_t)M * K * sizeof(float), cudaMemcpyDeviceToDevice, s));
+    SPMM_CUDA(cudaEventRecord(rs->done, s));
     return SPMM_OK;
 }
 

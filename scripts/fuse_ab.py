@@ -80,7 +80,7 @@ with open(args.out, "a") as fo:
                     if ref is None:
                         ref = out.copy()
                     info = h.schedule_info()
-                    rec = dict(env=os.environ.get("SPMM_FUSE_R", ""), matrix=name, M=a.M, nnz=a.nnz, K=K, policy=pol, fuse_rows=fuse, ms=statistics.median(ts),
+                    rec = dict(matrix=name, M=a.M, nnz=a.nnz, K=K, policy=pol, fuse_rows=fuse, ms=statistics.median(ts),
                                gflops=2 * a.nnz * K / statistics.median(ts) / 1e6, bit_identical=same, **info)
                     print(json.dumps(rec), flush=True)
                     fo.write(json.dumps(rec) + "\n")

@@ -8,7 +8,7 @@ for c in ${BENCH_CONFIGS:-c5 c3 c2}; do
 done
 for cp in ${PROFILES:-c5:cta_aware c3:cta_aware c3:identity c2:identity}; do
   c=${cp%%:*}; pol=${cp##*:}
-  PENVS="def:SPMM_KERNEL=1" CONFIG=$c POLICY=$pol bash scripts/gpu_prof_env.sh
+  PENVS="def:PROF=1" CONFIG=$c POLICY=$pol bash scripts/gpu_prof_env.sh
 done
 if [ -z "$NO_LAUNCHES" ]; then
   timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \

@@ -317,70 +317,77 @@ def test_torch_allocator_and_streams():
         pkg.use_torch_allocator(False)
 
 
-_SUBPROC = r"""
-import sys, numpy as np, torch
-sys.path.insert(0, {root!r})
-import oracle, synthetic as syn, paper_conf_ispass_mehrabilcslo21_b200 as pkg
-a = syn.rmat(12, 10, 3, "natural", int_values=True)
-B = syn.dense(a.N, 128, 4, int_values=True)
-ref, _ = oracle.spmm(a, B)
-h = pkg.SpMM.from_csr(a)
-for K in (128, 64, 32, 256):
-    BK = np.ascontiguousarray(B[:, :K]) if K <= 128 else np.ascontiguousarray(np.tile(B, (1, 2)))
-    refK, _ = oracle.spmm(a, BK)
-    for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_1"):
-        h.permute(pol, split_nnz=32)
-        C = h.run(torch.from_numpy(BK).cuda()).cpu().numpy()
-        assert np.array_equal(C.astype(np.float64), refK), (K, pol)
-# real-valued tolerance + permutation invariance
-Bf = syn.dense(a.N, 128, 9)
-af = syn.rmat(12, 10, 3, "local")
-ref, bound = oracle.spmm(af, Bf)
-hf = pkg.SpMM.from_csr(af)
-first = None
-for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_2_1"):
-    hf.permute(pol)
-    C = hf.run(torch.from_numpy(Bf).cuda()).cpu().numpy()
-    assert np.all(np.abs(C - ref) <= 1e-5 * bound + 1e-6), pol
-    if first is None: first = C
-    assert np.array_equal(C.view(np.int32), first.view(np.int32)), pol
-# row fusion forced on a stencil (fused tasks + a split row's chunk tasks in one launch)
-st = syn.stencil27(12, 5, int_values=True)
-rows = [st.colidx[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
-vals = [st.value[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
-rows[100] = list(range(0, st.N, 3)); vals[100] = [1.0 + (t % 3) for t in range(len(rows[100]))]
-st = syn.from_lists(st.M, st.N, rows, vals)
-hs = pkg.SpMM.from_csr(st)
-for K in (32, 64, 128):
-    Bs = syn.dense(st.N, K, 6, int_values=True)
-    refs, _ = oracle.spmm(st, Bs)
-    for pol in ("identity", "cta_aware"):
-        hs.permute(pol, fuse_rows=2)
-        C = hs.run(torch.from_numpy(Bs).cuda()).cpu().numpy()
-        assert np.array_equal(C.astype(np.float64), refs), (K, pol)
-print("OK")
-"""
+def _dev(x, offset16):
+    """A contiguous CUDA copy of x; offset16: placed 16 bytes past a 256-byte aligned base (16- but not
+    32-byte aligned -> the 128-bit-load geometry W = 4 instead of the 256-bit one)."""
+    t = torch.from_numpy(np.ascontiguousarray(x))
+    if not offset16:
+        return t.cuda()
+    buf = torch.empty(t.numel() + 4, dtype=torch.float32, device="cuda")
+    v = buf[4:].view(t.shape)
+    v.copy_(t)
+    assert v.data_ptr() % 32 == 16
+    return v
 
 
-@pytest.mark.parametrize("env", [{"SPMM_SCHED": "1"}, {"SPMM_VARIANT": "1"}, {"SPMM_VARIANT": "2"},
-                                 {"SPMM_VARIANT": "3"}, {"SPMM_W": "4"}, {"SPMM_SORT_WIN": "0"},
-                                 {"SPMM_SORT_WIN": "128"}, {"SPMM_ZERO_SIDE": "0"}, {"SPMM_KERNEL": "3"},
-                                 {"SPMM_KERNEL": "3", "SPMM_AFF_V": "2", "SPMM_AFF_LD": "0"},
-                                 {"SPMM_KERNEL": "3", "SPMM_AFF_PPT": "4"}, {"SPMM_KERNEL": "3", "SPMM_AFF_V": "4"},
-                                 {"SPMM_W": "4", "SPMM_KERNEL": "3"}, {"SPMM_VARIANT": "4"}, {"SPMM_VARIANT": "8"},
-                                 {"SPMM_VARIANT": "12"}, {"SPMM_FUSE_R": "2"}, {"SPMM_FUSE": "0"},
-                                 {"SPMM_FUSE_R": "2", "SPMM_VARIANT": "16"}])
-def test_kernel_variants_exact(env):
-    """The run-time kernel variants (CTA-contiguous queue, cache hints, U=4, 128-bit lane loads, schedule
-    windows, SM-affine column tiles, 4 CTAs/SM, next-task L2 prefetch, row fusion R = 2 / off) are exact on
-    integer inputs and permutation-invariant on real inputs."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", _SUBPROC.format(root=root)], env={**os.environ, **env},
-                       capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0 and "OK" in r.stdout, r.stderr[-2000:]
+@pytest.mark.parametrize("offset16", [False, True])
+@pytest.mark.parametrize("fuse_rows", [0, 1, 2])
+def test_kernel_geometries_exact(offset16, fuse_rows):
+    """Every lane geometry (256-bit loads when B / C are 32-byte aligned, 128-bit otherwise), row fusion auto /
+    off / forced, split rows (split_nnz = 32), K = 32..256: exact on integer inputs, permutation-invariant bits
+    and within the north-star tolerance on real inputs."""
+    a = syn.rmat(12, 10, 3, "natural", int_values=True)
+    B = syn.dense(a.N, 128, 4, int_values=True)
+    h = pkg.SpMM.from_csr(a)
+    for K in (128, 64, 32, 256):
+        BK = np.ascontiguousarray(B[:, :K]) if K <= 128 else np.ascontiguousarray(np.tile(B, (1, 2)))
+        refK, _ = oracle.spmm(a, BK)
+        Bd = _dev(BK, offset16)
+        Cd = _dev(np.zeros((a.M, K), np.float32), offset16)
+        for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_1"):
+            h.permute(pol, split_nnz=32, fuse_rows=fuse_rows)
+            h.run(Bd, Cd)
+            assert np.array_equal(Cd.cpu().numpy().astype(np.float64), refK), (K, pol)
+    h.close()
+    Bf = syn.dense(2 ** 12, 128, 9)
+    af = syn.rmat(12, 10, 3, "local")
+    ref, bound = oracle.spmm(af, Bf)
+    hf = pkg.SpMM.from_csr(af)
+    Bd = _dev(Bf, offset16)
+    Cd = _dev(np.zeros((af.M, 128), np.float32), offset16)
+    first = None
+    for pol in ("identity", "nnz_sort", "cta_aware", "hybrid_2_1"):
+        hf.permute(pol, fuse_rows=fuse_rows)
+        hf.run(Bd, Cd)
+        C = Cd.cpu().numpy()
+        assert np.all(np.abs(C - ref) <= 1e-5 * bound + 1e-6), pol
+        if first is None:
+            first = C
+        assert np.array_equal(C.view(np.int32), first.view(np.int32)), pol
+    hf.close()
+    # row fusion on a stencil (fused tasks + a split row's chunk tasks in one launch when forced)
+    st = syn.stencil27(12, 5, int_values=True)
+    rows = [st.colidx[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
+    vals = [st.value[st.rowidx[i]:st.rowidx[i + 1]].tolist() for i in range(st.M)]
+    rows[100] = list(range(0, st.N, 3))
+    vals[100] = [1.0 + (t % 3) for t in range(len(rows[100]))]
+    st = syn.from_lists(st.M, st.N, rows, vals)
+    hs = pkg.SpMM.from_csr(st)
+    for K in (32, 64, 128):
+        Bs = syn.dense(st.N, K, 6, int_values=True)
+        refs, _ = oracle.spmm(st, Bs)
+        Bd = _dev(Bs, offset16)
+        Cd = _dev(np.zeros((st.M, K), np.float32), offset16)
+        for pol in ("identity", "cta_aware"):
+            hs.permute(pol, fuse_rows=fuse_rows)
+            hs.run(Bd, Cd)
+            assert np.array_equal(Cd.cpu().numpy().astype(np.float64), refs), (K, pol)
+            fused = hs.schedule_info()["fuse"]
+            if fuse_rows == 1 or offset16 or K == 32:
+                assert fused == 1, (K, pol, fused)
+            elif fuse_rows == 2:
+                assert fused == (4 if K == 64 else 2), (K, pol, fused)
+    hs.close()
 
 
 def test_kernel_timing_api():

@@ -33,10 +33,10 @@ __device__ __forceinline__ f8 ld8(const void *p) {
     return r;
 }
 
-// random row index stream: counter-based hash, no memory traffic
+// random row index stream: a multiplicative hash of a counter, nrows a power of two (2 integer ops: the probe
+// must stay bound by its loads, not by index arithmetic)
 __device__ __forceinline__ uint32_t hrow(uint64_t x, uint32_t nrows) {
-    x ^= x >> 33; x *= 0xff51afd7ed558ccdULL; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ULL; x ^= x >> 33;
-    return (uint32_t)(x % nrows);
+    return ((uint32_t)x * 0x9E3779B1u) >> 7 & (nrows - 1);
 }
 
 constexpr int U = 4;   // independent row loads in flight per lane
@@ -57,7 +57,7 @@ __global__ void __launch_bounds__(256, 3) k_probe(const char *__restrict__ B, ui
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const uint32_t r = hrow(((wid * iters + it) * U + u) * 8 + g, nrows);
-                const char *p = B + (size_t)r * RB + (size_t)((it * U + u) % (RB / span)) * span + gl * 32;
+                const char *p = B + (size_t)r * RB + (size_t)((it * U + u) & (RB / span - 1)) * span + gl * 32;
                 x[u] = ld8<SHAPE == 4>(p);
             }
 #pragma unroll
@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(256, 3) k_probe(const char *__restrict__ B, ui
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const uint32_t r = hrow((wid * iters + it) * U + u, nrows);
-                x[u] = __ldg(reinterpret_cast<const float4 *>(B + (size_t)r * RB) + ((it * U + u) % (RB / 512)) * 32 + lane);
+                x[u] = __ldg(reinterpret_cast<const float4 *>(B + (size_t)r * RB) + ((it * U + u) & (RB / 512 - 1)) * 32 + lane);
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) acc += x[u].x + x[u].w;
@@ -80,7 +80,7 @@ __global__ void __launch_bounds__(256, 3) k_probe(const char *__restrict__ B, ui
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const uint32_t r = hrow((wid * iters + it) * U + u, nrows);
-                x[u] = __ldg(reinterpret_cast<const float *>(B + (size_t)r * RB) + ((it * U + u) % (RB / 128)) * 32 + lane);
+                x[u] = __ldg(reinterpret_cast<const float *>(B + (size_t)r * RB) + ((it * U + u) & (RB / 128 - 1)) * 32 + lane);
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) acc += x[u];
@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(256, 1) k_probe_smem(const char *__restrict__ 
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const uint32_t r = hrow((wid * iters + it) * U + u, nrows);
-            x[u] = reinterpret_cast<const float4 *>(sm + (size_t)r * RB)[((it * U + u) % (RB / 512)) * 32 + lane];
+            x[u] = reinterpret_cast<const float4 *>(sm + (size_t)r * RB)[((it * U + u) & (RB / 512 - 1)) * 32 + lane];
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) acc += x[u].x + x[u].w;
@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(256, 1) k_probe_smem(const char *__restrict__ 
 int main(int argc, char **argv) {
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-    const int RB = argc > 1 ? atoi(argv[1]) : 512;
+    const int RB = argc > 1 ? atoi(argv[1]) : 512;   // a power of two >= 512
     const size_t Bbytes = (size_t)1 << 30;
     char *B;
     float *out;
