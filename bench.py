@@ -243,59 +243,83 @@ def run_reference(args):
     }))
 
 
-def p2p_send(dist, t, dst):
-    """NCCL: send the device tensor.  gloo (one-GPU dry runs of the N>1 path only): via host memory."""
-    dist.send(t if dist.get_backend() == "nccl" else t.cpu(), dst=dst)
-
-
-def p2p_recv(torch, dist, t, src):
-    if dist.get_backend() == "nccl":
-        dist.recv(t, src=src)
-    else:
-        h = torch.empty(t.shape, dtype=t.dtype)
-        dist.recv(h, src=src)
-        t.copy_(h)
-
-
-def shard_inputs(torch, dist, a_full, world, rank, dev, pkg, compact=False):
-    """Rank 0 holds the generated matrix; every rank gets its nnz-balanced row shard as CUDA tensors
-    (NCCL send/recv for N>1).  Returns (M_r, lo, (rowidx, colidx, value), meta, cols) with rowidx rebased to 0.
-    compact (N>1, sharded.py compact_B): the shard's columns are renumbered to their index in its sorted list of
-    distinct columns `cols` (int64, device), so the rank needs only B[cols] (|cols| x K)."""
-    from paper_conf_ispass_mehrabilcslo21_b200.sharded import compact_shard, make_shard, shard_columns
-    if rank == 0:
-        bounds = pkg.spmm_partition_by_nnz(a_full.rowidx, world)
-        cols_all = [shard_columns(a_full.rowidx, a_full.colidx, bounds, r) for r in range(world)] if compact else None
-        meta = torch.tensor([[int(bounds[r + 1] - bounds[r]), int(a_full.rowidx[bounds[r + 1]] - a_full.rowidx[bounds[r]]),
-                              int(bounds[r]), len(cols_all[r]) if compact else a_full.N] for r in range(world)],
-                            dtype=torch.int64, device=dev)
-    else:
-        meta = torch.empty((world, 4), dtype=torch.int64, device=dev)
+def timed_max(torch, dist, world, fn, reps, stream):
+    """Mean CUDA-event time (ms) of fn() on `stream`, barrier before each rep, max over ranks."""
+    ts = []
+    for _ in range(reps):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fn()
+        e1.record(stream)
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.mean(ts)], dtype=torch.float64, device="cuda")
     if world > 1:
-        dist.broadcast(meta, src=0)
-    parts = None
-    if rank == 0:
-        parts = []
-        for r in range(world):
-            sh = make_shard(a_full.M, a_full.N, a_full.rowidx, a_full.colidx, a_full.value, bounds, r)
-            if compact:
-                sh = compact_shard(sh, cols_all[r])
-            parts.append((torch.from_numpy(sh.rowidx), torch.from_numpy(sh.colidx), torch.from_numpy(sh.value))
-                         + ((torch.from_numpy(cols_all[r]),) if compact else ()))
-        for r in range(1, world):
-            for t in parts[r]:
-                p2p_send(dist, t.to(dev), r)
-        mine = tuple(t.to(dev) for t in parts[0])
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps=5, chunks=4):
+    """N>1: the data-path communication of the sharded mode, timed on the device (max over
+    ranks) and reported in GB/s of bytes moved between GPUs:
+      b_exchange   -- per-rank B rows (distribute_B) or the broadcast of all of B;
+      c_allgather  -- NCCL all_gather of the C shards (allgather_C);
+      fused        -- the SpMM with its epilogue storing every row into every rank's symmetric-memory full-C
+                      buffer (spmm_run_to), against the plain SpMM: the all-gather's added cost;
+      multicast    -- the same through the NVLS multicast address (spmm_run_multicast), where the group has one;
+      pipelined    -- one end-to-end step with B sent in column chunks, the SpMM of chunk c overlapping the
+                      transfer of chunk c + 1 (run_pipelined), against the sequential exchange + SpMM."""
+    world = sh.world
+    out = {}
+    mine = torch.tensor([Bd.shape[0]], dtype=torch.int64, device="cuda")
+    every = [torch.empty_like(mine) for _ in range(world)]
+    dist.all_gather(every, mine)
+    b_rows = [int(t.item()) for t in every]          # B rows each rank holds
+    b_bytes = (sum(b_rows) - b_rows[0]) * K * 4 if compact else (world - 1) * sh.N * K * 4   # sent by rank 0
+    if compact:
+        fn_b = lambda: sh.distribute_B(Bfull, K=K, src=0, device=Bd.device)  # noqa: E731
     else:
-        Mr, nnzr, nc = int(meta[rank, 0]), int(meta[rank, 1]), int(meta[rank, 3])
-        mine = (torch.empty(Mr + 1, dtype=torch.int64, device=dev), torch.empty(nnzr, dtype=torch.int32, device=dev),
-                torch.empty(nnzr, dtype=torch.float32, device=dev))
-        if compact:
-            mine = mine + (torch.empty(nc, dtype=torch.int64, device=dev),)
-        for t in mine:
-            p2p_recv(torch, dist, t, 0)
-    cols = mine[3] if compact else None
-    return int(meta[rank, 0]), int(meta[rank, 2]), mine[:3], meta, cols, (cols_all if rank == 0 else None)
+        fn_b = lambda: sh.broadcast_B(Bd, src=0)  # noqa: E731
+    tb = timed_max(torch, dist, world, fn_b, reps, stream)
+    out["b_exchange"] = {"ms": tb, "bytes": b_bytes, "GBps": b_bytes / (tb * 1e-3) / 1e9,
+                         "how": "distribute_B (NCCL sends of B[cols_p])" if compact else "NCCL broadcast"}
+    c_bytes = (sh.M - Cd.shape[0]) * K * 4      # the other ranks' C rows this rank receives
+    tc = timed_max(torch, dist, world, lambda: sh.allgather_C(Cd), reps, stream)
+    out["c_allgather"] = {"ms": tc, "bytes_received_rank": c_bytes, "GBps_received_rank": c_bytes / (tc * 1e-3) / 1e9,
+                          "how": "NCCL all_gather of padded shards (allgather_C)"}
+    t_plain = timed_max(torch, dist, world, lambda: h.run(Bd, Cd), reps, stream)
+    out["spmm_ms"] = t_plain
+    if sh.comm.nccl:
+        try:
+            buf, ptrs, hdl = sh.symmetric_C(K)
+            t_f = timed_max(torch, dist, world, lambda: sh.run_allgather_fused(Bd, ptrs), reps, stream)
+            out["fused"] = {"ms": t_f, "allgather_added_ms": t_f - t_plain,
+                            "GBps_per_rank_out": (world - 1) * Cd.shape[0] * K * 4 / max(t_f * 1e-3, 1e-9) / 1e9,
+                            "how": "spmm_run_to: per-peer stores into the symmetric-memory full-C buffers"}
+            mc = int(getattr(hdl, "multicast_ptr", 0) or 0)
+            if mc:
+                t_m = timed_max(torch, dist, world, lambda: sh.run_allgather_multicast(Bd, mc), reps, stream)
+                out["multicast"] = {"ms": t_m, "allgather_added_ms": t_m - t_plain,
+                                    "how": "spmm_run_multicast: one multimem.st per element (NVLS)"}
+            else:
+                out["multicast"] = {"skipped": "the symmetric-memory rendezvous has no multicast address"}
+            del buf
+        except Exception as e:  # noqa: BLE001
+            out["fused"] = {"error": str(e)[:200]}
+    else:
+        out["fused"] = {"skipped": "symmetric memory needs NCCL"}
+    if compact:
+        Cp = torch.empty_like(Cd)
+        t_seq = timed_max(torch, dist, world, lambda: h.run(fn_b(), Cd), reps, stream)
+        t_pipe = timed_max(torch, dist, world, lambda: sh.run_pipelined(Bfull, K=K, chunks=chunks, C_local=Cp,
+                                                                         src=0, device=Bd.device), reps, stream)
+        torch.cuda.synchronize()
+        out["pipelined"] = {"ms": t_pipe, "sequential_ms": t_seq, "chunks": chunks,
+                            "bit_identical_to_run": bool(torch.equal(Cp.view(torch.int32), Cd.view(torch.int32)))}
+    return out
 
 
 def main():
@@ -348,49 +372,52 @@ def main():
     a_full = make_matrix(cfg) if rank == 0 else None
     gen_s = time.perf_counter() - t0
     compact = world > 1 and args.b_exchange == "rows"
-    Mr, lo, (rowidx_d, colidx_d, value_d), meta, cols_d, cols_all = shard_inputs(torch, dist, a_full, world, rank,
-                                                                                dev, pkg, compact=compact)
-    N = a_full.N if rank == 0 else None
-    nN = torch.tensor([N or 0], dtype=torch.int64, device=dev)
-    if world > 1:
-        dist.broadcast(nN, src=0)
-    N = int(nN.item())                 # global N (B rows)
-    N_loc = int(meta[rank, 3].item()) if compact else N   # B rows this rank holds
-    nnz_r = int(colidx_d.numel())
-    nnz_total = int(meta[:, 1].sum().item())
-    seen = torch.zeros(N_loc, dtype=torch.bool, device=dev)
-    seen[colidx_d.long()] = True
-    ncols = int(seen.sum().item())
-    del seen
+    pkg.use_torch_allocator(True)
+    sh = None
+    if world == 1:
+        h = pkg.SpMM.from_csr(a_full)
+        Mr, lo, N, N_loc, nnz_r, nnz_total = a_full.M, 0, a_full.N, a_full.N, a_full.nnz, a_full.nnz
+        seen = np.zeros(a_full.N, dtype=bool)
+        seen[a_full.colidx] = True
+        ncols = int(seen.sum())
+        del seen
+    else:
+        # one sharding path (sharded.py): rank 0 partitions by nnz and sends every rank its own shard (NCCL p2p of
+        # device tensors; compact columns with --b-exchange rows); no rank holds another rank's rows
+        from paper_conf_ispass_mehrabilcslo21_b200.sharded import ShardedSpMM
+        sh = ShardedSpMM.scatter(a_full if rank == 0 else None, src=0, compact_B=compact, device=dev)
+        h = sh.local
+        Mr, lo, N, N_loc, nnz_r = sh.shard.M, sh.row_offset, sh.N, sh.shard.N, sh.shard.nnz
+        cidx = torch.as_tensor(sh.shard.colidx).to(dev).long()
+        seen = torch.zeros(N_loc, dtype=torch.bool, device=dev)
+        seen[cidx] = True
+        ncols = int(seen.sum().item())
+        del seen, cidx
+        nt = torch.tensor([nnz_r], dtype=torch.int64, device=dev)
+        dist.all_reduce(nt)
+        nnz_total = int(nt.item())
     alg_bytes = 4 * (Mr + 1) + 8 * nnz_r + 4 * K * ncols + 4 * Mr * K   # north star, this rank's shard
     flops = 2.0 * nnz_r * K
     total_flops = 2.0 * nnz_total * K
 
     # B: drawn on rank 0 (host); N>1: broadcast over NCCL, or (--b-exchange rows, default) each rank receives
-    # only the rows its shard references (NCCL send of B[cols_p]; sharded.py compact_B) -- outside the timed region
+    # only the rows its shard references (sharded.py distribute_B: NCCL sends of B[cols_p]) -- outside the timed region
     B_host = torch.from_numpy(syn.dense(N, K, bseed)) if rank == 0 else None
-    if compact:
-        if rank == 0:
-            Bfull = B_host.to(dev)
-            for r in range(1, world):
-                p2p_send(dist, Bfull.index_select(0, torch.from_numpy(cols_all[r]).to(dev)).contiguous(), r)
-            Bd = Bfull.index_select(0, cols_d).contiguous()
-            del Bfull
-        else:
-            Bd = torch.empty((N_loc, K), dtype=torch.float32, device=dev)
-            p2p_recv(torch, dist, Bd, 0)
+    Bfull = None
+    if world == 1:
+        Bd = B_host.to(dev)
+    elif compact:
+        Bfull = B_host.to(dev) if rank == 0 else None
+        Bd = sh.distribute_B(Bfull, K=K, src=0, device=dev)
     else:
         Bd = B_host.to(dev) if rank == 0 else torch.empty((N, K), dtype=torch.float32, device=dev)
-        if world > 1:
-            dist.broadcast(Bd, src=0)
+        sh.broadcast_B(Bd, src=0)
     Cd = torch.empty((Mr, K), dtype=torch.float32, device=dev)
     flush_buf = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
 
     def flush():
         flush_buf.fill_(1.0)
 
-    pkg.use_torch_allocator(True)
-    h = pkg.SpMM(Mr, N_loc, rowidx_d, colidx_d, value_d)
     torch.cuda.synchronize()
     feat_t0 = time.perf_counter()
     feats = h.features()
@@ -462,15 +489,33 @@ def main():
     step_achieved = alg_bytes / (statistics.mean(ts) * 1e-3) / 1e9
     l2 = None
     if rank == 0:
-        try:   # second ceiling: every nnz pulls a 4K-byte B row through L2 unless it hits in L1
+        # second ceiling: the SM load path.  Every B-row load (one per nnz, or one per union record of a fused row
+        # group) brings 4K bytes into registers; tools/ldpathprobe.cu measures how many bytes per SM clock k_spmm's
+        # load shape (8-lane groups x one 256-bit load per lane, random rows) can gather from an L2-resident window
+        # and from an L1-resident one.  At the clock sampled in the timed region, 4K * loads / that rate bounds the
+        # kernel whatever HBM does.
+        try:
             import tools
-            l2_bw = tools.l2_read_bandwidth() / 1e9
-            l2_bytes = 4.0 * K * nnz_r
-            l2 = {"read_peak_gbs": l2_bw, "b_row_bytes_per_launch": l2_bytes,
-                  "ceiling_frac_without_l1_reuse": (kern_bytes / peak) / (l2_bytes / l2_bw),
-                  "how": "tools/l2probe.cu: float4 __ldcg over a 64 MiB L2-resident buffer, CUDA events"}
+            sch = pol_res[best]["schedule"]
+            loads = (nnz_r - sch["fused_nnz"] + sch["records"]) if sch["fuse"] > 1 else nnz_r
+            g_bytes = 4.0 * K * loads
+            l2_gbs, l2_bpc = tools.ldpath_gather(0, 16 << 20, 4 * K)
+            l1_gbs, l1_bpc = tools.ldpath_gather(0, 32 << 10, 4 * K)
+            nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+            mhz = clocks.get("sm_mhz") or clocks.get("sm_max_mhz") or 1965.0
+            l2_at_clk = l2_bpc * nsm * mhz * 1e6 / 1e9
+            l2 = {"gather_l2_gbs": l2_gbs, "gather_l2_bytes_per_sm_clk": l2_bpc,
+                  "gather_l1_gbs": l1_gbs, "gather_l1_bytes_per_sm_clk": l1_bpc,
+                  "b_row_loads_per_launch": loads, "b_row_bytes_per_launch": g_bytes,
+                  "timed_region_sm_mhz": mhz, "gather_l2_gbs_at_timed_clock": l2_at_clk,
+                  "kernel_frac_of_l2_gather_ceiling": (g_bytes / (kern_ms * 1e-3) / 1e9) / l2_at_clk if kern_ms else None,
+                  "hbm_ceiling_frac_without_l1_reuse": (kern_bytes / peak) / (g_bytes / l2_at_clk),
+                  "how": "tools/ldpathprobe.cu shape 0 (k_spmm's load shape) over a 16 MiB (L2) / 32 KiB (L1) window of "
+                         f"random {4 * K}-byte rows; bytes per SM clock x SMs x the timed region's median SM clock"}
         except Exception as e:  # noqa: BLE001
             l2 = {"error": str(e)[:200]}
+
+    multi = measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream) if world > 1 else None
 
     # ---- e2e through the public API with host buffers ----
     # N=1: spmm_run_host (H2D of B, SpMM, D2H of C).  N>1: rank 0 H2D of B, NCCL broadcast, SpMM on every
@@ -493,7 +538,7 @@ def main():
             else:
                 if rank == 0:
                     Bd.copy_(Bp, non_blocking=True)
-                dist.broadcast(Bd, src=0)
+                sh.broadcast_B(Bd, src=0)
             h.run(Bd, Cd)
             Cp.copy_(Cd, non_blocking=True)
             torch.cuda.current_stream().synchronize()
@@ -531,9 +576,12 @@ def main():
             del Cp2
         except Exception as e:  # noqa: BLE001
             e2e_pipe = {"error": str(e)[:200]}
-    h2d = int(meta[:, 3].sum().item()) * K * 4 if compact else N * K * 4
+    rows_tot = torch.tensor([N_loc, Mr], dtype=torch.int64, device=dev)   # B rows copied in, C rows copied out
+    if world > 1:
+        dist.all_reduce(rows_tot)
+    h2d = int(rows_tot[0].item()) * K * 4 if compact else N * K * 4
     e2e = {"value": total_flops / float(e2e_t.item()) / 1e6, "unit": "GFLOP/s",
-           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(int(meta[:, 0].sum().item()) * K * 4),
+           "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(rows_tot[1].item()) * K * 4,
            "ms_per_step": float(e2e_t.item()),
            "path": "spmm_run_host" if world == 1 else
            ("per-rank H2D of its B rows (pinned) + spmm_run + D2H of its C shard" if compact else
@@ -553,7 +601,10 @@ def main():
     cus = None
     if not args.no_cusparse and rank == 0:
         import tools
-        rp32 = rowidx_d.to(torch.int32)
+        src_csr = a_full if world == 1 else sh.shard
+        rp32 = torch.as_tensor(np.asarray(src_csr.rowidx)).to(dev).to(torch.int32)
+        colidx_d = torch.as_tensor(np.asarray(src_csr.colidx)).to(dev)
+        value_d = torch.as_tensor(np.asarray(src_csr.value)).to(dev)
         Cc = torch.empty_like(Cd)
         h.run(Bd, Cd)                 # our C of the selected policy, for the sanity diff
         torch.cuda.synchronize()
@@ -579,7 +630,7 @@ def main():
                    "via": "cusparseSpMM (CUSPARSE_SPMM_CSR_ALG1/2/3, default), row-major, best-of, rank 0 shard"}
         else:
             cus = {"error": "no cuSPARSE algorithm ran", "per_alg": per_alg}
-        del Cc, rp32
+        del Cc, rp32, colidx_d, value_d
 
     if rank != 0:
         if world > 1:
@@ -590,18 +641,15 @@ def main():
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(a_full, B_host.numpy(), K)
-    # DRAM bytes of one k_spmm launch on this config from the committed ncu --set full capture (scripts/
-    # collect_profiles.py); the selected policy's capture if there is one, else the closest-timed profiled policy
-    traffic, traffic_from = None, None
+    # DRAM bytes of one k_spmm launch of the SELECTED policy on this config, from the committed ncu --set full
+    # capture (scripts/profile_policies.py -> scripts/collect_profiles.py); null when that policy has none
+    traffic, traffic_from = None, f"no committed ncu capture of {args.config}/{best}"
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(prof) and world == 1:
-        allp = json.load(open(prof))
-        cands = [p for p in pol_res if f"{args.config}/{p}" in allp]
-        if cands:
-            pick = best if best in cands else min(cands, key=lambda p: abs(pol_res[p]["ms"] - pol_res[best]["ms"]))
-            d = allp[f"{args.config}/{pick}"]
+        d = json.load(open(prof)).get(f"{args.config}/{best}")
+        if d:
             traffic = d.get("dram_bytes_per_launch")
-            traffic_from = f"ncu --set full of {d.get('kernel', 'k_spmm')} on {args.config}/{pick} ({d.get('round')})"
+            traffic_from = f"ncu --set full of {d.get('kernel', 'k_spmm')} on {args.config}/{best} ({d.get('round')})"
 
     for pol, r in pol_res.items():
         r["roofline_frac"] = alg_bytes / (r["ms"] * 1e-3) / 1e9 / peak
@@ -610,7 +658,7 @@ def main():
         "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": cfg["desc"], "M": int(meta[:, 0].sum().item()), "N": N, "nnz": nnz_total, "K": K,
+        "config": {"workload": cfg["desc"], "M": a_full.M if world == 1 else sh.M, "N": N, "nnz": nnz_total, "K": K,
                    "policy": best, "window": args.window, "parallelism": f"rows sharded by nnz over {world} GPU(s)",
                    "b_exchange": ("per-rank B rows (compact shards)" if compact else "broadcast") if world > 1 else None,
                    "l2": "256 MiB scratch written between timed steps (L2 flush); B, C also > L2",
@@ -628,6 +676,7 @@ def main():
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
+        "multi_gpu": multi,
         "clocks": clocks,
         "policies": pol_res,
         "cusparse": cus,

@@ -173,6 +173,22 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
 spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
                         int64_t row_offset, void *cuda_stream);
 
+/* spmm_run into a C whose rows are ldc floats apart (ldc >= K, ldc % 4 == 0): C[r * ldc + k], k < K; the other
+ * columns are untouched.  Lets a caller compute column blocks of a wider C, e.g. the column chunks of a B that
+ * arrives in pieces (ShardedSpMM.run_pipelined: the SpMM of chunk c overlaps the transfer of chunk c + 1,
+ * SURVEY §8(f) f2 iii).  Errors as spmm_run, plus UNSUPPORTED for a bad ldc. */
+spmm_status spmm_run_ld(spmm_handle h, const float *B, int64_t K, float *C, int64_t ldc, void *cuda_stream);
+
+/* spmm_run_to through an NVLink-SHARP multicast address (SURVEY §8(f) f2 ii, NVLS): C_mc is the multicast
+ * address of a [>= row_offset + M][K] float32 buffer bound on every GPU of the group (e.g. torch symmetric
+ * memory's multicast_ptr); every C row this handle computes is stored ONCE, with multimem.st, and the NVSwitch
+ * delivers it to the buffer on every member GPU (this one included) -- one store per element instead of one
+ * per peer.  Needs K % 8 == 0 and 32-byte aligned B and destination rows (the 256-bit lane geometry).
+ * Asynchrony as spmm_run; the caller orders completion across GPUs (e.g. a barrier after the kernels).
+ * Errors: INVALID_ARG (NULL, negative row_offset), UNSUPPORTED (K / alignment), STATE, OOM, CUDA. */
+spmm_status spmm_run_multicast(spmm_handle h, const float *B, int64_t K, float *C_mc, int64_t row_offset,
+                               void *cuda_stream);
+
 /* End-to-end variant: B_host -> device, spmm_run, C -> C_host, all on cuda_stream with handle-owned
  * staging buffers (grown on demand).  Host buffers should be pinned for full copy bandwidth.
  * Synchronises cuda_stream before returning. */

@@ -56,7 +56,7 @@ _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, c
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
 EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_prepare", "spmm_get_perm",
-           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_to", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
+           "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_to", "spmm_run_ld", "spmm_run_multicast", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
 
@@ -85,6 +85,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_features_b200": (st, [vp, ctypes.c_int, i64, vp, vp]),
         "spmm_run": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_to": (st, [vp, vp, i64, vp, i32, i64, vp]),
+        "spmm_run_ld": (st, [vp, vp, i64, vp, i64, vp]),
+        "spmm_run_multicast": (st, [vp, vp, i64, vp, i64, vp]),
         "spmm_run_host": (st, [vp, vp, i64, vp, vp]),
         "spmm_run_host_batch": (st, [vp, i64, vp, i64, vp, vp]),
         "spmm_predict": (st, [vp, vp, i64, i32, vp, vp]),
@@ -307,6 +309,26 @@ class SpMM:
         _check(load_library().spmm_run_to(self._h, B.data_ptr(), K, arr, len(ptrs), int(row_offset),
                                           _stream_ptr(stream)))
         return dsts
+
+    def run_ld(self, B, C, col_offset=0, stream=None):
+        """spmm_run_ld: C[:, col_offset:col_offset + K] = A.B for a wider row-major C (cuda float32 [M, ldc]); the
+        other columns are untouched (column blocks of C, e.g. chunks of a B that arrives in pieces)."""
+        _check_dense(B, "B", self.N)
+        K = int(B.shape[1])
+        _check_dense(C, "C", self.M)
+        ldc = int(C.shape[1])
+        _need(0 <= int(col_offset) and int(col_offset) + K <= ldc, "column block outside C")
+        _check(load_library().spmm_run_ld(self._h, B.data_ptr(), K, C.data_ptr() + 4 * int(col_offset), ldc,
+                                          _stream_ptr(stream)))
+        return C
+
+    def run_multicast(self, B, C_mc, row_offset=0, stream=None):
+        """spmm_run_multicast: this handle's C rows stored once through an NVLS multicast address (int: e.g. torch
+        symmetric memory's multicast_ptr) at rows row_offset + r of the group-wide buffer."""
+        _check_dense(B, "B", self.N)
+        _need(isinstance(C_mc, int) and C_mc != 0, "C_mc must be a (nonzero) multicast device address")
+        _check(load_library().spmm_run_multicast(self._h, B.data_ptr(), int(B.shape[1]), C_mc, int(row_offset),
+                                                 _stream_ptr(stream)))
 
     def run_host(self, B_host, C_host, stream=None):
         """End-to-end: host B -> device, SpMM, device -> host C (host buffers, ideally pinned)."""

@@ -330,7 +330,7 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
     SPMM_TRY(check_run_args(h, B, K, C, true));
     SPMM_TRY(check_device(h));
     try {
-        return launch_spmm(h, B, K, C, (cudaStream_t)cuda_stream, &g_last_launches, CExtra{});
+        return launch_spmm(h, B, K, C, K, (cudaStream_t)cuda_stream, &g_last_launches, CExtra{});
     } catch (const std::exception &e) {
         return fail(SPMM_ERR_OOM, e.what());
     }
@@ -367,7 +367,41 @@ spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *
     cx.n = n_dsts - 1;
     for (int32_t i = 1; i < n_dsts; ++i) cx.p[i - 1] = reinterpret_cast<float4 *>(C_dsts[i] + row_offset * K);
     try {
-        return launch_spmm(h, B, K, C_dsts[0] + row_offset * K, (cudaStream_t)cuda_stream, &g_last_launches, cx);
+        return launch_spmm(h, B, K, C_dsts[0] + row_offset * K, K, (cudaStream_t)cuda_stream, &g_last_launches, cx);
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
+}
+
+spmm_status spmm_run_ld(spmm_handle h, const float *B, int64_t K, float *C, int64_t ldc, void *cuda_stream) {
+    g_last_launches = 0;
+    SPMM_TRY(check_run_args(h, B, K, C, true));
+    if (ldc < K || ldc % 4 != 0) return fail(SPMM_ERR_UNSUPPORTED, "ldc must be >= K and a multiple of 4");
+    SPMM_TRY(check_device(h));
+    try {
+        return launch_spmm(h, B, K, C, ldc, (cudaStream_t)cuda_stream, &g_last_launches, CExtra{});
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
+}
+
+spmm_status spmm_run_multicast(spmm_handle h, const float *B, int64_t K, float *C_mc, int64_t row_offset,
+                               void *cuda_stream) {
+    g_last_launches = 0;
+    if (!h || !C_mc) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    if (row_offset < 0) return fail(SPMM_ERR_INVALID_ARG, "negative row_offset");
+    SPMM_TRY(check_run_args(h, B, K, C_mc, true));
+    float *dst = C_mc + row_offset * K;
+    if (K % 8 != 0 || (((uintptr_t)B | (uintptr_t)dst) & 31u))
+        return fail(SPMM_ERR_UNSUPPORTED, "multicast stores need K % 8 == 0 and 32-byte aligned B and C rows");
+    SPMM_TRY(check_device(h));
+    CExtra cx{};
+    cx.n = 1;
+    cx.p[0] = reinterpret_cast<float4 *>(dst);
+    cx.mc = 1u;
+    cx.skip_main = 1;     // the multicast store also reaches this GPU's buffer: no second local store
+    try {
+        return launch_spmm(h, B, K, dst, K, (cudaStream_t)cuda_stream, &g_last_launches, cx);
     } catch (const std::exception &e) {
         return fail(SPMM_ERR_OOM, e.what());
     }
@@ -382,7 +416,7 @@ spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *
     if (h->stage_B.bytes < bB) SPMM_TRY(h->stage_B.alloc(bB, s));
     if (h->stage_C.bytes < bC) SPMM_TRY(h->stage_C.alloc(bC, s));
     if (bB) SPMM_CUDA(cudaMemcpyAsync(h->stage_B.p, B_host, bB, cudaMemcpyHostToDevice, s));
-    SPMM_TRY(launch_spmm(h, h->stage_B.as<float>(), K, h->stage_C.as<float>(), s, &g_last_launches, CExtra{}));
+    SPMM_TRY(launch_spmm(h, h->stage_B.as<float>(), K, h->stage_C.as<float>(), K, s, &g_last_launches, CExtra{}));
     if (bC) SPMM_CUDA(cudaMemcpyAsync(C_host, h->stage_C.p, bC, cudaMemcpyDeviceToHost, s));
     SPMM_CUDA(cudaStreamSynchronize(s));
     return SPMM_OK;
@@ -428,7 +462,7 @@ spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_
         SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_in[k], 0));
         if (i >= 2) SPMM_CUDA(cudaStreamWaitEvent(s, h->ev_out[k], 0));
         int32_t l = 0;
-        SPMM_TRY(launch_spmm(h, Bs, K, Cs, s, &l, CExtra{}));
+        SPMM_TRY(launch_spmm(h, Bs, K, Cs, K, s, &l, CExtra{}));
         launches += l;
         SPMM_CUDA(cudaEventRecord(h->ev_comp[k], s));
         // D2H of C_i (overlaps the H2D of B_{i+1}: PCIe is full duplex)

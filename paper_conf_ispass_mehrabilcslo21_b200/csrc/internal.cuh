@@ -123,6 +123,8 @@ constexpr int SPMM_MAX_CDST = 8;
 struct CExtra {
     float4 *p[SPMM_MAX_CDST - 1];
     int32_t n;
+    uint32_t mc;          // bit i: p[i] is an NVLS multicast address (stores through multimem.st)
+    int32_t skip_main;    // 1: the main C pointer is not written (every row goes to p[0..n-1] only)
 };
 
 struct spmm_ctx {
@@ -185,8 +187,8 @@ spmm_status prepare_schedule(spmm_ctx *h, int64_t K, const float *B, const float
 spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params &p, double out[24],
                              cudaStream_t s);
 spmm_status compute_features_b200(spmm_ctx *h, bool current_order, int64_t K, double out[7], cudaStream_t s);
-spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches,
-                        const CExtra &cx);
+spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_t ldc, cudaStream_t s,
+                        int32_t *launches, const CExtra &cx);
 void release_run_slots(spmm_ctx *h);   // waits for the slots' last runs, frees their scratch and streams
 
 // signatures of the rows (sorted unique col/bw), used by chains and features

@@ -67,6 +67,22 @@ __device__ __forceinline__ void vstore_cs(float8 *p, const float8 &v) {
                  "f"(v.lo.z), "f"(v.lo.w), "f"(v.hi.x), "f"(v.hi.y), "f"(v.hi.z), "f"(v.hi.w) : "memory");
 }
 __device__ __forceinline__ void vstore(float4 *p, const float4 &v) { *p = v; }
+// NVLS multicast store (SURVEY §8(f) f2 ii): p is a multicast address -- one store reaches the buffer on every
+// member GPU through the NVSwitch (multimem.st, at most 128 bits per instruction)
+__device__ __forceinline__ void mcstore(float4 *p, const float4 &v) {
+    asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z),
+                 "f"(v.w) : "memory");
+}
+__device__ __forceinline__ void mcstore(float8 *p, const float8 &v) {
+    mcstore(reinterpret_cast<float4 *>(p), v.lo);
+    mcstore(reinterpret_cast<float4 *>(p) + 1, v.hi);
+}
+// a store to extra destination i of spmm_run_to (mc bit i: a multicast address)
+template <class VT>
+__device__ __forceinline__ void xstore(VT *p, const VT &v, bool mc) {
+    if (mc) mcstore(p, v);
+    else vstore_cs(p, v);
+}
 __device__ __forceinline__ void vstore(float8 *p, const float8 &v) {
     asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(v.lo.x), "f"(v.lo.y),
                  "f"(v.lo.z), "f"(v.lo.w), "f"(v.hi.x), "f"(v.hi.y), "f"(v.hi.z), "f"(v.hi.w) : "memory");
@@ -98,8 +114,8 @@ __device__ __forceinline__ int2 ld_cv(const int2 *ptr) { return __ldg(ptr); }
 template <int V, int G, int U, class VT, bool MD = false>
 __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int gl, const int col0, const bool (&colok)[V],
                                           const int2 *__restrict__ cv, const VT *__restrict__ BV,
-                                          VT *__restrict__ CV, const int32_t KV, VT *__restrict__ PV,
-                                          const CExtra &cx) {
+                                          VT *__restrict__ CV, const int32_t KV, const int32_t LC,
+                                          VT *__restrict__ PV, const CExtra &cx) {
     constexpr int BATCH = (G >= 8 ? G : 8) >= U ? (G >= 8 ? G : 8) : U;   // (col, val) pairs per group per batch
     constexpr int PL = BATCH / G;                // pairs held per lane
     const int32_t start = u.x, len = u.y, dst = u.z;
@@ -163,17 +179,20 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
         for (int p = 0; p < PL; ++p) cur[p] = nxt[p];
     }
     if (dst >= 0) {                                    // a whole row: C[perm[p]] (+ the extra destinations)
+        if (!MD || !cx.skip_main) {
 #pragma unroll
-        for (int v = 0; v < V; ++v)
-            if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[v]);
+            for (int v = 0; v < V; ++v)
+                if (colok[v]) vstore_cs(CV + (size_t)dst * LC + col0 + v * G, acc[v]);
+        }
         if constexpr (MD) {   // spmm_run_to instantiations only: no cost for plain runs
 #pragma unroll
             for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in parameter space
                 if (i >= cx.n) break;
                 VT *X = reinterpret_cast<VT *>(cx.p[i]);
+                const bool mc = (cx.mc >> i) & 1u;
 #pragma unroll
                 for (int v = 0; v < V; ++v)
-                    if (colok[v]) vstore_cs(X + (size_t)dst * KV + col0 + v * G, acc[v]);
+                    if (colok[v]) xstore(X + (size_t)dst * LC + col0 + v * G, acc[v], mc);
             }
         }
     } else if (dst != NOSTORE) {                       // chunk group of a long row (warp-uniform)
@@ -214,7 +233,8 @@ template <int V, int G, int R, int U, class VT, bool MD = false>
 __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const int gl, const int col0,
                                                 const bool (&colok)[V], const RecT<R> *__restrict__ recs,
                                                 const int32_t *__restrict__ gdst, const VT *__restrict__ BV,
-                                                VT *__restrict__ CV, const int32_t KV, const CExtra &cx) {
+                                                VT *__restrict__ CV, const int32_t KV, const int32_t LC,
+                                                const CExtra &cx) {
     constexpr int BATCH = G >= 8 ? G : 8;        // records per group per batch
     constexpr int PL = BATCH / G;                // records held per lane
     const int32_t start = u.x, len = u.y, gid = u.z;
@@ -281,17 +301,20 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
         for (int r = 0; r < R; ++r) {
             const int32_t dst = __ldg(gdst + (size_t)gid * R + r);
             if (dst >= 0) {
+                if (!MD || !cx.skip_main) {
 #pragma unroll
-                for (int v = 0; v < V; ++v)
-                    if (colok[v]) vstore_cs(CV + (size_t)dst * KV + col0 + v * G, acc[r][v]);
+                    for (int v = 0; v < V; ++v)
+                        if (colok[v]) vstore_cs(CV + (size_t)dst * LC + col0 + v * G, acc[r][v]);
+                }
                 if constexpr (MD) {   // spmm_run_to instantiations only: no cost for plain runs
 #pragma unroll
                     for (int i = 0; i < SPMM_MAX_CDST - 1; ++i) {   // constant indices: cx stays in param space
                         if (i >= cx.n) break;
                         VT *X = reinterpret_cast<VT *>(cx.p[i]);
+                        const bool mc = (cx.mc >> i) & 1u;
 #pragma unroll
                         for (int v = 0; v < V; ++v)
-                            if (colok[v]) vstore_cs(X + (size_t)dst * KV + col0 + v * G, acc[r][v]);
+                            if (colok[v]) xstore(X + (size_t)dst * LC + col0 + v * G, acc[r][v], mc);
                     }
                 }
             }
@@ -312,8 +335,8 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
 template <int V, int G, bool MASK, int W, int FR, bool MD>
 __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? 2 : 3) k_spmm(const int4 *__restrict__ units, int64_t n_tasks,
                                                        const int2 *__restrict__ cv, const float4 *__restrict__ B4,
-                                                       float4 *__restrict__ C4, int32_t K4, float4 *__restrict__ P4,
-                                                       unsigned int *__restrict__ counter,
+                                                       float4 *__restrict__ C4, int32_t K4, int32_t ldc4,
+                                                       float4 *__restrict__ P4, unsigned int *__restrict__ counter,
                                                        const int4 *__restrict__ recs,
                                                        const int32_t *__restrict__ gdst, const CExtra cx) {
     using VT = typename VecT<W>::T;
@@ -322,7 +345,7 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? 2 : 3) k_spmm(const int
     constexpr int U = V * W >= 12 ? 2 : 4;        // nnz per inner step (B loads in flight per lane: U*V)
     constexpr int FU = V == 1 ? 4 : 2;            // union records per inner step of a fused unit
     constexpr bool PF = FR > 1;
-    const int32_t KV = K4 * 4 / W;
+    const int32_t KV = K4 * 4 / W, LC = ldc4 * 4 / W;   // B row / C row strides in W-float vectors
     const int lane = threadIdx.x & 31;
     const int g = lane / G, gl = lane % G;
     const int col0 = blockIdx.y * CTV + gl;      // this lane's first vector column; then + v*G
@@ -377,10 +400,10 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? 2 : 3) k_spmm(const int
             spmm_unit_fused<V, G, (FR > 1 ? FR : 2), FU, VT, MD>(u, g, gl, col0, colok,
                                                      reinterpret_cast<const RecT<(FR > 1 ? FR : 2)> *>(recs), gdst,
                                                      reinterpret_cast<const VT *>(B4), reinterpret_cast<VT *>(C4), KV,
-                                                     cx);
+                                                     LC, cx);
         } else {
             spmm_unit<V, G, U, VT, MD>(u, g, gl, col0, colok, cv, reinterpret_cast<const VT *>(B4),
-                                       reinterpret_cast<VT *>(C4), KV, reinterpret_cast<VT *>(P4), cx);
+                                       reinterpret_cast<VT *>(C4), KV, LC, reinterpret_cast<VT *>(P4), cx);
         }
         t = t_next;
         u = u_next;
@@ -392,12 +415,12 @@ __global__ void __launch_bounds__(SPMM_THREADS, FR > 1 ? 2 : 3) k_spmm(const int
 // column of C.
 __global__ void __launch_bounds__(256) k_combine(const float4 *__restrict__ P4, const int32_t *__restrict__ pslot_ptr,
                                                  const int32_t *__restrict__ long_dst, int64_t n_long,
-                                                 float4 *__restrict__ C4, int32_t K4, const CExtra cx) {
+                                                 float4 *__restrict__ C4, int32_t K4, int32_t ldc4, const CExtra cx) {
     const int lane = threadIdx.x & 31;
     for (int64_t l = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; l < n_long;
          l += ((int64_t)gridDim.x * blockDim.x) >> 5) {
         const int32_t c0 = pslot_ptr[l], c1 = pslot_ptr[l + 1];
-        float4 *dst = C4 + (size_t)long_dst[l] * K4;
+        float4 *dst = C4 + (size_t)long_dst[l] * ldc4;
         for (int32_t col = lane; col < K4; col += 32) {
             float4 stk[24];
             int sp = 0;
@@ -414,24 +437,24 @@ __global__ void __launch_bounds__(256) k_combine(const float4 *__restrict__ P4, 
                 const float4 y = stk[--sp];
                 r = make_float4(y.x + r.x, y.y + r.y, y.z + r.z, y.w + r.w);
             }
-            __stcs(dst + col, r);
+            if (!cx.skip_main) __stcs(dst + col, r);
 #pragma unroll
             for (int i = 0; i < SPMM_MAX_CDST - 1; ++i)
-                if (i < cx.n) __stcs(cx.p[i] + (size_t)long_dst[l] * K4 + col, r);
+                if (i < cx.n) xstore(cx.p[i] + (size_t)long_dst[l] * ldc4 + col, r, (cx.mc >> i) & 1u);
         }
     }
 }
 
 // empty rows: zero-fill their C rows (thread per float4)
-__global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, float4 *__restrict__ C4,
-                            const CExtra cx) {
+__global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, int32_t ldc4,
+                            float4 *__restrict__ C4, const CExtra cx) {
     const int64_t total = n * K4;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-        const size_t o = (size_t)rows[i / K4] * K4 + (i % K4);
-        __stcs(C4 + o, make_float4(0.f, 0.f, 0.f, 0.f));
+        const size_t o = (size_t)rows[i / K4] * ldc4 + (i % K4);
+        if (!cx.skip_main) __stcs(C4 + o, make_float4(0.f, 0.f, 0.f, 0.f));
 #pragma unroll
         for (int j = 0; j < SPMM_MAX_CDST - 1; ++j)
-            if (j < cx.n) __stcs(cx.p[j] + o, make_float4(0.f, 0.f, 0.f, 0.f));
+            if (j < cx.n) xstore(cx.p[j] + o, make_float4(0.f, 0.f, 0.f, 0.f), (cx.mc >> j) & 1u);
     }
 }
 
@@ -777,7 +800,7 @@ spmm_status build_schedule(spmm_ctx *h, Schedule &S, int32_t rpw, int32_t R, cud
     return SPMM_OK;
 }
 
-using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, float4 *,
+using SpmmKernel = void (*)(const int4 *, int64_t, const int2 *, const float4 *, float4 *, int32_t, int32_t, float4 *,
                             unsigned int *, const int4 *, const int32_t *, const CExtra);
 
 // W = 4 (LDG.128) geometries: any power-of-two G <= 32, V in 1..4 (no extra-destination variants: spmm_run_to
@@ -870,8 +893,8 @@ Config choose(int32_t K4, bool w8ok) {
     return {pick_w4<4, true, false>(G), 4, G, (int)ceil_div(K4, 4 * G), 4};
 }
 
-Config choose_for(spmm_ctx *h, int64_t K, const float *B, const float *C, const CExtra &cx) {
-    uintptr_t align = (uintptr_t)B | (uintptr_t)C;
+Config choose_for(spmm_ctx *h, int64_t K, const float *B, const float *C, const CExtra &cx, int64_t ldc) {
+    uintptr_t align = (uintptr_t)B | (uintptr_t)C | (uintptr_t)(4 * ldc);   // C rows start at C + r * ldc
     for (int i = 0; i < cx.n; ++i) align |= (uintptr_t)cx.p[i];
     const bool w8ok = K % 8 == 0 && (align % 32) == 0;
     Config cfg = cx.n > 0 ? choose<true>((int32_t)(K / 4), w8ok) : choose<false>((int32_t)(K / 4), w8ok);
@@ -908,7 +931,7 @@ static spmm_status get_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_
 }
 
 spmm_status prepare_schedule(spmm_ctx *h, int64_t K, const float *B, const float *C, cudaStream_t s) {
-    const Config cfg = choose_for(h, K, B, C, CExtra{});
+    const Config cfg = choose_for(h, K, B, C, CExtra{}, K);
     std::lock_guard<std::mutex> lk(h->mu);
     int slot = 0;
     SPMM_TRY(get_schedule(h, 32 / cfg.G, cfg.R, s, &slot));
@@ -938,16 +961,19 @@ void release_run_slots(spmm_ctx *h) {
     }
 }
 
-spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaStream_t s, int32_t *launches,
-                        const CExtra &cx) {
+spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_t ldc, cudaStream_t s,
+                        int32_t *launches, const CExtra &cx) {
     *launches = 0;
     const int64_t M = h->M;
     if (M == 0) return SPMM_OK;
-    const int32_t K4 = (int32_t)(K / 4);
-    Config cfg = choose_for(h, K, B, C, cx);
+    const int32_t K4 = (int32_t)(K / 4), ldc4 = (int32_t)(ldc / 4);
+    Config cfg = choose_for(h, K, B, C, cx, ldc);   // (W = 8 needs 32-byte aligned rows: C and ldc)
     bool copy_extra = false;      // spmm_run_to on a geometry without a multi-destination kernel: copy afterwards
     if (cx.n > 0 && !(cfg.W == 8 && cfg.tiles == 1)) {
-        cfg = choose_for(h, K, B, C, CExtra{});
+        if (cx.mc || cx.skip_main || ldc != K)
+            return fail(SPMM_ERR_UNSUPPORTED, "multicast / strided extra destinations need K % 8 == 0 and 32-byte "
+                                              "aligned B and C rows");
+        cfg = choose_for(h, K, B, C, CExtra{}, ldc);
         copy_extra = true;
     }
     const int32_t rpw = 32 / cfg.G;
@@ -983,7 +1009,7 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     if (S.n_empty > 0) {
         SPMM_CUDA(cudaEventRecord(rs->fork, s));
         SPMM_CUDA(cudaStreamWaitEvent(rs->side, rs->fork, 0));
-        k_zero_rows<<<(unsigned)h->num_sms, 128, 0, rs->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, C4,
+        k_zero_rows<<<(unsigned)h->num_sms, 128, 0, rs->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, ldc4, C4,
                                                                 copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
         SPMM_CUDA(cudaEventRecord(rs->join, rs->side));
@@ -1002,7 +1028,7 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
         SPMM_CUDA(cudaMemsetAsync(rs->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
         if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
-                                           reinterpret_cast<const float4 *>(B), C4, K4, P4,
+                                           reinterpret_cast<const float4 *>(B), C4, K4, ldc4, P4,
                                            rs->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>(),
                                            copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
@@ -1014,7 +1040,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, cudaSt
     }
     if (S.n_long > 0) {
         k_combine<<<(unsigned)std::min<int64_t>(ceil_div(S.n_long, 8), 148 * 64), 256, 0, s>>>(
-            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, copy_extra ? CExtra{} : cx);
+            P4, S.pslot_ptr.as<int32_t>(), S.long_dst.as<int32_t>(), S.n_long, C4, K4, ldc4,
+            copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
         ++*launches;
     }

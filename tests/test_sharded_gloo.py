@@ -21,7 +21,8 @@ class OracleLocal:
     """CPU stand-in for the per-rank CUDA SpMM (tests only)."""
 
     def __init__(self, shard):
-        self.csr = syn.CSR(shard.M, shard.N, shard.rowidx, shard.colidx, shard.value)
+        self.csr = syn.CSR(shard.M, shard.N, np.asarray(shard.rowidx), np.asarray(shard.colidx),
+                           np.asarray(shard.value))
         self.policy = "identity"
 
     def permute(self, policy, **kw):
@@ -31,6 +32,11 @@ class OracleLocal:
     def run(self, B, C=None):
         out, _ = oracle.spmm(self.csr, B.numpy())
         return torch.from_numpy(out.astype(np.float32))
+
+    def run_ld(self, B, C, col_offset=0):
+        """spmm_run_ld semantics: C[:, col_offset:col_offset + K] = A.B, other columns untouched."""
+        C[:, col_offset:col_offset + B.shape[1]] = self.run(B)
+        return C
 
     def run_to(self, B, dsts, row_offset=0, stream=None):
         """spmm_run_to semantics: this shard's rows stored into every destination at row_offset + r."""
@@ -48,28 +54,48 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, K, results, compact=False):
+def _init(rank, world, port):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
+
+
+def _worker(rank, world, port, K, results, compact, how):
+    _init(rank, world, port)
     try:
         from paper_conf_ispass_mehrabilcslo21_b200.sharded import ShardedSpMM
         a = syn.rmat(10, 8, 99, "natural", int_values=True)
-        sh = ShardedSpMM(a.M, a.N, a.rowidx, a.colidx, a.value, local_factory=OracleLocal, compact_B=compact)
+        if how == "scatter":      # rank 0 alone holds the matrix
+            sh = ShardedSpMM.scatter(a if rank == 0 else None, src=0, compact_B=compact, local_factory=OracleLocal)
+        else:
+            sh = ShardedSpMM.from_full(a.M, a.N, a.rowidx, a.colidx, a.value, local_factory=OracleLocal,
+                                       compact_B=compact)
+        assert (sh.M, sh.N) == (a.M, a.N)
         sh.permute("nnz_sort")
-        B = torch.from_numpy(syn.dense(a.N, K, 5, int_values=True)) if rank == 0 else torch.zeros((a.N, K))
+        Bfull = syn.dense(a.N, K, 5, int_values=True)
+        B = torch.from_numpy(Bfull) if rank == 0 else torch.zeros((a.N, K))
+        ref, _ = oracle.spmm(a, Bfull)
+        lo, hi = sh.shard.lo, sh.shard.hi
+        # the shard is exactly this rank's rows (columns through cols_p when compact)
+        r0 = a.rowidx[lo]
+        cc = np.asarray(sh.shard.colidx)
+        ok_shard = (np.array_equal(np.asarray(sh.shard.rowidx), a.rowidx[lo:hi + 1] - r0)
+                    and np.array_equal(np.asarray(sh.cols)[cc] if compact else cc, a.colidx[r0:r0 + len(cc)]))
         if compact:
             Bl = sh.distribute_B(B if rank == 0 else None, K=K, src=0)
             assert Bl.shape == (sh.shard.N, K) and sh.shard.N < a.N
-            # the compact rows are exactly B[cols_p] and the shard's columns index them
-            assert np.array_equal(Bl.numpy(), syn.dense(a.N, K, 5, int_values=True)[sh.cols])
-            assert int(sh.shard.colidx.max()) < sh.shard.N
+            assert np.array_equal(Bl.numpy(), Bfull[np.asarray(sh.cols)])
+            assert int(cc.max()) < sh.shard.N
             C_local = sh.run(Bl)
+            # f2 (iii): B in column chunks, each chunk's SpMM into its C columns as it arrives
+            for chunks in (1, 3, 4):
+                Cp = torch.full((sh.shard.M, K), float("nan"))
+                sh.run_pipelined(B if rank == 0 else None, K=K, chunks=chunks, C_local=Cp, src=0)
+                assert torch.equal(Cp, C_local), chunks
         else:
             sh.broadcast_B(B, src=0)
             C_local = sh.run(B)
         C = sh.allgather_C(C_local)
-        ref, _ = oracle.spmm(a, syn.dense(a.N, K, 5, int_values=True))
         if not compact:
             # fused all-gather (f2 ii): each rank stores its rows into "every rank's" full-C buffer at its row
             # offset; here the peers' buffers are local stand-ins, so the disjoint writes are summed over ranks
@@ -78,62 +104,42 @@ def _worker(rank, world, port, K, results, compact=False):
             for b in bufs:
                 dist.all_reduce(b)
                 assert np.array_equal(b.numpy().astype(np.float64), ref)
-        nnz_local = sh.shard.nnz
-        results[rank] = (bool(np.array_equal(C.numpy().astype(np.float64), ref)), nnz_local, a.nnz,
-                         int(np.diff(a.rowidx).max()), sh.shard.lo, sh.shard.hi)
+        results[rank] = (bool(np.array_equal(C.numpy().astype(np.float64), ref)) and ok_shard, sh.shard.nnz, a.nnz,
+                         int(np.diff(a.rowidx).max()), lo, hi)
     finally:
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("how", ["scatter", "full"])
 @pytest.mark.parametrize("compact", [False, True])
-@pytest.mark.parametrize("world", [2, 3])
-def test_sharded_gloo(world, compact):
-    """Partition, shard slicing, B exchange (broadcast, or per-rank compact B rows: SURVEY.md §8(f) f2(i)),
-    local SpMM and the C all-gather reassemble the oracle's C exactly (integer-valued inputs)."""
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_sharded_gloo(world, compact, how):
+    """Partition, shard scatter from rank 0 (or local slicing when every rank holds A), B exchange (broadcast, or
+    per-rank compact B rows: SURVEY.md §8(f) f2(i)), the column-chunk pipeline (f2 iii), local SpMM and the C
+    all-gather reassemble the oracle's C exactly (integer-valued inputs)."""
     mgr = mp.Manager()
     results = mgr.dict()
     port = _free_port()
-    mp.spawn(_worker, args=(world, port, 8, results, compact), nprocs=world, join=True)
+    mp.spawn(_worker, args=(world, port, 24, results, compact, how), nprocs=world, join=True)
     assert len(results) == world
     lo_hi = sorted((results[r][4], results[r][5]) for r in range(world))
     assert lo_hi[0][0] == 0 and all(lo_hi[i][1] == lo_hi[i + 1][0] for i in range(world - 1))
     for r in range(world):
         ok, nnz_local, nnz, maxrow, _, _ = results[r]
-        assert ok, f"rank {r}: reassembled C differs from the oracle"
+        assert ok, f"rank {r}: shard or reassembled C differs from the oracle"
         assert nnz_local <= -(-nnz // world) + maxrow
 
 
-def _bench_worker(rank, world, port, compact, results):
-    """bench.py's own N>1 input path (rank 0 generates, shards by nnz, optionally compacts the columns) on gloo/CPU."""
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
-    try:
-        import bench
-        import paper_conf_ispass_mehrabilcslo21_b200 as pkg
-        a = syn.rmat(10, 8, 98, "local", int_values=True)
-        Mr, lo, (r, c, v), meta, cols, _ = bench.shard_inputs(torch, dist, a if rank == 0 else None, world, rank,
-                                                               torch.device("cpu"), pkg, compact=compact)
-        r, c, v = r.numpy(), c.numpy(), v.numpy()
-        orig_c = cols.numpy()[c] if compact else c
-        r0 = a.rowidx[lo]
-        ok = (np.array_equal(r, a.rowidx[lo:lo + Mr + 1] - r0) and np.array_equal(orig_c, a.colidx[r0:r0 + len(c)])
-              and np.array_equal(v, a.value[r0:r0 + len(v)]))
-        if compact:
-            ok = ok and np.array_equal(cols.numpy(), np.unique(a.colidx[r0:r0 + len(c)])) and int(meta[rank, 3]) == len(cols)
-        results[rank] = (bool(ok), int(Mr), int(a.M))
-    finally:
-        dist.destroy_process_group()
-
-
-@pytest.mark.parametrize("compact", [False, True])
-def test_bench_shard_inputs_gloo(compact):
-    """bench.py --gpus 2 input distribution: shards cover the rows exactly; compact shards index B[cols]."""
-    mgr = mp.Manager()
-    results = mgr.dict()
-    mp.spawn(_bench_worker, args=(2, _free_port(), compact, results), nprocs=2, join=True)
-    assert all(results[r][0] for r in range(2)), dict(results)
-    assert results[0][1] + results[1][1] == results[0][2]
+def test_chunk_bounds():
+    from paper_conf_ispass_mehrabilcslo21_b200.sharded import chunk_bounds
+    assert chunk_bounds(128, 4) == [(0, 32), (32, 64), (64, 96), (96, 128)]
+    assert chunk_bounds(24, 3) == [(0, 8), (8, 16), (16, 24)]
+    assert chunk_bounds(64, 1) == [(0, 64)]
+    for K in (8, 24, 64, 72, 128, 256):
+        for c in (1, 2, 3, 4, 5, 16):
+            cb = chunk_bounds(K, c)
+            assert cb[0][0] == 0 and cb[-1][1] == K and all(x[1] == y[0] for x, y in zip(cb, cb[1:]))
+            assert all(c0 % 8 == 0 for c0, _ in cb) and len(cb) <= c
 
 
 def test_bench_reference_arm_torchrun():

@@ -12,6 +12,7 @@ _lib = None
 
 
 _PROBE = os.path.join(_HERE, "libl2probe.so")
+_LDPATH = os.path.join(_HERE, "libldpath.so")
 
 
 def build():
@@ -22,6 +23,10 @@ def build():
     if not os.path.exists(_PROBE) or os.path.getmtime(_PROBE) < os.path.getmtime(psrc):
         subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
                                "-shared", "-Xcompiler", "-fPIC", psrc, "-o", _PROBE])
+    lsrc = os.path.join(_HERE, "ldpathprobe.cu")
+    if not os.path.exists(_LDPATH) or os.path.getmtime(_LDPATH) < os.path.getmtime(lsrc):
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
+                               "-DLDPATH_NO_MAIN", "-shared", "-Xcompiler", "-fPIC", lsrc, "-o", _LDPATH])
     csrc = os.path.join(_HERE, "cusparse_ref.cu")
     if not os.path.exists(_CUSP) or os.path.getmtime(_CUSP) < os.path.getmtime(csrc):
         subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2",
@@ -82,3 +87,16 @@ def l2_read_bandwidth_sms(limit, bytes_=64 << 20, reps=20):
     lib.l2probe_read_bw_sms.restype = ctypes.c_double
     lib.l2probe_read_bw_sms.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_int]
     return float(lib.l2probe_read_bw_sms(int(bytes_), int(reps), int(limit)))
+
+
+def ldpath_gather(shape=0, window=16 << 20, row_bytes=512, reps=5):
+    """SM load-path gather ceiling (tools/ldpathprobe.cu): random rows of row_bytes gathered from a window of
+    `window` bytes with k_spmm's load shape (shape 0: 8-lane groups x one 256-bit load per lane).  16 MiB window =
+    L2-resident, 32 KiB = L1-resident.  Returns (GB/s, bytes per SM clock)."""
+    build()
+    lib = ctypes.CDLL(_LDPATH)
+    lib.ldpath_gather.restype = ctypes.c_double
+    lib.ldpath_gather.argtypes = [ctypes.c_int, ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_void_p]
+    bpc = ctypes.c_double(0.0)
+    gbs = float(lib.ldpath_gather(int(shape), int(window), int(row_bytes), int(reps), ctypes.byref(bpc)))
+    return gbs, float(bpc.value)

@@ -117,6 +117,57 @@ __global__ void __launch_bounds__(256, 1) k_probe_smem(const char *__restrict__ 
     if (threadIdx.x == 0) atomicMax(cyc + blockIdx.x % 1024, (unsigned long long)(t1 - t0));
 }
 
+// Library entry (tools/__init__.py ldpath_gather): best of `reps` launches of one shape over one window;
+// returns GB/s (-1 on error) and the bytes per SM clock in *bpc.
+extern "C" double ldpath_gather(int shape, int64_t window, int RB, int reps, double *bpc) {
+    int sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    char *B = nullptr;
+    float *out = nullptr;
+    unsigned long long *cyc = nullptr;
+    if (cudaMalloc(&B, (size_t)window) != cudaSuccess) return -1.0;
+    cudaMemset(B, 0, (size_t)window);
+    cudaMalloc(&out, (size_t)sms * 3 * 256 * sizeof(float));
+    cudaMalloc(&cyc, 1024 * sizeof(unsigned long long));
+    const uint32_t nrows = (uint32_t)(window / RB);
+    const int blocks = sms * 3, iters = 512;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    double best = -1.0, best_bpc = 0.0;
+    for (int rep = 0; rep < reps; ++rep) {
+        cudaMemset(cyc, 0, 1024 * sizeof(unsigned long long));
+        cudaEventRecord(e0);
+        switch (shape) {
+            case 0: k_probe<0><<<blocks, 256>>>(B, nrows, RB, iters, out, cyc); break;
+            case 3: k_probe<3><<<blocks, 256>>>(B, nrows, RB, iters, out, cyc); break;
+            default: k_probe<1><<<blocks, 256>>>(B, nrows, RB, iters, out, cyc); break;
+        }
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        unsigned long long hc[1024];
+        cudaMemcpy(hc, cyc, sizeof(hc), cudaMemcpyDeviceToHost);
+        unsigned long long mc = 1;
+        for (int i = 0; i < 1024; ++i) mc = hc[i] > mc ? hc[i] : mc;
+        const double per_instr = (shape == 0 || shape == 3) ? 1024.0 : 512.0;
+        const double bytes = (double)blocks * 8 * iters * U * per_instr;
+        const double gbs = bytes / (ms * 1e-3) / 1e9;
+        if (gbs > best) { best = gbs; best_bpc = bytes / sms / (double)mc; }
+    }
+    if (cudaGetLastError() != cudaSuccess) best = -1.0;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(B);
+    cudaFree(out);
+    cudaFree(cyc);
+    if (bpc) *bpc = best_bpc;
+    return best;
+}
+
+#ifndef LDPATH_NO_MAIN
 int main(int argc, char **argv) {
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
@@ -179,3 +230,4 @@ int main(int argc, char **argv) {
     printf("\n]}\n");
     return 0;
 }
+#endif
