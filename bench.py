@@ -262,7 +262,7 @@ def timed_max(torch, dist, world, fn, reps, stream):
     return float(t.item())
 
 
-def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps=5, chunks=4):
+def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps=5, chunks=None):
     """N>1: the data-path communication of the sharded mode, timed on the device (max over
     ranks) and reported in GB/s of bytes moved between GPUs:
       b_exchange   -- per-rank B rows (distribute_B) or the broadcast of all of B;
@@ -317,7 +317,7 @@ def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps
         t_pipe = timed_max(torch, dist, world, lambda: sh.run_pipelined(Bfull, K=K, chunks=chunks, C_local=Cp,
                                                                          src=0, device=Bd.device), reps, stream)
         torch.cuda.synchronize()
-        out["pipelined"] = {"ms": t_pipe, "sequential_ms": t_seq, "chunks": chunks,
+        out["pipelined"] = {"ms": t_pipe, "sequential_ms": t_seq, "chunks": chunks or max(1, K // 64),
                             "bit_identical_to_run": bool(torch.equal(Cp.view(torch.int32), Cd.view(torch.int32)))}
     return out
 

@@ -247,17 +247,20 @@ class ShardedSpMM:
         """Local SpMM on this rank's row shard (B resident on every rank). Returns the C shard."""
         return self.local.run(B, C_local)
 
-    def run_pipelined(self, B=None, K=None, chunks: int = 4, C_local=None, src: int = 0, device=None):
+    def run_pipelined(self, B=None, K=None, chunks=None, C_local=None, src: int = 0, device=None):
         """f2 (iii): the compact B exchange and the SpMM pipelined over column chunks of B.  `src` sends each rank
         B[cols_p][:, c0:c1] chunk by chunk (all sends posted at once); a rank runs the SpMM of chunk c (spmm_run_ld
         into C_local[:, c0:c1]) as soon as chunk c has arrived -- under NCCL the wait is a stream dependency, so the
-        SpMM of chunk c overlaps the transfer of chunk c + 1.  Returns this rank's C shard [M_p, K]."""
+        SpMM of chunk c overlaps the transfer of chunk c + 1.  Returns this rank's C shard [M_p, K].
+        chunks=None: K // 64 chunks of 64 columns -- the lane geometry of K = 64 has the rows per warp task of
+        K = 128 / 256, so split rows are cut into the same chunks and C is bit-identical to spmm_run's; other chunk
+        widths change the split-row summation order (C within the north-star tolerance)."""
         import torch
         assert self.compact_B, "run_pipelined needs compact_B=True"
         if self.rank == src:
             K = int(B.shape[1])
         K = int(K)
-        cb = chunk_bounds(K, chunks)
+        cb = chunk_bounds(K, chunks if chunks is not None else max(1, K // 64))
         if C_local is None:
             C_local = torch.empty((self.shard.M, K), dtype=torch.float32,
                                   device=device if device is not None else (B.device if B is not None else None))

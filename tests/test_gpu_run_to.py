@@ -117,9 +117,9 @@ def test_run_allgather_fused_symmetric_memory():
         K = 64
         Bn = syn.dense(a.N, K, 3111)
         B = torch.from_numpy(Bn).cuda()
-        sh = ShardedSpMM(a.M, a.N, a.rowidx, a.colidx, a.value)
+        sh = ShardedSpMM.scatter(a, src=0, compact_B=False)     # NCCL group of one: the shard is all of A
         sh.permute("cta_aware")
-        buf, ptrs, _hdl = sh.symmetric_C(K)
+        buf, ptrs, hdl = sh.symmetric_C(K)
         assert len(ptrs) == 1
         buf.fill_(float("nan"))
         sh.run_allgather_fused(B, ptrs)
@@ -129,6 +129,70 @@ def test_run_allgather_fused_symmetric_memory():
         C_ref, bound = oracle.spmm(a, Bn)
         err = np.abs(buf.cpu().numpy().astype(np.float64) - C_ref)
         assert np.all(err <= 1e-5 * bound + 1e-6)
+        mc = int(getattr(hdl, "multicast_ptr", 0) or 0)
+        if mc:    # NVLS multicast store path, where the rendezvous provides one
+            buf.fill_(float("nan"))
+            torch.cuda.synchronize()
+            sh.run_allgather_multicast(B, mc)
+            torch.cuda.synchronize()
+            assert torch.equal(buf.view(torch.int32), ref.view(torch.int32))
         sh.close()
+        # the compact exchange + column-chunk pipeline on an NCCL group of one (the source's own chunks)
+        shc = ShardedSpMM.scatter(a, src=0, compact_B=True)
+        shc.permute("cta_aware")
+        Bl = shc.distribute_B(B, src=0)
+        refc = shc.run(Bl)
+        assert torch.equal(refc.view(torch.int32), ref.view(torch.int32))
+        Cp = shc.run_pipelined(B, src=0)              # default: 64-column chunks (here one)
+        torch.cuda.synchronize()
+        assert torch.equal(Cp.view(torch.int32), ref.view(torch.int32))
+        Cp = shc.run_pipelined(B, chunks=4, src=0)    # 16-column chunks: another lane geometry, same tolerance
+        torch.cuda.synchronize()
+        assert np.all(np.abs(Cp.cpu().numpy().astype(np.float64) - C_ref) <= 1e-5 * bound + 1e-6)
+        shc.close()
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_run_ld_column_blocks(name):
+    """spmm_run_ld (f2 iii's building block): column chunks of B computed into the matching columns of a wider C
+    reassemble the full-width spmm_run result bit for bit; columns outside a block stay untouched."""
+    gen, K, pol = CASES[name]
+    a = gen()
+    h = pkg.SpMM.from_csr(a)
+    h.permute(pol)
+    B = torch.from_numpy(syn.dense(a.N, K, 3300)).cuda()
+    ref = h.run(B)
+    from paper_conf_ispass_mehrabilcslo21_b200.sharded import chunk_bounds
+    C_ref, bound = oracle.spmm(a, B.cpu().numpy())
+    for chunks in (2, 3):
+        C = torch.full((a.M, K), float("nan"), device="cuda")
+        cb = chunk_bounds(K, chunks, align=4 if K % 8 else 8)
+        for c0, c1 in cb:
+            h.run_ld(B[:, c0:c1].contiguous(), C, col_offset=c0)
+            torch.cuda.synchronize()
+            assert torch.isnan(C[:, c1:]).all()            # later columns not written yet
+        assert np.all(np.abs(C.cpu().numpy().astype(np.float64) - C_ref) <= 1e-5 * bound + 1e-6), (name, chunks)
+        # bit-identical whenever the split rows are cut the same way: no split rows, or 64-column chunks of K = 128
+        if h.info()["split_rows"] == 0 or all(c1 - c0 == 64 for c0, c1 in cb):
+            assert torch.equal(C.view(torch.int32), ref.view(torch.int32)), (name, chunks)
+    h.close()
+
+
+def test_run_multicast_arguments():
+    """spmm_run_multicast needs a multicast address, K % 8 == 0 and 32-byte aligned rows (the NVLS store path itself
+    needs a multi-GPU multicast group: unmeasured on one GPU)."""
+    a = syn.rmat(10, 8, 3400, "natural")
+    h = pkg.SpMM.from_csr(a)
+    B = torch.from_numpy(syn.dense(a.N, 64, 3401)).cuda()
+    with pytest.raises(ValueError):
+        h.run_multicast(B, 0)
+    lib = pkg.load_library()
+    C = torch.empty((a.M, 64), device="cuda")
+    assert lib.spmm_run_multicast(h._h, B.data_ptr(), 64, None, 0, None) == 1            # NULL -> INVALID_ARG
+    assert lib.spmm_run_multicast(h._h, B.data_ptr(), 64, C.data_ptr(), -1, None) == 1   # negative row offset
+    B36 = torch.from_numpy(syn.dense(a.N, 36, 3402)).cuda()
+    assert lib.spmm_run_multicast(h._h, B36.data_ptr(), 36, C.data_ptr(), 0, None) == 3  # K % 8 -> UNSUPPORTED
+    assert lib.spmm_run_multicast(h._h, B.data_ptr(), 64, C.data_ptr() + 16, 0, None) == 3   # misaligned rows
+    h.close()
