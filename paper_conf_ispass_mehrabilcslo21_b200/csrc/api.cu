@@ -1,6 +1,7 @@
 // api.cu -- the C ABI of include/spmm.h: argument checking, CSR ingest + validation (a1), handle
 // lifetime, dispatch to the permutation builders, the SpMM launch, features and the predictor.
 #include "internal.cuh"
+#include <nvtx3/nvToolsExt.h>
 #include <algorithm>
 #include <cmath>
 #include <cstring>
@@ -10,6 +11,13 @@
 #include <vector>
 
 namespace spmm {
+
+// NVTX range per C-ABI call (SURVEY §5 tracing: phases show up by name in nsys / ncu timelines; a no-op without a
+// tool attached -- NVTX v3 is header-only and binds to an injection library only when one is loaded)
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 static thread_local std::string g_last_error;
 static thread_local int32_t g_last_launches = 0;
@@ -197,6 +205,7 @@ spmm_status spmm_set_allocator(void *(*alloc)(size_t, void *, void *), void (*fr
 
 spmm_status spmm_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, const int64_t *rowidx,
                         const int32_t *colidx, const float *value, int inputs_on_device, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_create");
     try {
         return do_create(out, M, N, nnz, rowidx, colidx, value, inputs_on_device, (cudaStream_t)cuda_stream);
     } catch (const std::exception &e) {
@@ -205,6 +214,7 @@ spmm_status spmm_create(spmm_handle *out, int64_t M, int64_t N, int64_t nnz, con
 }
 
 spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *params, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_permute");
     if (!h) return fail(SPMM_ERR_INVALID_ARG, "handle is NULL");
     if ((int)policy < 0 || (int)policy >= SPMM_POLICY_COUNT) return fail(SPMM_ERR_INVALID_ARG, "unknown policy");
     SPMM_TRY(check_device(h));
@@ -238,6 +248,7 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
 }
 
 spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out) {
+    NvtxRange nvtx_("spmm_get_perm");
     if (!h || (!perm_out && h->M > 0)) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     SPMM_TRY(check_device(h));
     if (h->M == 0) return SPMM_OK;
@@ -249,6 +260,7 @@ spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out) {
 }
 
 spmm_status spmm_get_permuted_csr(spmm_handle h, int64_t *rowidx, int32_t *colidx, float *value) {
+    NvtxRange nvtx_("spmm_get_permuted_csr");
     if (!h || !rowidx || (h->nnz > 0 && (!colidx || !value))) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     SPMM_TRY(check_device(h));
     std::vector<int32_t> r32(h->M + 1);
@@ -293,6 +305,7 @@ spmm_status spmm_get_schedule_info(spmm_handle h, int64_t out[6]) {
 
 spmm_status spmm_features(spmm_handle h, int use_current_order, const spmm_params *params, double out[24],
                           void *cuda_stream) {
+    NvtxRange nvtx_("spmm_features");
     if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     SPMM_TRY(check_device(h));
     spmm_params p;
@@ -306,6 +319,7 @@ spmm_status spmm_features(spmm_handle h, int use_current_order, const spmm_param
 }
 
 spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, double out[7], void *cuda_stream) {
+    NvtxRange nvtx_("spmm_features_b200");
     if (!h || !out) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     if (K <= 0) return fail(SPMM_ERR_INVALID_ARG, "K must be positive");
     SPMM_TRY(check_device(h));
@@ -326,6 +340,7 @@ static spmm_status check_run_args(spmm_handle h, const void *B, int64_t K, const
 }
 
 spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run");
     g_last_launches = 0;
     SPMM_TRY(check_run_args(h, B, K, C, true));
     SPMM_TRY(check_device(h));
@@ -337,6 +352,7 @@ spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *c
 }
 
 spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *C, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_prepare");
     if (!h) return fail(SPMM_ERR_INVALID_ARG, "handle is NULL");
     if (K <= 0) return fail(SPMM_ERR_INVALID_ARG, "K must be positive");
     if (K % 4 != 0 || K > 1024) return fail(SPMM_ERR_UNSUPPORTED, "K must be a multiple of 4 and <= 1024");
@@ -353,6 +369,7 @@ spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *
 
 spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *C_dsts, int32_t n_dsts,
                         int64_t row_offset, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run_to");
     g_last_launches = 0;
     if (!h || !C_dsts) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     if (n_dsts < 1 || n_dsts > SPMM_MAX_CDST) return fail(SPMM_ERR_INVALID_ARG, "n_dsts must be in [1, 8]");
@@ -374,6 +391,7 @@ spmm_status spmm_run_to(spmm_handle h, const float *B, int64_t K, float *const *
 }
 
 spmm_status spmm_run_ld(spmm_handle h, const float *B, int64_t K, float *C, int64_t ldc, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run_ld");
     g_last_launches = 0;
     SPMM_TRY(check_run_args(h, B, K, C, true));
     if (ldc < K || ldc % 4 != 0) return fail(SPMM_ERR_UNSUPPORTED, "ldc must be >= K and a multiple of 4");
@@ -387,6 +405,7 @@ spmm_status spmm_run_ld(spmm_handle h, const float *B, int64_t K, float *C, int6
 
 spmm_status spmm_run_multicast(spmm_handle h, const float *B, int64_t K, float *C_mc, int64_t row_offset,
                                void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run_multicast");
     g_last_launches = 0;
     if (!h || !C_mc) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
     if (row_offset < 0) return fail(SPMM_ERR_INVALID_ARG, "negative row_offset");
@@ -408,6 +427,7 @@ spmm_status spmm_run_multicast(spmm_handle h, const float *B, int64_t K, float *
 }
 
 spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *C_host, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run_host");
     g_last_launches = 0;
     SPMM_TRY(check_run_args(h, B_host, K, C_host, false));
     SPMM_TRY(check_device(h));
@@ -424,6 +444,7 @@ spmm_status spmm_run_host(spmm_handle h, const float *B_host, int64_t K, float *
 
 spmm_status spmm_run_host_batch(spmm_handle h, int64_t n, const float *const *B_host, int64_t K,
                                 float *const *C_host, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_run_host_batch");
     g_last_launches = 0;
     if (!h || n < 0 || (n > 0 && (!B_host || !C_host))) return fail(SPMM_ERR_INVALID_ARG, "NULL argument or n < 0");
     for (int64_t i = 0; i < n; ++i) SPMM_TRY(check_run_args(h, B_host[i], K, C_host[i], false));
@@ -526,6 +547,7 @@ spmm_status spmm_partition_by_nnz(const int64_t *rowidx, int64_t M, int32_t P, i
 }
 
 spmm_status spmm_destroy(spmm_handle h) {
+    NvtxRange nvtx_("spmm_destroy");
     if (!h) return SPMM_OK;
     // wait for this handle's own work only (its runs' slot events, its copy streams), not the whole device
     release_run_slots(h);

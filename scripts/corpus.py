@@ -5,8 +5,11 @@ policy timed on the B200 (the exhaustive-timing label) plus the 24 featu
   python scripts/corpus.py --n-per-family 50 --out gpurun_out/corpus.jsonl
 
 Families: power-law R-MAT (natural / local / random-label), banded random,
-uniform random (Poisson degrees), block-clustered.  M log-uniform in [2^12, 2^max_log2m], nnz/row
-log-uniform in [2, 64].  Seeds 0..4n-1.
+uniform random (Poisson degrees), block-clustered.  M log-uniform in [2^12, 2^max_log2m] (round 2: up to 2^22,
+so that B at K >= 64 is far beyond the 126 MB L2 for a large part of the corpus), nnz/row log-uniform in [2, 64].
+Half of the power-law (natural / local) and banded matrices get their rows randomly relabelled ("shuffled":
+the original order then has no locality for the column-similarity orders to exploit).
+Policies: all twelve of the C-ABI plus CTA-aware over the median-block pre-order ("cta_aware+md").  Seeds 0..4n-1.
 """
 import argparse
 import json
@@ -26,6 +29,16 @@ import synthetic as syn  # noqa: E402
 import paper_conf_ispass_mehrabilcslo21_b200 as pkg  # noqa: E402
 
 FAMILIES = ["powerlaw", "banded", "uniform", "block"]
+
+
+def shuffle_rows(a, seed):
+    """Random row relabel (columns unchanged), as bench.make_matrix's shuffled configs."""
+    q = np.random.default_rng(seed).permutation(a.M)
+    lens = np.diff(a.rowidx)[q]
+    r = np.zeros(a.M + 1, dtype=np.int64)
+    np.cumsum(lens, out=r[1:])
+    idx = np.repeat(a.rowidx[q] - r[:-1], lens) + np.arange(a.nnz, dtype=np.int64)
+    return syn.CSR(a.M, a.N, r, a.colidx[idx], a.value[idx])
 
 
 def draw(i, max_log2m):
@@ -52,17 +65,23 @@ def draw(i, max_log2m):
         dd = int(min(round(d), c * 32))
         a = syn.blockcluster(M, M, g, c, dd, i)
         params = dict(g=g, c=c, d=dd)
+    if fam == "banded" or (fam == "powerlaw" and params["variant"] != "random-label"):
+        if rng.uniform() < 0.5:
+            a = shuffle_rows(a, 20_000 + i)
+            params["shuffled"] = True
     return fam, params, a
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n-per-family", type=int, default=50)
-    ap.add_argument("--max-log2m", type=float, default=20.0)
+    ap.add_argument("--max-log2m", type=float, default=22.0)
     ap.add_argument("--K", default="32,64,128,256")
-    ap.add_argument("--policies", default=",".join(pkg.HOT_PATH_POLICIES + ["lpt", "warp_aware", "dcsr"]))
-    ap.add_argument("--reps", type=int, default=7)
+    ap.add_argument("--policies", default=",".join(list(pkg.POLICIES) + ["cta_aware+md"]))
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=2)
     ap.add_argument("--start", type=int, default=0)
+    ap.add_argument("--stop", type=int, default=None)
     ap.add_argument("--out", default="gpurun_out/corpus.jsonl")
     args = ap.parse_args()
     Ks = [int(k) for k in args.K.split(",")]
@@ -71,7 +90,8 @@ def main():
     flush = torch.empty(64 * 1024 * 1024, device="cuda")   # 256 MiB
     stream = torch.cuda.current_stream()
     out = open(args.out, "a")
-    n = 4 * args.n_per_family
+    import bench
+    n = 4 * args.n_per_family if args.stop is None else args.stop
     for i in range(args.start, n):
         t0 = time.perf_counter()
         fam, params, a = draw(i, args.max_log2m)
@@ -84,11 +104,11 @@ def main():
         build = {}
         for pol in pols:
             tb = time.perf_counter()
-            h.permute(pol, window=1024)
+            bench.permute_spec(h, pol, 1024)
             build[pol] = 1e3 * (time.perf_counter() - tb)
             for K in Ks:
                 Ck = C[:, :K] if K == max(Ks) else torch.empty((a.M, K), device="cuda")
-                for _ in range(3):
+                for _ in range(args.warmup):
                     h.run(Bs[K], Ck)
                 ts = []
                 for _ in range(args.reps):

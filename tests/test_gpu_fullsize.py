@@ -5,9 +5,10 @@ features checked against the oracle (-m gpu).
 * C2  27-point stencil 100^3 (configs[1]), K=64 (row fusion engaged by default: R = 4)
 * C3  R-MAT S=22 "local", nnz 99.6M (configs[2]), K=128
 * C5  R-MAT S=24 "local", nnz 505M (configs[4], bench.py's default workload), K=128
-Sorted policies are compared in full; chain policies on sampled windows (each window's chain depends
-only on its own rows, so the oracle runs on the window's rows alone -- SURVEY.md §8(d) "Permutation
-parity at C5 checks ... a seeded random sample of windows plus the first and last").
+Sorted policies (incl. f1's LPT, Flipped Sort, DCSR) are compared in full; chain policies (incl. f1's Warp-aware,
+Hybrid-2.2, Hybrid-2.3 and the median-block pre-order) on 64 sampled windows plus the first and the last (each
+window's chain depends only on its own rows, so the oracle runs on the window's rows alone -- SURVEY.md §8(d)
+"Permutation parity at C5 checks ... a seeded random sample of 64 windows plus the first and last").
 """
 import numpy as np
 import pytest
@@ -57,10 +58,11 @@ def sample_rows(a, n=3000, seed=5):
     return np.array(sorted(picks), dtype=np.int64)
 
 
-@pytest.mark.parametrize("policy", pkg.HOT_PATH_POLICIES)
+@pytest.mark.parametrize("policy", pkg.HOT_PATH_POLICIES + ["flipped", "lpt", "warp_aware", "hybrid_2_2",
+                                                           "hybrid_2_3", "dcsr", "cta_aware+md"])
 def test_fullsize_spmm_sampled(full, policy):
     name, a, K, B, h = full
-    h.permute(policy, window=W)
+    bench.permute_spec(h, policy, W)
     Bd = torch.from_numpy(B).cuda()
     C = h.run(Bd)
     torch.cuda.synchronize()
@@ -80,12 +82,29 @@ def test_fullsize_sorts_and_features(full):
     np.testing.assert_array_equal(h.features_b200(K), oracle.features_b200(a, K))
 
 
-@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_1"])
-def test_fullsize_chain_windows_sampled(full, policy):
+@pytest.mark.parametrize("policy", ["lpt", "flipped", "dcsr"])
+def test_fullsize_f1_orders(full, policy):
+    """The rest of the paper's portfolio whose permutations are whole-matrix orders -- LPT
+    (reading A5: capacity-constrained over the nw warps), Flipped Sort and DCSR --
+    compared in full against the oracle at full size."""
     name, a, K, B, h = full
     h.permute(policy, window=W)
+    got = h.perm()
+    ref = oracle.permute(a, policy)
+    assert np.array_equal(got, ref), (name, policy, int(np.argmax(got != ref)))
+
+
+@pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_1", "warp_aware", "hybrid_2_2", "hybrid_2_3",
+                                    "cta_aware+md"])
+def test_fullsize_chain_windows_sampled(full, policy):
+    """Chain policies at full size on 64 seeded random windows plus the first and the last; each
+    window's chain depends only on its own rows, so the oracle runs on them alone.  '+md': windows over the
+    median-block pre-order (preorder = 2), recomputed here from the oracle's keys."""
+    name, a, K, B, h = full
+    bench.permute_spec(h, policy, W)
     perm = h.perm()
     rng = np.random.default_rng(11)
+    NS = 64
     if policy == "hybrid_1":
         plain = oracle.permute(a, "plain_sort")
         wl = (np.diff(a.rowidx) + 31) // 32
@@ -97,7 +116,7 @@ def test_fullsize_chain_windows_sampled(full, policy):
         run_start = np.maximum.accumulate(run_start)
         seg_starts = np.flatnonzero((np.arange(a.M) - run_start) % W == 0)
         seg_ends = np.r_[seg_starts[1:], a.M]
-        pick = sorted(set(rng.choice(len(seg_starts), size=min(40, len(seg_starts)), replace=False).tolist())
+        pick = sorted(set(rng.choice(len(seg_starts), size=min(NS, len(seg_starts)), replace=False).tolist())
                       | {0, len(seg_starts) - 1})
         for s in pick:
             lo, hi = seg_starts[s], seg_ends[s]
@@ -105,9 +124,13 @@ def test_fullsize_chain_windows_sampled(full, policy):
             ref = oracle.permute(sub_rows(a, rows), "hybrid_1", window=0)
             assert np.array_equal(perm[lo:hi], rows[ref]), (name, policy, s)
     else:
+        base = policy[:-3] if policy.endswith("+md") else policy
+        pre = (np.lexsort((np.arange(a.M), oracle.median_block_keys(a))) if policy.endswith("+md")
+               else np.arange(a.M))
         nwin = (a.M + W - 1) // W
-        pick = sorted(set(rng.choice(nwin, size=min(40, nwin), replace=False).tolist()) | {0, nwin - 1})
+        pick = sorted(set(rng.choice(nwin, size=min(NS, nwin), replace=False).tolist()) | {0, nwin - 1})
         for s in pick:
             lo, hi = s * W, min((s + 1) * W, a.M)
-            ref = oracle.permute(sub_rows(a, np.arange(lo, hi)), policy, window=0)
-            assert np.array_equal(perm[lo:hi], ref + lo), (name, policy, s)
+            rows = np.sort(pre[lo:hi])      # the window's row SET; every tie-break is by original row id (A2)
+            ref = oracle.permute(sub_rows(a, rows), base, window=0)
+            assert np.array_equal(perm[lo:hi], rows[ref]), (name, policy, s)
