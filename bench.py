@@ -333,6 +333,8 @@ def main():
     ap.add_argument("--window", type=int, default=1024)
     ap.add_argument("--policy-steps", type=int, default=5, help="timed steps per policy for the exhaustive selection")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-pipe-steps", type=int, default=16,
+                    help="right-hand sides per pipelined end-to-end measurement (fill and drain amortised over them)")
     ap.add_argument("--ref-sample-nnz", type=int, default=10_000_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cusparse", action="store_true")
@@ -561,7 +563,7 @@ def main():
     e2e_pipe = None
     if world == 1:
         try:
-            nst = max(3, args.e2e_steps)
+            nst = max(3, args.e2e_pipe_steps)
             Cp2 = [Cp, torch.empty((Mr, K), dtype=torch.float32).pin_memory()]
             Bs, Cs = [Bp] * nst, [Cp2[i % 2] for i in range(nst)]
             h.run_host_batch(Bs[:2], Cs[:2])          # warm-up (slots, streams)

@@ -100,6 +100,29 @@ def main():
             rd = to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
             traffic[f"{cfg}/{pol}"] = {"dram_bytes_per_launch": rd, "kernel": d["kernel"].split("(")[0],
                                        "duration": d["gpu__time_duration.sum"], "round": args.round}
+    # one process, one k_spmm launch per policy (scripts/profile_policies.py): prof_multi_<config>.raw.csv rows in
+    # the order of prof_multi_<config>.policies
+    for rc in sorted(glob.glob(os.path.join(OUT, "prof_multi_*.raw.csv"))):
+        cfg = re.match(r"prof_multi_([a-z0-9]+)\.raw\.csv", os.path.basename(rc)).group(1)
+        pols = [l.strip() for l in open(os.path.join(OUT, f"prof_multi_{cfg}.policies")) if l.strip()]
+        rows = list(csv.reader(open(rc)))
+        if len(rows) < 3:
+            continue
+        h, units = rows[0], rows[1]
+        for pol, r in zip(pols, rows[2:]):
+            d = {"kernel": r[h.index("Kernel Name")] if "Kernel Name" in h else ""}
+            for k in KEYS:
+                if k in h:
+                    d[k] = (r[h.index(k)], units[h.index(k)])
+            with open(os.path.join(PROF, f"{args.round}_ncu_{cfg}_{pol}.txt"), "w") as f:
+                f.write(f"# ncu --set full --clock-control none, one launch of {d['kernel']}\n")
+                f.write(f"# python scripts/profile_policies.py --config {cfg} (launch of policy {pol})\n")
+                for k in KEYS:
+                    if k in d:
+                        f.write(f"{k} {d[k][0]} {d[k][1]}\n")
+            rd = to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
+            traffic[f"{cfg}/{pol}"] = {"dram_bytes_per_launch": rd, "kernel": d["kernel"].split("(")[0],
+                                       "duration": d["gpu__time_duration.sum"], "round": args.round}
     with open(traffic_path, "w") as f:
         json.dump(traffic, f, indent=1, sort_keys=True)
     for bj in sorted(glob.glob(os.path.join(OUT, "bench*.json"))):
