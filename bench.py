@@ -68,11 +68,7 @@ def make_matrix(cfg):
 
 def permute_spec(h, pol, window):
     """A policy name, optionally with '+mh' / '+md': chain windows over the MinHash / median-block pre-order
-    (spmm_params.preorder = 1 / 2)."""
-    if pol.endswith("+mh"):
-        return h.permute(pol[:-3], window=window, preorder=1, seed=1)
-    if pol.endswith("+md"):
-        return h.permute(pol[:-3], window=window, preorder=2)
+    (spmm_params.preorder = 1 / 2; parsed by the binding's SpMM.permute)."""
     return h.permute(pol, window=window)
 
 

@@ -231,6 +231,13 @@ class SpMM:
         return cls(csr.M, csr.N, csr.rowidx, csr.colidx, csr.value, stream=stream)
 
     def permute(self, policy, stream=None, **params):
+        """spmm_permute.  policy: a name of POLICIES, optionally with a pre-order suffix for the chain policies --
+        "+md" (median-block pre-order, preorder = 2) or "+mh" (MinHash pre-order, preorder = 1, seed 1 unless given)."""
+        if isinstance(policy, str) and policy.endswith(("+md", "+mh")):
+            params.setdefault("preorder", 2 if policy.endswith("+md") else 1)
+            if policy.endswith("+mh"):
+                params.setdefault("seed", 1)
+            policy = policy[:-3]
         pid = POLICIES[policy] if isinstance(policy, str) else int(policy)
         p = make_params(**params)
         _check(load_library().spmm_permute(self._h, pid, ctypes.byref(p), _stream_ptr(stream)))
@@ -413,7 +420,9 @@ def spmm_predict_n(features, weights, n_policies):
     return int(pol.value), times
 
 
-PREDICTOR_POLICIES = HOT_PATH_POLICIES          # classes of the bundled predictor (reading A20)
+# classes of the bundled predictor (reading A20): the hot-path policies plus CTA-aware over the median-block
+# pre-order (round 2: the corpus' shuffled matrices make the pre-order the most frequent winner)
+PREDICTOR_POLICIES = HOT_PATH_POLICIES + ["cta_aware+md"]
 PAPER4_POLICIES = ["identity", "dcsr", "lpt", "warp_aware"]   # the paper's four classes
 
 

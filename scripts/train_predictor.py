@@ -1,6 +1,6 @@
 """Train and evaluate the permutation predictor on the C4 corpus (§V.B-E).
 
-  python scripts/train_predictor.py --corpus profiles/corpus_r1.jsonl --out profiles/predictor_r1.json
+  python scripts/train_predictor.py --corpus profiles/corpus_r2.jsonl --out profiles/predictor_r2.json
 
 Per K: a 24-64-32-P MLP with L2 regularisation regresses the execution times of the P policies
 (relative to the original order's time, reading A19), loss = mean absolute percentage error, samples
@@ -107,11 +107,13 @@ def evaluate(T, pred_choice, policies):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--corpus", default=os.path.join(ROOT, "profiles", "corpus_r1.jsonl"))
-    ap.add_argument("--policies", default="identity,nnz_sort,plain_sort,cta_aware,hybrid_1,hybrid_2_1")
+    ap.add_argument("--corpus", default=os.path.join(ROOT, "profiles", "corpus_r2.jsonl"))
+    ap.add_argument("--policies", default="identity,nnz_sort,plain_sort,cta_aware,hybrid_1,hybrid_2_1,cta_aware+md")
+    ap.add_argument("--table-policies", default=None,
+                    help="policies of the Table-I analogue (default: every policy timed in the corpus)")
     ap.add_argument("--K", default="32,64,128,256")
     ap.add_argument("--epochs", type=int, default=3000)
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "predictor_r1.json"))
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "predictor_r2.json"))
     ap.add_argument("--weights-dir", default=os.path.join(ROOT, "paper_conf_ispass_mehrabilcslo21_b200", "predictor"))
     args = ap.parse_args()
     policies = args.policies.split(",")
@@ -134,12 +136,16 @@ def main():
         w = cw[best_tr]
         res = {"n_train": int(ntr), "n_test": int(len(te)), "class_population_train": pop.astype(int).tolist(),
                "class_weights": cw.tolist()}
-        # Table-I analogue over the whole corpus: per-policy speedup vs the original order
-        sp = T[:, :1] / T
+        # Table-I analogue over the whole corpus: per-policy speedup vs the original order, every timed policy
+        tab_pols = (args.table_policies.split(",") if args.table_policies else
+                    list(json.loads(open(args.corpus).readline())["times_ms"][str(K)].keys()))
+        _, TT, _ = load(args.corpus, K, tab_pols)
+        sp = TT[:, :1] / TT
         res["table1"] = {p: {"max": float(sp[:, i].max()), "mean": float(sp[:, i].mean()), "min": float(sp[:, i].min())}
-                         for i, p in enumerate(policies)}
-        res["table1"]["oracle"] = {"max": float((T[:, 0] / T.min(1)).max()), "mean": float((T[:, 0] / T.min(1)).mean()),
-                                   "min": float((T[:, 0] / T.min(1)).min())}
+                         for i, p in enumerate(tab_pols)}
+        res["table1"]["oracle"] = {"max": float((TT[:, 0] / TT.min(1)).max()),
+                                   "mean": float((TT[:, 0] / TT.min(1)).mean()), "min": float((TT[:, 0] / TT.min(1)).min())}
+        res["table1_best_share"] = dict(zip(tab_pols, (np.bincount(TT.argmin(1), minlength=len(tab_pols)) / len(TT)).tolist()))
         res["best_policy_share"] = dict(zip(policies, (np.bincount(T.argmin(1), minlength=P) / len(T)).tolist()))
         all_feats = list(range(24))
         net, mu, sg = train(X[tr], Y[tr], w, all_feats, epochs=args.epochs, seed=K)
@@ -149,6 +155,19 @@ def main():
         ape = np.abs(Y[te] - pr) / Y[te] * 100
         res["regression"]["abs_error_pct_cdf"] = {"under_2": float((ape < 2).mean()), "under_10": float((ape < 10).mean()),
                                                   "median": float(np.median(ape))}
+        # 5-fold cross-validation: every matrix of the corpus predicted once by a model that did not see it (a test
+        # set of the whole corpus instead of one 20 % split)
+        folds = np.array_split(rng.permutation(len(X)), 5)
+        cv_choice = np.zeros(len(X), dtype=int)
+        for f in range(5):
+            te_f = folds[f]
+            tr_f = np.concatenate([folds[g] for g in range(5) if g != f])
+            bt = T[tr_f].argmin(1)
+            pp = np.bincount(bt, minlength=P).astype(np.float64)
+            cwf = np.where(pp > 0, pp.sum() / np.maximum(pp, 1) / P, 0.0)
+            netf, muf, sgf = train(X[tr_f], Y[tr_f], cwf[bt], all_feats, epochs=args.epochs, seed=K + 100 * f)
+            cv_choice[te_f] = predict(netf, muf, sgf, X[te_f], all_feats).argmin(1)
+        res["cv5_regression"] = evaluate(T, cv_choice, policies)
         # C inference through the library must agree with the torch forward
         wflat = flat_weights(net, mu, sg)
         agree = 0
@@ -183,6 +202,9 @@ def main():
         print(f"K={K}: n={len(X)} acc={r['accuracy']:.2f} oracle {r['speedup_oracle']:.3f}x predicted "
               f"{r['speedup_predicted']:.3f}x gain {r['oracle_gain_fraction']:.2f} loss {r['mean_loss']:.3f} "
               f"C-agree {res['c_inference_agreement']:.2f}")
+        c = res["cv5_regression"]
+        print(f"   5-fold CV (n={c['n']}): acc={c['accuracy']:.2f} oracle {c['speedup_oracle']:.3f}x predicted "
+              f"{c['speedup_predicted']:.3f}x gain {c['oracle_gain_fraction']:.2f} loss {c['mean_loss']:.3f}")
     with open(args.out, "w") as f:
         json.dump(report, f, indent=1)
 

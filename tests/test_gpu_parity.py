@@ -419,8 +419,11 @@ def test_select_policy_runs():
         pol4 = pkg.select_policy(h, K, paper_classes=True)
         assert pol4 in pkg.PAPER4_POLICIES
         assert pkg.select_policy(h, K, b200=True) in pkg.PREDICTOR_POLICIES    # f4: 24 + 7 features
-        h.permute(pol)
-        assert np.array_equal(h.perm(), oracle.permute(a, pol, window=1024))
+        for p in (pol, "cta_aware+md", "hybrid_2_1+mh"):     # the binding's pre-order suffixes
+            h.permute(p)
+            pre = {"+md": dict(preorder=2), "+mh": dict(preorder=1, seed=1)}.get(p[-3:], {})
+            base = p[:-3] if pre else p
+            assert np.array_equal(h.perm(), oracle.permute(a, base, window=1024, **pre)), p
     h.close()
 
 
