@@ -116,6 +116,15 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
  * Synchronises cuda_stream.  Errors: INVALID_ARG (NULL h, K <= 0), UNSUPPORTED (K), STATE, OOM, CUDA. */
 spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *C, void *cuda_stream);
 
+/* Install a caller-supplied permutation instead of building one -- e.g. a permutation computed offline and cached
+ * ("row permutations happen offline or the cost is amortized"; SURVEY §5 checkpoint / resume: the Python
+ * package's permcache stores spmm_get_perm results keyed by a hash of the CSR, policy and parameters).  perm: HOST
+ * int32[M], perm[p] = original row at position p; checked on the device to be a bijection on [0, M).  Builds the
+ * permuted CSR and row classes as spmm_permute does (params: split_nnz; NULL = defaults), atomically: on any error
+ * the handle keeps its previous permutation.  Synchronises cuda_stream.  Errors: INVALID_ARG (NULL, not a
+ * bijection, bad params), STATE, OOM, CUDA. */
+spmm_status spmm_set_perm(spmm_handle h, const int32_t *perm, const spmm_params *params, void *cuda_stream);
+
 /* Copy the current permutation (M int32, HOST buffer).  Reads it back on the handle's own non-blocking
  * stream (the permutation is complete when spmm_permute returns); no device-wide synchronisation. */
 spmm_status spmm_get_perm(spmm_handle h, int32_t *perm_out);

@@ -55,7 +55,7 @@ _lib = None
 _ALLOC_T = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 _FREE_T = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 _alloc_cbs = None
-EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_prepare", "spmm_get_perm",
+EXPORTS = ["spmm_default_params", "spmm_set_allocator", "spmm_create", "spmm_permute", "spmm_prepare", "spmm_set_perm", "spmm_get_perm",
            "spmm_get_permuted_csr", "spmm_get_info", "spmm_get_schedule_info", "spmm_features", "spmm_features_b200", "spmm_run", "spmm_run_to", "spmm_run_ld", "spmm_run_multicast", "spmm_run_host", "spmm_run_host_batch", "spmm_predict", "spmm_predict_n",
            "spmm_partition_by_nnz", "spmm_destroy", "spmm_status_string", "spmm_last_error",
            "spmm_last_run_launches", "spmm_set_kernel_timing", "spmm_last_kernel_ms"]
@@ -77,6 +77,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
         "spmm_create": (st, [vp, i64, i64, i64, vp, vp, vp, ctypes.c_int, vp]),
         "spmm_permute": (st, [vp, ctypes.c_int, vp, vp]),
         "spmm_prepare": (st, [vp, i64, vp, vp, vp]),
+        "spmm_set_perm": (st, [vp, vp, vp, vp]),
         "spmm_get_perm": (st, [vp, vp]),
         "spmm_get_permuted_csr": (st, [vp, vp, vp, vp]),
         "spmm_get_info": (st, [vp, vp]),
@@ -249,6 +250,16 @@ class SpMM:
         (B / C: the buffers the runs will use -- only their alignment matters; None = aligned)."""
         _check(load_library().spmm_prepare(self._h, int(K), None if B is None else B.data_ptr(),
                                            None if C is None else C.data_ptr(), _stream_ptr(stream)))
+        return self
+
+    def set_perm(self, perm, stream=None, **params):
+        """spmm_set_perm: install a caller-supplied permutation (perm[p] = original row at position p), e.g. one
+        cached from an earlier spmm_permute (permcache.py)."""
+        pm = np.ascontiguousarray(perm, dtype=np.int32)
+        _need(pm.shape == (self.M,), f"perm must have M = {self.M} entries")
+        p = make_params(**params)
+        _check(load_library().spmm_set_perm(self._h, pm.ctypes.data, ctypes.byref(p), _stream_ptr(stream)))
+        self.policy = "custom"
         return self
 
     def perm(self) -> np.ndarray:

@@ -93,6 +93,15 @@ __global__ void k_row_len_stats(const int32_t *rowidx, int64_t M, int32_t *maxle
     if ((threadIdx.x & 31) == 0) { atomicMax(maxlen, m); atomicAdd(empty, e); }
 }
 
+// a caller-supplied permutation must be a bijection on [0, M): every value in range and seen exactly once
+__global__ void k_check_perm(const int32_t *perm, int64_t M, unsigned int *seen, int *err) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < M; p += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t r = perm[p];
+        if (r < 0 || (int64_t)r >= M) { atomicOr(err, 1); continue; }
+        if (atomicAdd(seen + r, 1u) != 0u) atomicOr(err, 2);
+    }
+}
+
 unsigned grid1d(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 32)); }
 
 spmm_status check_device(spmm_ctx *h) {
@@ -239,6 +248,51 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
         h->rc = rc;
         h->params = p;
         h->policy = policy;
+        for (int i = 0; i < SCHED_CACHE; ++i) h->sched[i].built = 0;
+        h->last_sched.store(-1);
+    } catch (const std::exception &e) {
+        return fail(SPMM_ERR_OOM, e.what());
+    }
+    return SPMM_OK;
+}
+
+spmm_status spmm_set_perm(spmm_handle h, const int32_t *perm_in, const spmm_params *params, void *cuda_stream) {
+    NvtxRange nvtx_("spmm_set_perm");
+    if (!h || (!perm_in && h->M > 0)) return fail(SPMM_ERR_INVALID_ARG, "NULL argument");
+    SPMM_TRY(check_device(h));
+    spmm_params p;
+    if (params) p = *params; else spmm_default_params(&p);
+    SPMM_TRY(check_params(p));
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    const int64_t M = h->M;
+    try {
+        DevBuf perm, rowptr_p, cv_p, seen, flag;
+        RowClasses rc;
+        SPMM_TRY(perm.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
+        if (M > 0) {
+            SPMM_TRY(seen.alloc(M * sizeof(unsigned int), s));
+            SPMM_TRY(flag.alloc(sizeof(int), s));
+            SPMM_CUDA(cudaMemcpyAsync(perm.p, perm_in, M * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+            SPMM_CUDA(cudaMemsetAsync(seen.p, 0, M * sizeof(unsigned int), s));
+            SPMM_CUDA(cudaMemsetAsync(flag.p, 0, sizeof(int), s));
+            k_check_perm<<<grid1d(M), 256, 0, s>>>(perm.as<int32_t>(), M, seen.as<unsigned int>(), flag.as<int>());
+            SPMM_CUDA(cudaGetLastError());
+            int herr = 0;
+            SPMM_CUDA(cudaMemcpyAsync(&herr, flag.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+            SPMM_CUDA(cudaStreamSynchronize(s));
+            if (herr) return fail(SPMM_ERR_INVALID_ARG, "perm is not a bijection on [0, M)");
+        }
+        SPMM_TRY(build_permuted_csr(h, p.split_nnz, perm, rowptr_p, cv_p, rc, s));
+        SPMM_CUDA(cudaStreamSynchronize(s));
+        std::lock_guard<std::mutex> lk(h->mu);
+        for (int i = 0; i < RUN_SLOTS; ++i)
+            if (h->slots[i].used) SPMM_CUDA(cudaEventSynchronize(h->slots[i].done));
+        h->perm.swap(perm);
+        h->rowptr_p.swap(rowptr_p);
+        h->cv_p.swap(cv_p);
+        h->rc = rc;
+        h->params = p;
+        h->policy = SPMM_POLICY_COUNT;      // a caller-supplied order (no builder)
         for (int i = 0; i < SCHED_CACHE; ++i) h->sched[i].built = 0;
         h->last_sched.store(-1);
     } catch (const std::exception &e) {

@@ -134,3 +134,17 @@ def test_bundled_predictor_matches_oracle_forward():
                 best, ref = oracle.mlp_forward(f, w, P)
                 assert pol == best
                 np.testing.assert_allclose(t, ref, rtol=1e-9, atol=1e-9)
+
+
+def test_permcache_key():
+    """permcache keys: a function of the CSR structure, the policy and its parameters only (CPU, no GPU)."""
+    import synthetic as syn
+    from paper_conf_ispass_mehrabilcslo21_b200.permcache import cache_key
+    a = syn.rmat(8, 4, 1)
+    k = cache_key(a.rowidx, a.colidx, "cta_aware", {"window": 1024})
+    assert k == cache_key(a.rowidx.copy(), a.colidx.copy(), "cta_aware", {"window": 1024})
+    assert k != cache_key(a.rowidx, a.colidx, "hybrid_2_1", {"window": 1024})
+    assert k != cache_key(a.rowidx, a.colidx, "cta_aware", {"window": 2048})
+    c = a.colidx.copy()
+    c[0] = (c[0] + 1) % a.N
+    assert k != cache_key(a.rowidx, c, "cta_aware", {"window": 1024})

@@ -164,3 +164,36 @@ def test_binding_argument_checks():
     ref, bound = oracle.spmm(a, B.cpu().numpy())
     assert np.all(np.abs(C.cpu().numpy() - ref) <= 1e-5 * bound + 1e-6)
     h.close()
+
+
+def test_set_perm_and_cache(tmp_path):
+    """spmm_set_perm installs a caller-supplied permutation (C bit-identical to the built one; a non-bijection is
+    rejected and leaves the handle unchanged); permcache stores a build and reinstalls it on the next call."""
+    from paper_conf_ispass_mehrabilcslo21_b200 import permcache
+    a = _matrix()
+    B = torch.from_numpy(syn.dense(a.N, 64, 4500)).cuda()
+    h = pkg.SpMM.from_csr(a)
+    h.permute("hybrid_2_1", window=2048)
+    built = h.perm()
+    C1 = h.run(B).clone()
+    h.permute("identity")
+    h.set_perm(built)
+    assert np.array_equal(h.perm(), built)
+    assert torch.equal(h.run(B).view(torch.int32), C1.view(torch.int32))
+    bad = built.copy()
+    bad[1] = bad[0]                                        # a duplicate: not a bijection
+    with pytest.raises(pkg.SpmmError):
+        h.set_perm(bad)
+    assert np.array_equal(h.perm(), built)                 # unchanged
+    bad[1] = a.M                                           # out of range
+    with pytest.raises(pkg.SpmmError):
+        h.set_perm(bad)
+    h2 = pkg.SpMM.from_csr(a)
+    p1, hit1 = permcache.permute_cached(h2, a, "cta_aware+md", str(tmp_path), window=1024)
+    p2, hit2 = permcache.permute_cached(h2, a, "cta_aware+md", str(tmp_path), window=1024)
+    assert (hit1, hit2) == (False, True) and np.array_equal(p1, p2) and np.array_equal(h2.perm(), p1)
+    assert np.array_equal(p1, oracle.permute(a, "cta_aware", window=1024, preorder=2))
+    _, hit3 = permcache.permute_cached(h2, a, "cta_aware+md", str(tmp_path), window=2048)   # other params: miss
+    assert not hit3
+    h.close()
+    h2.close()
