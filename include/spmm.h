@@ -113,6 +113,7 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
  * fully asynchronous.  B / C (device, may be NULL) only select the lane geometry: 32-byte aligned (or NULL)
  * -> 256-bit lane loads, else 128-bit; pass the buffers the runs will use.  Up to 4 geometries are cached per
  * permutation.  A run whose geometry was not prepared builds it itself (and then synchronises its stream).
+ * Also sizes the scratch of runs captured into CUDA graphs (spmm_run).
  * Synchronises cuda_stream.  Errors: INVALID_ARG (NULL h, K <= 0), UNSUPPORTED (K), STATE, OOM, CUDA. */
 spmm_status spmm_prepare(spmm_handle h, int64_t K, const float *B, const float *C, void *cuda_stream);
 
@@ -167,7 +168,12 @@ spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, 
  * with this K): no host synchronisation, and runs on one handle may be issued concurrently from several
  * streams / host threads -- each run takes one of 4 handle-owned scratch slots (task counter, split-row
  * partials, zero-fill side stream) round-robin and waits, on its own stream, for that slot's previous run.
- * (The kernel-timing aid, spmm_set_kernel_timing, is the exception: its events belong to the handle.) */
+ * (The kernel-timing aid, spmm_set_kernel_timing, is the exception: its events belong to the handle.)
+ * CUDA graphs: a run may be captured (cudaStreamBeginCapture on cuda_stream, e.g. torch.cuda.graph) once
+ * spmm_prepare has built its K's schedule and sized the handle's capture scratch; the captured run allocates
+ * nothing and waits on nothing outside the graph (its zero-fill side stream forks from and joins the capture).
+ * Replays of graphs holding runs of one handle share that scratch and must be ordered (e.g. one stream).
+ * Capturing an unprepared K fails with SPMM_ERR_STATE before any work is queued. */
 spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream);
 
 /* spmm_run with the C all-gather fused into the epilogue (SURVEY §8(f) f2 ii): every row this handle computes

@@ -149,6 +149,7 @@ struct spmm_ctx {
     std::atomic<int> last_sched{-1};        // slot of the most recent run (spmm_get_schedule_info)
     std::mutex mu;                          // schedule builds and run-slot hand-out
     spmm::RunSlot slots[spmm::RUN_SLOTS];
+    spmm::RunSlot cap_slot;                 // scratch of runs captured into CUDA graphs (sized by spmm_prepare)
     uint32_t next_slot = 0;
     cudaStream_t aux = nullptr;             // non-blocking stream of host read-backs (no device-wide sync)
     // host-run staging (spmm_run_host: one slot; spmm_run_host_batch: two slots each, double-buffered)

@@ -908,8 +908,10 @@ Config choose_for(spmm_ctx *h, int64_t K, const float *B, const float *C, const 
 }  // namespace
 
 // The schedule for (rpw, R): a cached slot, else built into the oldest slot (waiting for this handle's runs in
-// flight first, since they may read the slot being replaced).  Called with h->mu held.
-static spmm_status get_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s, int *slot_out) {
+// flight first, since they may read the slot being replaced).  Called with h->mu held.  allow_build = false (a run
+// being captured into a CUDA graph): a missing schedule is an error, since building one synchronises.
+static spmm_status get_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_t s, int *slot_out,
+                                bool allow_build = true) {
     int oldest = 0;
     for (int i = 0; i < SCHED_CACHE; ++i) {
         const Schedule &S = h->sched[i];
@@ -919,6 +921,9 @@ static spmm_status get_schedule(spmm_ctx *h, int32_t rpw, int32_t R, cudaStream_
         }
         if (S.built < h->sched[oldest].built) oldest = i;
     }
+    if (!allow_build)
+        return fail(SPMM_ERR_STATE, "no run schedule for this K: call spmm_prepare(h, K, ...) before capturing spmm_run "
+                                    "into a CUDA graph");
     for (int i = 0; i < RUN_SLOTS; ++i)
         if (h->slots[i].used) SPMM_CUDA(cudaEventSynchronize(h->slots[i].done));
     Schedule &S = h->sched[oldest];
@@ -935,14 +940,20 @@ spmm_status prepare_schedule(spmm_ctx *h, int64_t K, const float *B, const float
     std::lock_guard<std::mutex> lk(h->mu);
     int slot = 0;
     SPMM_TRY(get_schedule(h, 32 / cfg.G, cfg.R, s, &slot));
+    // the scratch of runs captured into CUDA graphs (no allocation may happen inside a capture)
+    RunSlot &cs = h->cap_slot;
+    if (cs.counters.bytes < 64 * sizeof(unsigned int)) SPMM_TRY(cs.counters.alloc(64 * sizeof(unsigned int), s));
+    const size_t need = (size_t)h->sched[slot].n_pslots * K * sizeof(float);
+    if (cs.partials.bytes < need) SPMM_TRY(cs.partials.alloc(need, s));
+    SPMM_CUDA(cudaStreamSynchronize(s));
     // the fused kernel's schedule falls back to R = 1 when the unions do not pay; the W = 4 geometry of the same K
     // (misaligned B / C) shares rpw only when G matches, so it is prepared on first use
     return SPMM_OK;
 }
 
 void release_run_slots(spmm_ctx *h) {
-    for (int i = 0; i < RUN_SLOTS; ++i) {
-        RunSlot &r = h->slots[i];
+    for (int i = 0; i <= RUN_SLOTS; ++i) {
+        RunSlot &r = i < RUN_SLOTS ? h->slots[i] : h->cap_slot;
         if (r.done) {
             cudaEventSynchronize(r.done);
             cudaEventDestroy(r.done);
@@ -977,12 +988,18 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
         copy_extra = true;
     }
     const int32_t rpw = 32 / cfg.G;
+    // a run being captured into a CUDA graph (cudaStreamBeginCapture / torch.cuda.graph) uses the handle's capture
+    // slot: no host synchronisation, no allocation, no wait on events recorded outside the capture -- its schedule and
+    // scratch come from spmm_prepare.  Replays of graphs capturing runs of one handle must be ordered (one stream).
+    cudaStreamCaptureStatus cst = cudaStreamCaptureStatusNone;
+    SPMM_CUDA(cudaStreamIsCapturing(s, &cst));
+    const bool capturing = cst != cudaStreamCaptureStatusNone;
     RunSlot *rs = nullptr;
     int sidx = 0;
     {
         std::lock_guard<std::mutex> lk(h->mu);
-        SPMM_TRY(get_schedule(h, rpw, cfg.R, s, &sidx));
-        rs = &h->slots[h->next_slot++ % RUN_SLOTS];
+        SPMM_TRY(get_schedule(h, rpw, cfg.R, s, &sidx, !capturing));
+        rs = capturing ? &h->cap_slot : &h->slots[h->next_slot++ % RUN_SLOTS];
         if (!rs->done) {
             SPMM_CUDA(cudaEventCreateWithFlags(&rs->done, cudaEventDisableTiming));
             SPMM_CUDA(cudaStreamCreateWithFlags(&rs->side, cudaStreamNonBlocking));
@@ -990,8 +1007,8 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
             SPMM_CUDA(cudaEventCreateWithFlags(&rs->join, cudaEventDisableTiming));
         }
         // the slot's previous run (maybe on another stream) must be done with its scratch
-        if (rs->used) SPMM_CUDA(cudaStreamWaitEvent(s, rs->done, 0));
-        rs->used = true;
+        if (rs->used && !capturing) SPMM_CUDA(cudaStreamWaitEvent(s, rs->done, 0));
+        rs->used = !capturing;
         h->last_sched.store(sidx);
     }
     const Schedule &S = h->sched[sidx];
@@ -1000,7 +1017,10 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
     float4 *P4 = nullptr;
     if (S.n_pslots > 0) {
         const size_t need = (size_t)S.n_pslots * K * sizeof(float);
-        if (rs->partials.bytes < need) SPMM_TRY(rs->partials.alloc(need, s));
+        if (rs->partials.bytes < need) {
+            if (capturing) return fail(SPMM_ERR_STATE, "capture: call spmm_prepare with this K first (scratch)");
+            SPMM_TRY(rs->partials.alloc(need, s));
+        }
         P4 = rs->partials.as<float4>();
     }
     // empty rows: zero fill on the slot's side stream forked from / joined to `s`, one small CTA per SM, so its HBM
@@ -1023,16 +1043,19 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
         const int64_t blocks = std::max<int64_t>(1, std::min<int64_t>(ceil_div(S.n_tasks, SPMM_THREADS / 32),
                                                                       (int64_t)h->num_sms * occ));
         const dim3 grid((unsigned)blocks, (unsigned)cfg.tiles);
-        if (rs->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int))
+        if (rs->counters.bytes < (size_t)cfg.tiles * sizeof(unsigned int)) {
+            if (capturing) return fail(SPMM_ERR_STATE, "capture: call spmm_prepare with this K first (scratch)");
             SPMM_TRY(rs->counters.alloc(64 * sizeof(unsigned int), s));
+        }
         SPMM_CUDA(cudaMemsetAsync(rs->counters.p, 0, (size_t)cfg.tiles * sizeof(unsigned int), s));
-        if (h->timing) SPMM_CUDA(cudaEventRecord(h->ev0, s));
+        const bool timed = h->timing && !capturing;
+        if (timed) SPMM_CUDA(cudaEventRecord(h->ev0, s));
         kern<<<grid, SPMM_THREADS, 0, s>>>(S.units.as<int4>(), S.n_tasks, h->cv_p.as<int2>(),
                                            reinterpret_cast<const float4 *>(B), C4, K4, ldc4, P4,
                                            rs->counters.as<unsigned int>(), S.recs.as<int4>(), S.gdst.as<int32_t>(),
                                            copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
-        if (h->timing) {
+        if (timed) {
             SPMM_CUDA(cudaEventRecord(h->ev1, s));
             h->timed = true;
         }
@@ -1049,7 +1072,7 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
     if (copy_extra)
         for (int i = 0; i < cx.n; ++i)
             SPMM_CUDA(cudaMemcpyAsync(cx.p[i], C, (size_t)M * K * sizeof(float), cudaMemcpyDeviceToDevice, s));
-    SPMM_CUDA(cudaEventRecord(rs->done, s));
+    if (!capturing) SPMM_CUDA(cudaEventRecord(rs->done, s));
     return SPMM_OK;
 }
 

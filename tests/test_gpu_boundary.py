@@ -197,3 +197,42 @@ def test_set_perm_and_cache(tmp_path):
     assert not hit3
     h.close()
     h2.close()
+
+
+def test_cuda_graph_capture():
+    """spmm_run captured into a CUDA graph (torch.cuda.graph) after spmm_prepare: replays with new B values give
+    C bit-identical to eager runs (split rows, empty rows and the side-stream zero fill included); capturing an
+    unprepared K fails cleanly with SPMM_ERR_STATE."""
+    a = _matrix()
+    h = pkg.SpMM.from_csr(a)
+    h.permute("cta_aware")
+    K = 64
+    Bs = [torch.from_numpy(syn.dense(a.N, K, 4600 + i)).cuda() for i in range(3)]
+    eager = [h.run(B).clone() for B in Bs]
+    B_static = torch.empty_like(Bs[0])
+    C_static = torch.full((a.M, K), float("nan"), device="cuda")
+    h.prepare(K, B_static, C_static)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            h.run(B_static, C_static, stream=s)
+    for B, ref in zip(Bs, eager):
+        B_static.copy_(B)
+        g.replay()
+        torch.cuda.synchronize()
+        assert torch.equal(C_static.view(torch.int32), ref.view(torch.int32))
+    g.reset()
+    h.permute("identity")                                   # drops the schedules: K = 64 is unprepared now
+    g2 = torch.cuda.CUDAGraph()
+    with pytest.raises(pkg.SpmmError) as e:
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g2, stream=s):
+                h.run(B_static, C_static, stream=s)
+    assert e.value.status == 6                                # SPMM_ERR_STATE
+    torch.cuda.synchronize()
+    C = h.run(Bs[0])                                          # the handle is fine afterwards
+    ref, bound = oracle.spmm(a, Bs[0].cpu().numpy())
+    assert np.all(np.abs(C.cpu().numpy() - ref) <= 1e-5 * bound + 1e-6)
+    h.close()
