@@ -91,6 +91,31 @@ __global__ void __launch_bounds__(256, 3) k_probe(const char *__restrict__ B, ui
     if (threadIdx.x == 0) atomicMax(cyc + blockIdx.x % 1024, (unsigned long long)(t1 - t0));
 }
 
+// shape 0 with UU row loads in flight per lane and MINB CTAs per SM (in-flight bytes per SM = 8 warps x MINB x 32
+// lanes x UU x 32 B): how the L2 gather rate grows with the bytes in flight (latency- vs bandwidth-bound)
+template <int UU, int MINB>
+__global__ void __launch_bounds__(256, MINB) k_probe_u(const char *__restrict__ B, uint32_t nrows, int RB, int iters,
+                                                     float *out, unsigned long long *cyc) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t wid = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    float acc = 0.f;
+    const long long t0 = clock64();
+    const int g = lane / 8, gl = lane % 8;
+    for (int it = 0; it < iters; ++it) {
+        f8 x[UU];
+#pragma unroll
+        for (int u = 0; u < UU; ++u) {
+            const uint32_t r = hrow(((wid * iters + it) * UU + u) * 8 + g, nrows);
+            x[u] = ld8<false>(B + (size_t)r * RB + (size_t)((it * UU + u) & (RB / 256 - 1)) * 256 + gl * 32);
+        }
+#pragma unroll
+        for (int u = 0; u < UU; ++u) acc += x[u].lo.x + x[u].hi.w;
+    }
+    const long long t1 = clock64();
+    out[(uint64_t)blockIdx.x * blockDim.x + threadIdx.x] = acc;
+    if (threadIdx.x == 0) atomicMax(cyc + blockIdx.x % 1024, (unsigned long long)(t1 - t0));
+}
+
 // shape 5: rows staged in shared memory (window <= 192 KB), gathered with LDS.128 (warp per 512-B row)
 __global__ void __launch_bounds__(256, 1) k_probe_smem(const char *__restrict__ B, uint32_t nrows, int RB, int iters,
                                                        float *out, unsigned long long *cyc) {
@@ -168,7 +193,84 @@ extern "C" double ldpath_gather(int shape, int64_t window, int RB, int reps, dou
 }
 
 #ifndef LDPATH_NO_MAIN
+// ./ldpathprobe sweep: shape 0 (k_spmm's) over windows x row sizes
+static int sweep() {
+    printf("{\"sweep\": [\n");
+    bool first = true;
+    for (int64_t wmb : {1, 4, 16, 32, 64, 100}) {
+        for (int rb : {256, 512, 1024, 2048}) {
+            double bpc = 0;
+            const double gbs = ldpath_gather(0, wmb << 20, rb, 5, &bpc);
+            printf("%s{\"window_mb\": %lld, \"row_bytes\": %d, \"GBps\": %.1f, \"bytes_per_sm_clk\": %.2f}",
+                   first ? "" : ",\n", (long long)wmb, rb, gbs, bpc);
+            first = false;
+        }
+    }
+    printf("\n]}\n");
+    return 0;
+}
+
+template <int UU, int MINB>
+static void run_u(const char *B, int64_t window, int RB, int sms, float *out, unsigned long long *cyc, bool &first) {
+    const uint32_t nrows = (uint32_t)(window / RB);
+    const int blocks = sms * MINB, iters = 2048 / UU;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    double best = 0, best_bpc = 0;
+    for (int rep = 0; rep < 5; ++rep) {
+        cudaMemset(cyc, 0, 1024 * sizeof(unsigned long long));
+        cudaEventRecord(e0);
+        k_probe_u<UU, MINB><<<blocks, 256>>>(B, nrows, RB, iters, out, cyc);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        unsigned long long hc[1024];
+        cudaMemcpy(hc, cyc, sizeof(hc), cudaMemcpyDeviceToHost);
+        unsigned long long mc = 1;
+        for (int i = 0; i < 1024; ++i) mc = hc[i] > mc ? hc[i] : mc;
+        const double bytes = (double)blocks * 8 * iters * UU * 1024.0;
+        const double gbs = bytes / (ms * 1e-3) / 1e9;
+        if (gbs > best) { best = gbs; best_bpc = bytes / sms / (double)mc; }
+    }
+    printf("%s{\"window_mb\": %lld, \"U\": %d, \"ctas_per_sm\": %d, \"inflight_kb_per_sm\": %d, \"GBps\": %.1f, "
+           "\"bytes_per_sm_clk\": %.2f, \"err\": \"%s\"}", first ? "" : ",\n", (long long)(window >> 20), UU, MINB,
+           8 * MINB * 32 * UU * 32 / 1024, best, best_bpc, cudaGetErrorString(cudaGetLastError()));
+    first = false;
+}
+
+static int inflight() {
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    char *B;
+    float *out;
+    unsigned long long *cyc;
+    cudaMalloc(&B, (size_t)1 << 30);
+    cudaMemset(B, 0, (size_t)1 << 30);
+    cudaMalloc(&out, (size_t)sms * 8 * 256 * sizeof(float));
+    cudaMalloc(&cyc, 1024 * sizeof(unsigned long long));
+    printf("{\"inflight\": [\n");
+    bool first = true;
+    for (int64_t wmb : {16, 100, 1024}) {
+        const int64_t w = wmb << 20;
+        run_u<1, 3>(B, w, 512, sms, out, cyc, first);
+        run_u<2, 3>(B, w, 512, sms, out, cyc, first);
+        run_u<4, 3>(B, w, 512, sms, out, cyc, first);
+        run_u<4, 2>(B, w, 512, sms, out, cyc, first);
+        run_u<8, 2>(B, w, 512, sms, out, cyc, first);
+        run_u<8, 1>(B, w, 512, sms, out, cyc, first);
+        run_u<16, 1>(B, w, 512, sms, out, cyc, first);
+        run_u<2, 4>(B, w, 512, sms, out, cyc, first);
+        run_u<4, 4>(B, w, 512, sms, out, cyc, first);
+    }
+    printf("\n]}\n");
+    return 0;
+}
+
 int main(int argc, char **argv) {
+    if (argc > 1 && argv[1][0] == 's') return sweep();
+    if (argc > 1 && argv[1][0] == 'i') return inflight();
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     const int RB = argc > 1 ? atoi(argv[1]) : 512;   // a power of two >= 512
