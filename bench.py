@@ -282,6 +282,28 @@ def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps
     tb = timed_max(torch, dist, world, fn_b, reps, stream)
     out["b_exchange"] = {"ms": tb, "bytes": b_bytes, "GBps": b_bytes / (tb * 1e-3) / 1e9,
                          "how": "distribute_B (NCCL sends of B[cols_p])" if compact else "NCCL broadcast"}
+    if compact:
+        # B arriving row-sharded (rank q owns rows [bo[q], bo[q+1])): one all-to-allv of exactly the referenced rows
+        bo = sh.b_owner_bounds()
+        n_q = int(bo[sh.rank + 1] - bo[sh.rank])
+        if sh.rank == 0:
+            for q in range(1, world):
+                sh.comm.send(Bfull[int(bo[q]):int(bo[q + 1])], q)
+            Bsl = Bfull[:n_q].contiguous()
+        else:
+            Bsl = torch.empty((n_q, K), dtype=torch.float32, device=Bd.device)
+            sh.comm.recv(Bsl, 0)
+        sh.setup_alltoall(Bd.device)
+        Ba = sh.exchange_B_alltoall(Bsl, K)
+        same = bool(torch.equal(Ba, Bd))
+        ta = timed_max(torch, dist, world, lambda: sh.exchange_B_alltoall(Bsl, K), reps, stream)
+        moved = torch.tensor([Bd.shape[0] - sh._a2a_need[sh.rank]], dtype=torch.int64, device=Bd.device)
+        dist.all_reduce(moved)       # rows that crossed GPUs (a rank's own slice stays local)
+        out["b_alltoall"] = {"ms": ta, "bytes": int(moved.item()) * K * 4,
+                             "GBps_aggregate": int(moved.item()) * K * 4 / (ta * 1e-3) / 1e9,
+                             "equals_distribute_B": same,
+                             "how": "B row-sharded over the ranks; exchange_B_alltoall (one all-to-allv of B[cols_p])"}
+        del Bsl, Ba
     c_bytes = (sh.M - Cd.shape[0]) * K * 4      # the other ranks' C rows this rank receives
     tc = timed_max(torch, dist, world, lambda: sh.allgather_C(Cd), reps, stream)
     out["c_allgather"] = {"ms": tc, "bytes_received_rank": c_bytes, "GBps_received_rank": c_bytes / (tc * 1e-3) / 1e9,

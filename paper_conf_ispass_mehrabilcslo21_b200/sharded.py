@@ -9,7 +9,9 @@ One process per GPU (torchrun), torch.distributed for the plumbing:
   3. B exchange (compact_B, f2 i): a rank holds only the B rows its shard references -- the shard's columns are
      renumbered to their index in its sorted distinct-column list cols_p (a monotone map: every row keeps its
      ascending column order, so C is bit-identical) and `src` sends each rank B[cols_p] (|cols_p| / N of a
-     broadcast); compact_B=False keeps the plain NCCL broadcast of all N rows;
+     broadcast); when B arrives row-sharded (each rank owns N/P rows), exchange_B_alltoall moves exactly those rows
+     in ONE all-to-allv in which every rank sends and receives at once; compact_B=False keeps the plain NCCL
+     broadcast of all N rows;
   4. each rank runs spmm_run on its shard -- C stays row-sharded in original row order;
   5. optionally C is all-gathered: NCCL all_gather (allgather_C), or fused into the SpMM epilogue -- per-peer
      stores into every rank's symmetric-memory buffer (run_allgather_fused, spmm_run_to) or one NVLS multicast
@@ -242,6 +244,51 @@ class ShardedSpMM:
         mine = torch.empty((len(self.cols), int(K)), dtype=dtype or torch.float32, device=device)
         self.comm.recv(mine, src)
         return mine
+
+    # ---- B arriving row-sharded: all-to-allv of exactly the rows each shard references ----------------------------
+    def b_owner_bounds(self):
+        """Row ranges of B owned by the ranks when B arrives row-sharded: rank q holds B[b_lo[q]:b_lo[q + 1]]
+        (equal splits of N)."""
+        return np.array([(q * self.N) // self.world for q in range(self.world + 1)], dtype=np.int64)
+
+    def setup_alltoall(self, device=None):
+        """Once per sharding (structure only): every rank tells every owner which of its B rows it needs (its sorted
+        columns cols_p cut at the owner boundaries), so that exchange_B_alltoall moves exactly B[cols_p]."""
+        import torch
+        assert self.compact_B, "the all-to-all exchange needs compact_B=True"
+        dev = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
+                                                 if self.comm.nccl else torch.device("cpu"))
+        bo = self.b_owner_bounds()
+        cols = torch.as_tensor(self.cols).to(dev).long()
+        cuts = torch.searchsorted(cols, torch.from_numpy(bo).to(dev))
+        need = (cuts[1:] - cuts[:-1]).to(torch.int64)           # rows I need from each owner q
+        give = torch.empty_like(need)                              # rows each rank p needs from me
+        self.dist.all_to_all_single(give, need, group=self.group)
+        self._a2a_need = [int(x) for x in need.cpu().tolist()]
+        self._a2a_give = [int(x) for x in give.cpu().tolist()]
+        req = torch.empty(sum(self._a2a_give), dtype=torch.int64, device=dev)
+        self.dist.all_to_all_single(req, cols, output_split_sizes=self._a2a_give, input_split_sizes=self._a2a_need,
+                                    group=self.group)
+        self._a2a_rows = req - int(bo[self.rank])                  # local row ids of my B slice, per requester
+        self._a2a_dev = dev
+        return self
+
+    def exchange_B_alltoall(self, B_slice, K=None):
+        """f2 (i) when B arrives row-sharded (rank q holds B_slice = B[b_lo[q]:b_lo[q + 1]], [n_q, K]): one
+        all-to-allv in which every owner sends each rank exactly the rows of its slice that the rank's shard
+        references.  Every rank sends and receives at once (aggregate NVLink bandwidth instead of one source's
+        link); the result is this rank's compact B_p = B[cols_p] (|cols_p| x K, sorted by column: owners are
+        ordered by row range).  setup_alltoall() first."""
+        import torch
+        if not hasattr(self, "_a2a_rows"):
+            self.setup_alltoall(B_slice.device)
+        K = int(B_slice.shape[1]) if K is None else int(K)
+        send = B_slice.index_select(0, self._a2a_rows.to(B_slice.device)) if len(self._a2a_rows) else \
+            torch.empty((0, K), dtype=B_slice.dtype, device=B_slice.device)
+        out = torch.empty((sum(self._a2a_need), K), dtype=B_slice.dtype, device=B_slice.device)
+        self.dist.all_to_all_single(out, send, output_split_sizes=self._a2a_need, input_split_sizes=self._a2a_give,
+                                    group=self.group)
+        return out
 
     def run(self, B, C_local=None):
         """Local SpMM on this rank's row shard (B resident on every rank). Returns the C shard."""

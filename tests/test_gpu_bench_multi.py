@@ -40,4 +40,5 @@ def test_bench_two_ranks_one_gpu(exchange):
     assert m["b_exchange"]["ms"] > 0 and m["c_allgather"]["ms"] > 0 and m["spmm_ms"] > 0
     if exchange == "rows":
         assert m["pipelined"]["bit_identical_to_run"] is True
+        assert m["b_alltoall"]["equals_distribute_B"] is True and m["b_alltoall"]["ms"] > 0
         assert d["e2e"]["h2d_bytes_per_step"] < d["config"]["N"] * d["config"]["K"] * 4 * 2

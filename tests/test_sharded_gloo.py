@@ -87,6 +87,12 @@ def _worker(rank, world, port, K, results, compact, how):
             assert np.array_equal(Bl.numpy(), Bfull[np.asarray(sh.cols)])
             assert int(cc.max()) < sh.shard.N
             C_local = sh.run(Bl)
+            # B arriving row-sharded (rank q owns B[bo[q]:bo[q+1]]): one all-to-allv delivers exactly B[cols_p]
+            bo = sh.b_owner_bounds()
+            Ba = sh.exchange_B_alltoall(torch.from_numpy(Bfull[bo[rank]:bo[rank + 1]]))
+            assert torch.equal(Ba, Bl)
+            Ba2 = sh.exchange_B_alltoall(torch.from_numpy(Bfull[bo[rank]:bo[rank + 1]]) * 2)   # reuses the setup
+            assert torch.equal(Ba2, Bl * 2)
             # f2 (iii): B in column chunks, each chunk's SpMM into its C columns as it arrives
             for chunks in (1, 3, 4):
                 Cp = torch.full((sh.shard.M, K), float("nan"))
