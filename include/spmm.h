@@ -173,7 +173,10 @@ spmm_status spmm_features_b200(spmm_handle h, int use_current_order, int64_t K, 
  * spmm_prepare has built its K's schedule and sized the handle's capture scratch; the captured run allocates
  * nothing and waits on nothing outside the graph (its zero-fill side stream forks from and joins the capture).
  * Replays of graphs holding runs of one handle share that scratch and must be ordered (e.g. one stream).
- * Capturing an unprepared K fails with SPMM_ERR_STATE before any work is queued. */
+ * Capturing an unprepared K fails with SPMM_ERR_STATE before any work is queued.  A graph holds device addresses
+ * of the handle's permuted CSR, schedule and capture scratch: spmm_permute / spmm_set_perm (new arrays), an
+ * spmm_prepare that grows the capture scratch (a larger K), and spmm_destroy invalidate graphs captured from the
+ * handle -- re-capture after them. */
 spmm_status spmm_run(spmm_handle h, const float *B, int64_t K, float *C, void *cuda_stream);
 
 /* spmm_run with the C all-gather fused into the epilogue (SURVEY §8(f) f2 ii): every row this handle computes
