@@ -50,7 +50,7 @@ def load(path, K, policies, b200=False):
             continue
         X.append(r["features"] + (r["features_b200"][str(K)] if b200 else []))
         T.append([t[p] for p in policies])
-        meta.append((r["i"], r["family"], r["name"]))
+        meta.append((r["i"], r["family"], r["name"], bool(r.get("params", {}).get("shuffled"))))
     return np.array(X, dtype=np.float64), np.array(T, dtype=np.float64), meta
 
 
@@ -168,6 +168,11 @@ def main():
             netf, muf, sgf = train(X[tr_f], Y[tr_f], cwf[bt], all_feats, epochs=args.epochs, seed=K + 100 * f)
             cv_choice[te_f] = predict(netf, muf, sgf, X[te_f], all_feats).argmin(1)
         res["cv5_regression"] = evaluate(T, cv_choice, policies)
+        shuf = np.array([bool(m[3]) for m in meta])
+        if shuf.any() and (~shuf).any():     # rows relabelled (the pre-order's regime) vs the rest
+            res["cv5_regression"]["by_subset"] = {
+                "shuffled": evaluate(T[shuf], cv_choice[shuf], policies),
+                "not_shuffled": evaluate(T[~shuf], cv_choice[~shuf], policies)}
         # C inference through the library must agree with the torch forward
         wflat = flat_weights(net, mu, sg)
         agree = 0
@@ -205,6 +210,8 @@ def main():
         c = res["cv5_regression"]
         print(f"   5-fold CV (n={c['n']}): acc={c['accuracy']:.2f} oracle {c['speedup_oracle']:.3f}x predicted "
               f"{c['speedup_predicted']:.3f}x gain {c['oracle_gain_fraction']:.2f} loss {c['mean_loss']:.3f}")
+        for k, v in c.get("by_subset", {}).items():
+            print(f"      {k}: n={v['n']} oracle {v['speedup_oracle']:.3f}x gain {v['oracle_gain_fraction']:.2f}")
     with open(args.out, "w") as f:
         json.dump(report, f, indent=1)
 
