@@ -37,6 +37,22 @@ def _compile(src):
     return obj
 
 
+def build_variant(defines, suffix):
+    """An A/B build of the library with extra -D defines (scripts/ab_lib.py); never loaded by the product path."""
+    out = os.path.join(BUILD, f"variant_{suffix}")
+    os.makedirs(out, exist_ok=True)
+    objs = []
+    for src in SOURCES:
+        obj = os.path.join(out, src.replace(".cu", ".o"))
+        subprocess.check_call([NVCC, *FLAGS, *[f"-D{d}" for d in defines], "-c", os.path.join(CSRC, src), "-o", obj],
+                              stdout=subprocess.DEVNULL, stderr=subprocess.DEVNULL)
+        objs.append(obj)
+    lib = os.path.join(out, f"libspmm_b200_{suffix}.so")
+    subprocess.check_call([NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", *objs, "-o", lib,
+                           "-lcudart_static", "-lrt", "-ldl", "-lpthread"])
+    return lib
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
     if force:

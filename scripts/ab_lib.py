@@ -1,0 +1,62 @@
+"""A/B of a compile-time library variant against the product build: the k_spmm kernel time (library events,
+spmm_set_kernel_timing) of one policy on one config, alternating the two libraries in separate processes.
+
+  python scripts/ab_lib.py --define SPMM_EXP_A_POLICY --configs c3,c5 --policy cta_aware
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+CHILD = r"""
+import sys, json, statistics, torch
+sys.path.insert(0, {root!r})
+import bench, synthetic as syn, paper_conf_ispass_mehrabilcslo21_b200 as pkg
+if {lib!r}:
+    pkg.load_library({lib!r})
+cfg = bench.CONFIGS[{config!r}]
+a = bench.make_matrix(cfg); K = cfg["K"]
+pkg.use_torch_allocator(True)
+B = torch.from_numpy(syn.dense(a.N, K, 1)).cuda(); C = torch.empty((a.M, K), device="cuda")
+h = pkg.SpMM.from_csr(a); h.permute({policy!r}); h.prepare(K, B, C)
+flush = torch.empty(64 * 1024 * 1024, device="cuda")
+for _ in range(3): h.run(B, C)
+h.set_kernel_timing(True)
+ks = []
+for _ in range(15):
+    flush.fill_(1.0); h.run(B, C); ks.append(h.last_kernel_ms())
+print(json.dumps({{"ms": statistics.median(ks)}}))
+"""
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--define", action="append", required=True)
+    ap.add_argument("--configs", default="c3")
+    ap.add_argument("--policy", default="cta_aware")
+    ap.add_argument("--rounds", type=int, default=3)
+    args = ap.parse_args()
+    from paper_conf_ispass_mehrabilcslo21_b200 import _build
+    lib_b = _build.build_variant(args.define, "_".join(d.lower() for d in args.define))
+    res = {}
+    for c in args.configs.split(","):
+        t = {"product": [], "variant": []}
+        for _ in range(args.rounds):
+            for name, lib in (("product", ""), ("variant", lib_b)):
+                out = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policy=args.policy)],
+                                     capture_output=True, text=True, timeout=1200)
+                line = [l for l in out.stdout.splitlines() if l.startswith("{")]
+                t[name].append(json.loads(line[-1])["ms"] if line else None)
+        res[c] = {k: v for k, v in t.items()}
+        res[c]["median"] = {k: statistics.median([x for x in v if x]) for k, v in t.items()}
+        print(c, json.dumps(res[c]), flush=True)
+    print(json.dumps({"defines": args.define, "policy": args.policy, "results": res}))
+
+
+if __name__ == "__main__":
+    main()
