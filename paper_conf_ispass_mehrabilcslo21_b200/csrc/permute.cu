@@ -1021,7 +1021,8 @@ spmm_status build_permuted_csr(spmm_ctx *h, int32_t split, const DevBuf &perm, D
                                RowClasses &rc, cudaStream_t s) {
     const int64_t M = h->M;
     SPMM_TRY(rowptr_p.alloc((M + 1) * sizeof(int32_t), s));
-    SPMM_TRY(cv_p.alloc(std::max<int64_t>(h->nnz, 1) * sizeof(int2), s));
+    // two pairs of slack: whole 16-byte blocks of a row range can be bulk-copied without reading past the end
+    SPMM_TRY(cv_p.alloc((std::max<int64_t>(h->nnz, 1) + 2) * sizeof(int2), s));
     DevBuf len;
     SPMM_TRY(len.alloc(std::max<int64_t>(M, 1) * sizeof(int32_t), s));
     if (M > 0) {

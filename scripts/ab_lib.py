@@ -30,7 +30,9 @@ h.set_kernel_timing(True)
 ks = []
 for _ in range(15):
     flush.fill_(1.0); h.run(B, C); ks.append(h.last_kernel_ms())
-print(json.dumps({{"ms": statistics.median(ks)}}))
+w = torch.arange(C.numel(), device="cuda", dtype=torch.int64) % 1000003 + 1
+crc = int(((C.reshape(-1).view(torch.int32).to(torch.int64) & 0xffffffff) * w).sum().item())   # bits of C
+print(json.dumps({{"ms": statistics.median(ks), "crc": crc}}))
 """
 
 
@@ -46,14 +48,18 @@ def main():
     res = {}
     for c in args.configs.split(","):
         t = {"product": [], "variant": []}
+        crcs = {}
         for _ in range(args.rounds):
             for name, lib in (("product", ""), ("variant", lib_b)):
                 out = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policy=args.policy)],
                                      capture_output=True, text=True, timeout=1200)
                 line = [l for l in out.stdout.splitlines() if l.startswith("{")]
-                t[name].append(json.loads(line[-1])["ms"] if line else None)
+                d = json.loads(line[-1]) if line else {}
+                t[name].append(d.get("ms"))
+                crcs.setdefault(name, set()).add(d.get("crc"))
         res[c] = {k: v for k, v in t.items()}
         res[c]["median"] = {k: statistics.median([x for x in v if x]) for k, v in t.items()}
+        res[c]["C_bit_identical"] = crcs.get("product") == crcs.get("variant") and len(crcs.get("product", ())) == 1
         print(c, json.dumps(res[c]), flush=True)
     print(json.dumps({"defines": args.define, "policy": args.policy, "results": res}))
 
