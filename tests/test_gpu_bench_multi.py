@@ -23,11 +23,11 @@ def _port():
     return p
 
 
-@pytest.mark.parametrize("exchange", ["rows", "broadcast"])
-def test_bench_two_ranks_one_gpu(exchange):
+@pytest.mark.parametrize("exchange,ranks", [("rows", 2), ("broadcast", 2), ("rows", 3)])
+def test_bench_ranks_one_gpu(exchange, ranks):
     env = {**os.environ, "BENCH_GPU_INDEX": "0", "BENCH_DIST_BACKEND": "gloo"}
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
-           "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"), "--gpus", "2", "--config", "c1",
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(ranks), "--master-addr",
+           "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"), "--gpus", str(ranks), "--config", "c1",
            "--steps", "3", "--warmup", "3", "--policy-steps", "2", "--e2e-steps", "3", "--no-cpu-baseline",
            "--no-cusparse", "--b-exchange", exchange, "--policies", "identity,nnz_sort,cta_aware"]
     r = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
@@ -35,7 +35,7 @@ def test_bench_two_ranks_one_gpu(exchange):
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout[-2000:]
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["value"] > 0 and d["gpu_launches"] > 0
+    assert d["n_gpus"] == ranks and d["value"] > 0 and d["gpu_launches"] > 0
     m = d["multi_gpu"]
     assert m["b_exchange"]["ms"] > 0 and m["c_allgather"]["ms"] > 0 and m["spmm_ms"] > 0
     if exchange == "rows":
