@@ -309,8 +309,10 @@ class ShardedSpMM:
         K = int(K)
         cb = chunk_bounds(K, chunks if chunks is not None else max(1, K // 64))
         if C_local is None:
-            C_local = torch.empty((self.shard.M, K), dtype=torch.float32,
-                                  device=device if device is not None else (B.device if B is not None else None))
+            if device is None:
+                device = B.device if B is not None else (torch.device("cuda", torch.cuda.current_device())
+                                                         if self.comm.nccl else torch.device("cpu"))
+            C_local = torch.empty((self.shard.M, K), dtype=torch.float32, device=device)
         if self.rank == src:
             keep = []
             for p in range(self.world):
