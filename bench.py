@@ -258,7 +258,7 @@ def timed_max(torch, dist, world, fn, reps, stream):
     return float(t.item())
 
 
-def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps=5, chunks=None):
+def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps=5, chunks=None, multicast=False):
     """N>1: the data-path communication of the sharded mode, timed on the device (max over
     ranks) and reported in GB/s of bytes moved between GPUs:
       b_exchange   -- per-rank B rows (distribute_B) or the broadcast of all of B;
@@ -318,12 +318,12 @@ def measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, reps
                             "GBps_per_rank_out": (world - 1) * Cd.shape[0] * K * 4 / max(t_f * 1e-3, 1e-9) / 1e9,
                             "how": "spmm_run_to: per-peer stores into the symmetric-memory full-C buffers"}
             mc = int(getattr(hdl, "multicast_ptr", 0) or 0)
-            if mc:
+            if mc and multicast:        # opt-in (--multicast): the NVLS store path has not run on hardware yet
                 t_m = timed_max(torch, dist, world, lambda: sh.run_allgather_multicast(Bd, mc), reps, stream)
                 out["multicast"] = {"ms": t_m, "allgather_added_ms": t_m - t_plain,
                                     "how": "spmm_run_multicast: one multimem.st per element (NVLS)"}
             else:
-                out["multicast"] = {"skipped": "the symmetric-memory rendezvous has no multicast address"}
+                out["multicast"] = {"skipped": "no multicast address" if not mc else "not requested (--multicast)"}
             del buf
         except Exception as e:  # noqa: BLE001
             out["fused"] = {"error": str(e)[:200]}
@@ -358,6 +358,8 @@ def main():
     ap.add_argument("--no-cusparse", action="store_true")
     ap.add_argument("--no-ceiling", action="store_true", help="skip the host LRU model of L2 reuse")
     ap.add_argument("--out", default=None, help="also write the JSON line to this file")
+    ap.add_argument("--multicast", action="store_true",
+                    help="N>1: also time the C all-gather through NVLS multicast stores (spmm_run_multicast)")
     ap.add_argument("--b-exchange", default="rows", choices=["rows", "broadcast"],
                     help="N>1: send each rank only the B rows its shard references (rows) or broadcast all of B")
     args = ap.parse_args()
@@ -535,7 +537,8 @@ def main():
         except Exception as e:  # noqa: BLE001
             l2 = {"error": str(e)[:200]}
 
-    multi = measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream) if world > 1 else None
+    multi = (measure_exchange(torch, dist, sh, h, Bd, Cd, Bfull, K, compact, stream, multicast=args.multicast)
+             if world > 1 else None)
 
     # ---- e2e through the public API with host buffers ----
     # N=1: spmm_run_host (H2D of B, SpMM, D2H of C).  N>1: rank 0 H2D of B, NCCL broadcast, SpMM on every
