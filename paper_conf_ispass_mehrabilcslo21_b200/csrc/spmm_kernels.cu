@@ -101,6 +101,15 @@ __device__ __forceinline__ float8 ld_b(const float8 *ptr) {
 }
 __device__ __forceinline__ int2 ld_cv(const int2 *ptr) { return __ldg(ptr); }
 
+// B row offset in W-float vectors (64-bit: B exceeds 4 GB at C5).  V = 1: unsigned 32 x 32 -> 64-bit (IMAD.WIDE.U32,
+// no sign extensions; column ids and strides are non-negative); V >= 2: signed (the unsigned form makes ptxas spill
+// in the K = 128 fused kernel)
+template <int V>
+__device__ __forceinline__ size_t brow(int32_t col, int32_t KV) {
+    if constexpr (V == 1) return (size_t)(uint32_t)col * (uint32_t)KV;
+    else return (size_t)col * KV;
+}
+
 // One work unit per lane group: the G lanes of group g own the unit u = (start, len, dst) and the V vectors
 // (VT = W floats each) col0 + v*G of its C row (colok: inside K; indices in VT units, KV = K / W per row).
 // Per nnz the group broadcasts the (col, val) pair with two shuffles from a register batch prefetched one
@@ -152,7 +161,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
                 VT x[U][V];
 #pragma unroll
                 for (int w = 0; w < U; ++w) {
-                    const VT *b = BV + (size_t)col[w] * KV + col0;
+                    const VT *b = BV + brow<V>(col[w], KV) + col0;
 #pragma unroll
                     for (int v = 0; v < V; ++v) {
                         if (colok[v]) x[w][v] = ld_b(b + v * G);
@@ -167,7 +176,7 @@ __device__ __forceinline__ void spmm_unit(const int4 u, const int g, const int g
 #pragma unroll
                 for (int w = 0; w < U - 1; ++w) {
                     if (w < rem) {
-                        const VT *b = BV + (size_t)col[w] * KV + col0;
+                        const VT *b = BV + brow<V>(col[w], KV) + col0;
 #pragma unroll
                         for (int v = 0; v < V; ++v)
                             if (colok[v]) vfma(a[w], ld_b(b + v * G), acc[v]);
@@ -277,13 +286,15 @@ __device__ __forceinline__ void spmm_unit_fused(const int4 u, const int g, const
                 VT x[U][V];
 #pragma unroll
                 for (int w = 0; w < U; ++w) {
-                    const VT *b = BV + (size_t)col[w] * KV + col0;
+                    const VT *b = BV + brow<V>(col[w], KV) + col0;
 #pragma unroll
                     for (int v = 0; v < V; ++v) {
                         if (colok[v] && w < rem) x[w][v] = ld_b(b + v * G);
-                        else vzero(x[w][v]);
+                        else if (V > 1) vzero(x[w][v]);   // V = 1: unused (the FFMA2s below are predicated by
+                                                          // the same w < rem); V = 2: keeps ptxas from spilling
                     }
                 }
+
 #pragma unroll
                 for (int w = 0; w < U; ++w)
 #pragma unroll
