@@ -95,7 +95,7 @@ def test_fullsize_f1_orders(full, policy):
 
 
 @pytest.mark.parametrize("policy", ["cta_aware", "hybrid_2_1", "hybrid_1", "warp_aware", "hybrid_2_2", "hybrid_2_3",
-                                    "cta_aware+md"])
+                                    "cta_aware+md", "hybrid_2_1+mh"])
 def test_fullsize_chain_windows_sampled(full, policy):
     """Chain policies at full size on 64 seeded random windows plus the first and the last; each
     window's chain depends only on its own rows, so the oracle runs on them alone.  '+md': windows over the
@@ -124,9 +124,13 @@ def test_fullsize_chain_windows_sampled(full, policy):
             ref = oracle.permute(sub_rows(a, rows), "hybrid_1", window=0)
             assert np.array_equal(perm[lo:hi], rows[ref]), (name, policy, s)
     else:
-        base = policy[:-3] if policy.endswith("+md") else policy
-        pre = (np.lexsort((np.arange(a.M), oracle.median_block_keys(a))) if policy.endswith("+md")
-               else np.arange(a.M))
+        base = policy[:-3] if policy.endswith(("+md", "+mh")) else policy
+        if policy.endswith("+md"):
+            pre = np.lexsort((np.arange(a.M), oracle.median_block_keys(a)))
+        elif policy.endswith("+mh"):                 # the binding's "+mh" = MinHash pre-order with seed 1
+            pre = np.lexsort((np.arange(a.M), oracle.minhash_keys(a, seed=1)))
+        else:
+            pre = np.arange(a.M)
         nwin = (a.M + W - 1) // W
         pick = sorted(set(rng.choice(nwin, size=min(NS, nwin), replace=False).tolist()) | {0, nwin - 1})
         for s in pick:
