@@ -102,6 +102,23 @@ __global__ void k_check_perm(const int32_t *perm, int64_t M, unsigned int *seen,
     }
 }
 
+// drop every cached run schedule (they describe the previous permutation) and free their arrays; the caller has
+// waited for the handle's runs in flight
+void clear_schedules(spmm_ctx *h) {
+    for (int i = 0; i < SCHED_CACHE; ++i) {
+        Schedule &S = h->sched[i];
+        S.built = 0;
+        S.rpw = 0;
+        S.recs.release();
+        S.gdst.release();
+        S.units.release();
+        S.long_dst.release();
+        S.pslot_ptr.release();
+        S.empty_dst.release();
+    }
+    h->last_sched.store(-1);
+}
+
 unsigned grid1d(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 32)); }
 
 spmm_status check_device(spmm_ctx *h) {
@@ -248,8 +265,7 @@ spmm_status spmm_permute(spmm_handle h, spmm_policy policy, const spmm_params *p
         h->rc = rc;
         h->params = p;
         h->policy = policy;
-        for (int i = 0; i < SCHED_CACHE; ++i) h->sched[i].built = 0;
-        h->last_sched.store(-1);
+        clear_schedules(h);
     } catch (const std::exception &e) {
         return fail(SPMM_ERR_OOM, e.what());
     }
@@ -293,8 +309,7 @@ spmm_status spmm_set_perm(spmm_handle h, const int32_t *perm_in, const spmm_para
         h->rc = rc;
         h->params = p;
         h->policy = SPMM_POLICY_COUNT;      // a caller-supplied order (no builder)
-        for (int i = 0; i < SCHED_CACHE; ++i) h->sched[i].built = 0;
-        h->last_sched.store(-1);
+        clear_schedules(h);
     } catch (const std::exception &e) {
         return fail(SPMM_ERR_OOM, e.what());
     }

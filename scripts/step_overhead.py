@@ -18,3 +18,17 @@ for _ in range(20):
     flush.fill_(1.0); h.run(B, C); ks.append(h.last_kernel_ms())
 res["kernel"] = statistics.median(ks)
 print(json.dumps(res))
+
+# the same steps under bench.py's conditions: NVML clock sampling thread + library kernel-timing events
+clk = bench.ClockSampler(0)
+clk.start()
+h.set_kernel_timing(True)
+res2 = {}
+for name, fn in (("h.run+clocks+timing", lambda: h.run(B, C)),):
+    ts = bench.time_runs(torch, fn, 30, lambda: flush.fill_(1.0), s, after=lambda: h.last_kernel_ms())
+    res2[name] = statistics.median(ts)
+h.set_kernel_timing(False)
+ts = bench.time_runs(torch, lambda: h.run(B, C), 30, lambda: flush.fill_(1.0), s)
+res2["h.run+clocks"] = statistics.median(ts)
+clk.stop()
+print(json.dumps(res2))
