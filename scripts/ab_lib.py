@@ -54,6 +54,8 @@ def main():
                 out = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policy=args.policy)],
                                      capture_output=True, text=True, timeout=1200)
                 line = [l for l in out.stdout.splitlines() if l.startswith("{")]
+                if not line:
+                    print(f"{c} {name}: child failed: {out.stderr[-1500:]}", file=sys.stderr, flush=True)
                 d = json.loads(line[-1]) if line else {}
                 t[name].append(d.get("ms"))
                 crcs.setdefault(name, set()).add(d.get("crc"))
