@@ -185,7 +185,7 @@ def oracle_sample_rows(a, target_nnz, seed=7):
     return rows, int(np.diff(a.rowidx)[rows].sum())
 
 
-def cpu_baseline(a, B, K, budget_s=15.0):
+def cpu_baseline(a, B, K, budget_s=15.0, single_thread=False):
     """The oracle (oracle.c, float64, OpenMP) as it stands, on a bounded row sample, on this host's cores."""
     import oracle
     # every core of this process's affinity set, replacing any inherited OMP_NUM_THREADS (torchrun sets 1);
@@ -202,9 +202,19 @@ def cpu_baseline(a, B, K, budget_s=15.0):
         t0 = time.perf_counter()
         oracle.spmm(a, B, rows=rows)
         dt = time.perf_counter() - t0
-    return {"value": 2.0 * snnz * K / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
-            "sample": f"{len(rows)} seeded random whole rows ({snnz} nnz of {a.nnz}), K={K}, float64 oracle_spmm_rows",
-            "seconds": dt}
+    res = {"value": 2.0 * snnz * K / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+           "sample": f"{len(rows)} seeded random whole rows ({snnz} nnz of {a.nnz}), K={K}, float64 oracle_spmm_rows",
+           "seconds": dt}
+    if single_thread:   # a 1-thread number beside the all-core one (C1 / C2)
+        oracle.set_threads(1)
+        rows1, snnz1 = oracle_sample_rows(a, max(1, snnz // max(cores, 1)))
+        t0 = time.perf_counter()
+        oracle.spmm(a, B, rows=rows1)
+        dt1 = time.perf_counter() - t0
+        oracle.set_threads(cores)
+        res["single_thread"] = {"value": 2.0 * snnz1 * K / dt1 / 1e9, "unit": "GFLOP/s", "cores": 1,
+                                "sample": f"{len(rows1)} rows ({snnz1} nnz)", "seconds": dt1}
+    return res
 
 
 def run_reference(args):
@@ -663,7 +673,7 @@ def main():
         return
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        cpu = cpu_baseline(a_full, B_host.numpy(), K)
+        cpu = cpu_baseline(a_full, B_host.numpy(), K, single_thread=args.config in ("c1", "c2"))
     # DRAM bytes of one k_spmm launch of the SELECTED policy on this config, from the committed ncu --set full
     # capture (scripts/profile_policies.py -> scripts/collect_profiles.py); null when that policy has none
     traffic, traffic_from = None, f"no committed ncu capture of {args.config}/{best}"
