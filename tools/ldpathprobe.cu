@@ -17,6 +17,7 @@
 #include <stdint.h>
 #include <stdio.h>
 #include <stdlib.h>
+#include <algorithm>
 
 struct f8 { float4 lo, hi; };
 template <bool NA>
@@ -108,6 +109,43 @@ __global__ void __launch_bounds__(256, MINB) k_probe_u(const char *__restrict__ 
             const uint32_t r = hrow(((wid * iters + it) * UU + u) * 8 + g, nrows);
             x[u] = ld8<false>(B + (size_t)r * RB + (size_t)((it * UU + u) & (RB / 256 - 1)) * 256 + gl * 32);
         }
+#pragma unroll
+        for (int u = 0; u < UU; ++u) acc += x[u].lo.x + x[u].hi.w;
+    }
+    const long long t1 = clock64();
+    out[(uint64_t)blockIdx.x * blockDim.x + threadIdx.x] = acc;
+    if (threadIdx.x == 0) atomicMax(cyc + blockIdx.x % 1024, (unsigned long long)(t1 - t0));
+}
+
+// Mixed residency (C5-like): a fraction far_pct of the row gathers go to a 1 GB window (DRAM misses), the rest to a
+// small L2-resident window; PF: each lane also issues prefetch.global.L2 for its sector of the rows it will load
+// PFD iterations later (a register-free way to bring far rows into L2 ahead of the register loads).
+template <int UU, int PF>
+__global__ void __launch_bounds__(256, 3) k_probe_mix(const char *__restrict__ B, uint32_t near_rows, uint32_t far_rows,
+                                                      int far_pct, int RB, int iters, float *out,
+                                                      unsigned long long *cyc) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t wid = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int g = lane / 8, gl = lane % 8;
+    float acc = 0.f;
+    const long long t0 = clock64();
+    auto addr = [&](uint64_t q) -> const char * {
+        const uint32_t hsh = (uint32_t)q * 0x9E3779B1u;
+        const bool far = (hsh >> 25) % 100u < (uint32_t)far_pct;
+        const uint32_t r = far ? (((hsh * 0x85EBCA6Bu) >> 3) & (far_rows - 1)) + near_rows : (hsh >> 7) & (near_rows - 1);
+        return B + (size_t)r * RB;
+    };
+    for (int it = 0; it < iters; ++it) {
+        if (PF > 0) {
+#pragma unroll
+            for (int u = 0; u < UU; ++u) {
+                const char *p = addr(((wid * iters + it + PF) * UU + u) * 8 + g) + gl * 32;
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+            }
+        }
+        f8 x[UU];
+#pragma unroll
+        for (int u = 0; u < UU; ++u) x[u] = ld8<false>(addr(((wid * iters + it) * UU + u) * 8 + g) + gl * 32);
 #pragma unroll
         for (int u = 0; u < UU; ++u) acc += x[u].lo.x + x[u].hi.w;
     }
@@ -268,9 +306,58 @@ static int inflight() {
     return 0;
 }
 
+template <int UU, int PF>
+static void run_mix(const char *B, int far_pct, int sms, float *out, unsigned long long *cyc, bool &first) {
+    const int RB = 256;                                  // one group load = one 256-B row slice
+    const uint32_t near_rows = (4u << 20) / RB, far_rows = (512u << 20) / RB;   // 4 MB near (L2), 512 MB far
+    const int blocks = sms * 3, iters = 2048 / UU;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    double best = 0;
+    for (int rep = 0; rep < 5; ++rep) {
+        cudaEventRecord(e0);
+        k_probe_mix<UU, PF><<<blocks, 256>>>(B, near_rows, far_rows, far_pct, RB, iters, out, cyc);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        const double bytes = (double)blocks * 8 * iters * UU * 1024.0;
+        best = std::max(best, bytes / (ms * 1e-3) / 1e9);
+    }
+    printf("%s{\"far_pct\": %d, \"U\": %d, \"prefetch_ahead\": %d, \"GBps\": %.1f, \"err\": \"%s\"}",
+           first ? "" : ",\n", far_pct, UU, PF, best, cudaGetErrorString(cudaGetLastError()));
+    first = false;
+}
+
+static int mixed() {
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    char *B;
+    float *out;
+    unsigned long long *cyc;
+    cudaMalloc(&B, (size_t)1 << 30);
+    cudaMemset(B, 0, (size_t)1 << 30);
+    cudaMalloc(&out, (size_t)sms * 3 * 256 * sizeof(float));
+    cudaMalloc(&cyc, 1024 * sizeof(unsigned long long));
+    printf("{\"mixed\": [\n");
+    bool first = true;
+    for (int fp : {0, 10, 20, 40, 100}) {
+        run_mix<4, 0>(B, fp, sms, out, cyc, first);
+        run_mix<4, 1>(B, fp, sms, out, cyc, first);
+        run_mix<4, 2>(B, fp, sms, out, cyc, first);
+        run_mix<4, 4>(B, fp, sms, out, cyc, first);
+        run_mix<2, 0>(B, fp, sms, out, cyc, first);
+        run_mix<2, 2>(B, fp, sms, out, cyc, first);
+    }
+    printf("\n]}\n");
+    return 0;
+}
+
 int main(int argc, char **argv) {
     if (argc > 1 && argv[1][0] == 's') return sweep();
     if (argc > 1 && argv[1][0] == 'i') return inflight();
+    if (argc > 1 && argv[1][0] == 'm') return mixed();
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     const int RB = argc > 1 ? atoi(argv[1]) : 512;   // a power of two >= 512
