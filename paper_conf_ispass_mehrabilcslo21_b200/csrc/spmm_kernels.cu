@@ -23,6 +23,7 @@
 // Bound: HBM bandwidth (algorithmic bytes 4(M+1) + 8 nnz + 4K|cols(A)| + 4MK, BASELINE.json north star).
 #include "internal.cuh"
 #include <algorithm>
+#include <cmath>
 #include <climits>
 #include <cstdlib>
 #include <vector>
@@ -456,16 +457,29 @@ __global__ void __launch_bounds__(256) k_combine(const float4 *__restrict__ P4, 
     }
 }
 
-// empty rows: zero-fill their C rows (thread per float4)
+// Empty rows: zero-fill their C rows.  Warp per row: each lane loads one of 32 consecutive row ids (one coalesced
+// load per 32 rows), then the warp walks them, storing each row's K/4 float4 with consecutive lanes (coalesced
+// streaming stores).  (Round 1 strided the grid over flattened (row, column) pairs, so every store of a thread needed
+// a fresh L2 load of its row id: ≈ 0.8 TB/s, 6 ms for C5's 3.9 GB of empty C rows -- the floor of a step whose
+// SpMM is short, e.g. the last shard of C5 at 8 GPUs.)
 __global__ void k_zero_rows(const int32_t *__restrict__ rows, int64_t n, int32_t K4, int32_t ldc4,
                             float4 *__restrict__ C4, const CExtra cx) {
-    const int64_t total = n * K4;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-        const size_t o = (size_t)rows[i / K4] * ldc4 + (i % K4);
-        if (!cx.skip_main) __stcs(C4 + o, make_float4(0.f, 0.f, 0.f, 0.f));
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int64_t base = warp * 32; base < n; base += nwarps * 32) {
+        const int32_t mine = base + lane < n ? __ldg(rows + base + lane) : 0;
+        const int cnt = n - base < 32 ? (int)(n - base) : 32;
+        for (int j = 0; j < cnt; ++j) {
+            const size_t o = (size_t)__shfl_sync(0xffffffffu, mine, j) * ldc4;
+            for (int32_t c = lane; c < K4; c += 32) {
+                if (!cx.skip_main) __stcs(C4 + o + c, z);
 #pragma unroll
-        for (int j = 0; j < SPMM_MAX_CDST - 1; ++j)
-            if (j < cx.n) xstore(cx.p[j] + o, make_float4(0.f, 0.f, 0.f, 0.f), (cx.mc >> j) & 1u);
+                for (int e = 0; e < SPMM_MAX_CDST - 1; ++e)
+                    if (e < cx.n) xstore(cx.p[e] + o + c, z, (cx.mc >> e) & 1u);
+            }
+        }
     }
 }
 
@@ -1035,12 +1049,19 @@ spmm_status launch_spmm(spmm_ctx *h, const float *B, int64_t K, float *C, int64_
         P4 = rs->partials.as<float4>();
     }
     // empty rows: zero fill on the slot's side stream forked from / joined to `s`, one small CTA per SM, so its HBM
-    // writes run alongside the L2-bound SpMM kernel (measured 2-4 % faster steps than a preceding launch)
+    // writes run alongside the L2-bound SpMM kernel (measured 2-4 % faster steps than a preceding launch).  Its width
+    // follows the share of the step it has to hide under: 1 warp per SM when the empty rows' bytes are a small
+    // fraction of the SpMM's B-row gather bytes (C3 / C5: 1.5-2 %; a faster fill there only competes with the SpMM's
+    // own DRAM traffic: C5 k_spmm +4 %), up to 4 when they are large (the last C5 shard at 8 GPUs: 8 %, where the
+    // narrow fill outlasted the SpMM: shard step 4.0 -> 2.5 ms).
     bool joined = true;
     if (S.n_empty > 0) {
+        const double zero_bytes = (double)S.n_empty * K * 4.0;
+        const double gather_bytes = std::max(1.0, (double)(h->nnz) * K * 4.0);
+        const int zw = (int)std::min(4.0, std::max(1.0, std::ceil(50.0 * zero_bytes / gather_bytes)));
         SPMM_CUDA(cudaEventRecord(rs->fork, s));
         SPMM_CUDA(cudaStreamWaitEvent(rs->side, rs->fork, 0));
-        k_zero_rows<<<(unsigned)h->num_sms, 128, 0, rs->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, ldc4, C4,
+        k_zero_rows<<<(unsigned)h->num_sms, 32 * zw, 0, rs->side>>>(S.empty_dst.as<int32_t>(), S.n_empty, K4, ldc4, C4,
                                                                 copy_extra ? CExtra{} : cx);
         SPMM_CUDA(cudaGetLastError());
         SPMM_CUDA(cudaEventRecord(rs->join, rs->side));
