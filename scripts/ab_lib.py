@@ -27,12 +27,14 @@ h = pkg.SpMM.from_csr(a); h.permute({policy!r}); h.prepare(K, B, C)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 for _ in range(3): h.run(B, C)
 h.set_kernel_timing(True)
-ks = []
+ks = []; st = []
+e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
 for _ in range(15):
-    flush.fill_(1.0); h.run(B, C); ks.append(h.last_kernel_ms())
+    flush.fill_(1.0); e0.record(); h.run(B, C); e1.record(); e1.synchronize()
+    ks.append(h.last_kernel_ms()); st.append(e0.elapsed_time(e1))
 w = torch.arange(C.numel(), device="cuda", dtype=torch.int64) % 1000003 + 1
 crc = int(((C.reshape(-1).view(torch.int32).to(torch.int64) & 0xffffffff) * w).sum().item())   # bits of C
-print(json.dumps({{"ms": statistics.median(ks), "crc": crc}}))
+print(json.dumps({{"ms": statistics.median(ks), "step_ms": statistics.median(st), "crc": crc}}))
 """
 
 
@@ -42,15 +44,18 @@ def main():
     ap.add_argument("--configs", default="c3")
     ap.add_argument("--policy", default="cta_aware")
     ap.add_argument("--rounds", type=int, default=3)
+    ap.add_argument("--base", action="append", default=[], help="defines of the baseline build (default: product)")
     args = ap.parse_args()
     from paper_conf_ispass_mehrabilcslo21_b200 import _build
     lib_b = _build.build_variant(args.define, "_".join(d.lower() for d in args.define))
+    lib_a = _build.build_variant(args.base, "_".join(d.lower() for d in args.base)) if args.base else ""
     res = {}
     for c in args.configs.split(","):
         t = {"product": [], "variant": []}
+        steps = {"product": [], "variant": []}
         crcs = {}
         for _ in range(args.rounds):
-            for name, lib in (("product", ""), ("variant", lib_b)):
+            for name, lib in (("product", lib_a), ("variant", lib_b)):
                 out = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policy=args.policy)],
                                      capture_output=True, text=True, timeout=1200)
                 line = [l for l in out.stdout.splitlines() if l.startswith("{")]
@@ -58,12 +63,14 @@ def main():
                     print(f"{c} {name}: child failed: {out.stderr[-1500:]}", file=sys.stderr, flush=True)
                 d = json.loads(line[-1]) if line else {}
                 t[name].append(d.get("ms"))
+                steps[name].append(d.get("step_ms"))
                 crcs.setdefault(name, set()).add(d.get("crc"))
         res[c] = {k: v for k, v in t.items()}
         res[c]["median"] = {k: statistics.median([x for x in v if x]) for k, v in t.items()}
+        res[c]["step_median"] = {k: statistics.median([x for x in v if x]) for k, v in steps.items()}
         res[c]["C_bit_identical"] = crcs.get("product") == crcs.get("variant") and len(crcs.get("product", ())) == 1
         print(c, json.dumps(res[c]), flush=True)
-    print(json.dumps({"defines": args.define, "policy": args.policy, "results": res}))
+    print(json.dumps({"defines": args.define, "base": args.base, "policy": args.policy, "results": res}))
 
 
 if __name__ == "__main__":

@@ -22,7 +22,14 @@ ap.add_argument("--policy", default="identity")
 ap.add_argument("--runs", type=int, default=3)
 ap.add_argument("--window", type=int, default=1024)
 ap.add_argument("--split", type=int, default=128)
+ap.add_argument("--lib", default="", help="an A/B variant library (scripts/ab_lib.py) instead of the product build")
+ap.add_argument("--define", action="append", default=[], help="build and load a variant with these -D defines")
 args = ap.parse_args()
+if args.define:
+    from paper_conf_ispass_mehrabilcslo21_b200 import _build
+    args.lib = _build.build_variant(args.define, "_".join(d.lower() for d in args.define))
+if args.lib:
+    pkg.load_library(args.lib)
 cfg = bench.CONFIGS[args.config]
 a = bench.make_matrix(cfg)
 K = cfg["K"]
