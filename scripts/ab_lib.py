@@ -27,14 +27,22 @@ h = pkg.SpMM.from_csr(a); h.permute({policy!r}); h.prepare(K, B, C)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 for _ in range(3): h.run(B, C)
 h.set_kernel_timing(True)
+import threading, pynvml
+pynvml.nvmlInit(); _hd = pynvml.nvmlDeviceGetHandleByIndex(0); _smp = []; _stop = threading.Event()
+def _sample():
+    while not _stop.is_set():
+        _smp.append((pynvml.nvmlDeviceGetPowerUsage(_hd) / 1000.0, pynvml.nvmlDeviceGetClockInfo(_hd, pynvml.NVML_CLOCK_SM)))
+        _stop.wait(0.005)
+_th = threading.Thread(target=_sample, daemon=True); _th.start()
 ks = []; st = []
 e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
 for _ in range(15):
     flush.fill_(1.0); e0.record(); h.run(B, C); e1.record(); e1.synchronize()
     ks.append(h.last_kernel_ms()); st.append(e0.elapsed_time(e1))
+_stop.set(); _th.join()
 w = torch.arange(C.numel(), device="cuda", dtype=torch.int64) % 1000003 + 1
 crc = int(((C.reshape(-1).view(torch.int32).to(torch.int64) & 0xffffffff) * w).sum().item())   # bits of C
-print(json.dumps({{"ms": statistics.median(ks), "step_ms": statistics.median(st), "crc": crc}}))
+print(json.dumps({{"ms": statistics.median(ks), "step_ms": statistics.median(st), "crc": crc, "power_w": statistics.median([x[0] for x in _smp]), "sm_mhz": statistics.median([x[1] for x in _smp])}}))
 """
 
 
@@ -53,6 +61,7 @@ def main():
     for c in args.configs.split(","):
         t = {"product": [], "variant": []}
         steps = {"product": [], "variant": []}
+        pw = {"product": [], "variant": []}
         crcs = {}
         for _ in range(args.rounds):
             for name, lib in (("product", lib_a), ("variant", lib_b)):
@@ -64,9 +73,11 @@ def main():
                 d = json.loads(line[-1]) if line else {}
                 t[name].append(d.get("ms"))
                 steps[name].append(d.get("step_ms"))
+                pw[name].append((d.get("power_w"), d.get("sm_mhz")))
                 crcs.setdefault(name, set()).add(d.get("crc"))
         res[c] = {k: v for k, v in t.items()}
         res[c]["median"] = {k: statistics.median([x for x in v if x]) for k, v in t.items()}
+        res[c]["power_w_sm_mhz"] = pw
         res[c]["step_median"] = {k: statistics.median([x for x in v if x]) for k, v in steps.items()}
         res[c]["C_bit_identical"] = crcs.get("product") == crcs.get("variant") and len(crcs.get("product", ())) == 1
         print(c, json.dumps(res[c]), flush=True)
