@@ -102,6 +102,8 @@ class ClockSampler:
     def __init__(self, index=0):
         self.index = index
         self.samples = []          # (sm_mhz, max_mhz, [reason flags])
+        self.power = []            # board power draw, W (NVML only)
+        self.power_limit = None
         self.source = None
         self._stop = threading.Event()
         self._t = None
@@ -122,6 +124,10 @@ class ClockSampler:
             nv, hd = self._nvml_handle()
             mx = float(nv.nvmlDeviceGetMaxClockInfo(hd, nv.NVML_CLOCK_SM))
             self.source = "nvml 10 ms"
+            try:
+                self.power_limit = nv.nvmlDeviceGetEnforcedPowerLimit(hd) / 1000.0
+            except Exception:  # noqa: BLE001
+                self.power_limit = None
         except Exception:  # noqa: BLE001
             nv = hd = None
             self.source = "nvidia-smi 200 ms"
@@ -133,6 +139,10 @@ class ClockSampler:
                         sm = float(nv.nvmlDeviceGetClockInfo(hd, nv.NVML_CLOCK_SM))
                         r = int(nv.nvmlDeviceGetCurrentClocksEventReasons(hd))
                         self.samples.append((sm, mx, [bool(r & b) for b in self.BITS]))
+                        try:
+                            self.power.append(nv.nvmlDeviceGetPowerUsage(hd) / 1000.0)
+                        except Exception:  # noqa: BLE001
+                            pass
                     else:
                         out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
                                               "--format=csv,noheader,nounits"], capture_output=True, text=True,
@@ -155,7 +165,8 @@ class ClockSampler:
         mx = [s[1] for s in self.samples]
         reasons = sorted({self.NAMES[i] for s in self.samples for i in range(4) if s[2][i]})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.samples), "source": self.source}
+                "reasons": reasons, "samples": len(self.samples), "source": self.source,
+                "power_w": statistics.median(self.power) if self.power else None, "power_limit_w": self.power_limit}
 
 
 def time_runs(torch, fn, steps, flush, stream, after=None):
