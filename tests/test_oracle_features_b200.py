@@ -101,3 +101,16 @@ def test_order_invariants_and_permuted_csr():
         r, c, v = oracle.permuted_csr(a, perm)
         ap = syn.CSR(a.M, a.N, r, c, v)
         np.testing.assert_array_equal(oracle.features_b200(ap, 128), g)
+
+
+def test_split_boundary_by_hand():
+    """The split-row threshold is strict (A24: rows with more than split_nnz = 128 nnz are split rows, g5) and the
+    short rows of g6 are 0 < len <= 128: rows of 127, 128, 129, 200 and 0 nnz, every value worked by hand."""
+    lens = [127, 128, 129, 200, 0]
+    a = syn.from_lists(5, 256, [list(range(n)) for n in lens])
+    g = oracle.features_b200(a, K=64)
+    assert g[4] == 1 / 5                                  # one empty row
+    assert g[5] == (129 + 200) / (127 + 128 + 129 + 200)  # 128 is not a split row
+    assert g[6] == (127 + 128) / (4 * 128)                # one RPW = 4 group [128, 127], slots 4 * 128
+    # union features: rows 0..4 are nested prefixes of 0..199 -> pairs {0..127}, {0..199}, {} ; quad {0..199}, {}
+    assert g[0] == (128 + 200) / 584 and g[1] == 200 / 584 and g[2] == 200 / 584
