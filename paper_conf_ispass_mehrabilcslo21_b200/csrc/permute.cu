@@ -492,18 +492,45 @@ __device__ __forceinline__ int32_t lower_win(const int32_t *brow, const int32_t 
     }
     return lo;
 }
+// Multi-window chains: the sub-range of each signature entry's posting list that lies in its own row's window
+// (the lists are sorted by window), found once per entry here -- two binary searches per entry, independent, so the
+// whole pass runs at memory throughput -- instead of inside every greedy step, where the searches of the reference
+// row's blocks were a chain of ~2 log2(list) dependent loads on the step's critical path.  Warp per row.
+__global__ void k_xrange(const int32_t *sig_ptr, const int32_t *sig_blk, int64_t M, const int32_t *bptr,
+                         const int32_t *brow, const int32_t *win, int2 *xr) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M;
+         r += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int32_t w = win[r];
+        for (int32_t e = sig_ptr[r] + lane; e < sig_ptr[r + 1]; e += 32) {
+            const int32_t b = sig_blk[e];
+            const int32_t a = lower_win(brow, win, bptr[b], bptr[b + 1], w);
+            xr[e] = make_int2(a, lower_win(brow, win, a, bptr[b + 1], w + 1));
+        }
+    }
+}
+
 template <class PT>
 __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *bptr, int32_t c0, int32_t nb,
                                         PT *pre, int32_t *bst, PT *wsum, const int32_t *brow = nullptr,
-                                        const int32_t *win = nullptr, int32_t mwin = -1) {
+                                        const int32_t *win = nullptr, int32_t mwin = -1,
+                                        const int2 *xr = nullptr) {
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     int32_t len = 0;
     if (tid < nb) {
-        const int32_t b = sig_blk[c0 + tid];
-        int32_t a = bptr[b], e = bptr[b + 1];
-        if (mwin >= 0) {
-            a = lower_win(brow, win, a, e, mwin);
-            e = lower_win(brow, win, a, e, mwin + 1);
+        int32_t a, e;
+        if (mwin >= 0 && xr) {                  // the window's sub-range, precomputed per signature entry (k_xrange)
+            const int2 v = __ldg(xr + c0 + tid);
+            a = v.x;
+            e = v.y;
+        } else {
+            const int32_t b = sig_blk[c0 + tid];
+            a = bptr[b];
+            e = bptr[b + 1];
+            if (mwin >= 0) {
+                a = lower_win(brow, win, a, e, mwin);
+                e = lower_win(brow, win, a, e, mwin + 1);
+            }
         }
         len = e - a;
         bst[tid] = a;
@@ -551,11 +578,11 @@ __device__ __forceinline__ void xvisit(const PT *pre, const int32_t *bst, int32_
 template <class PT, class F>
 __device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, const int32_t *sig_blk,
                                            const int32_t *bptr, const int32_t *brow, PT *pre, int32_t *bst,
-                                           PT *wsum, const int32_t *win, int32_t mwin, F f) {
+                                           PT *wsum, const int32_t *win, int32_t mwin, const int2 *xr, F f) {
     const int32_t bs = sig_ptr[r0], be = sig_ptr[r0 + 1];
     for (int32_t c0 = bs; c0 < be; c0 += XCH_THREADS) {
         const int32_t nb = min(XCH_THREADS, be - c0);
-        xprefix(sig_blk, bptr, c0, nb, pre, bst, wsum, brow, win, mwin);
+        xprefix(sig_blk, bptr, c0, nb, pre, bst, wsum, brow, win, mwin, xr);
         xvisit(pre, bst, nb, brow, f);
         __syncthreads();
     }
@@ -566,7 +593,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                                                             int64_t M, int multiwin,
                                                             const int32_t *sig_ptr, const int32_t *sig_blk,
                                                             const int32_t *bptr, const int32_t *brow,
-                                                            const int32_t *win, const uint32_t *ord,
+                                                            const int32_t *win, const int2 *xr, const uint32_t *ord,
                                                             const int32_t *nnz, int32_t nt, int32_t nw,
                                                             uint32_t *placed, int32_t *cnt0, int32_t *cnt1,
                                                             int32_t *cnt2a, int32_t *cnt2b, int32_t *perm) {
@@ -630,29 +657,29 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         const bool cached = be - bs <= XCH_CACHE;
         // prefix of ref's lists (kept for the score pass and for the next step's reset); the previous
         // step's prefix lives in the other buffer
-        if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw);
+        if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw, xr);
         // reset the previous step's counters (other buffer), then count |b_r ∩ b_ref|
         if (pref >= 0) {
             auto reset = [&](int32_t r) { co[r] = 0; };
             if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], brow, reset);
-            else xvisit_all(pref, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, reset);
+            else xvisit_all(pref, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, xr, reset);
         }
         auto count = [&](int32_t r) {
             if (r != prev && !is_placed(placed, r)) atomicAdd(cc + r, 1);
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
-        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, count);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, xr, count);
         int32_t ref2 = -1;
         int32_t *cc2 = buf ? cnt2b : cnt2a;
         uint32_t cp2 = 0;
         if constexpr (TWOREF) {
             int32_t *co2 = buf ? cnt2a : cnt2b;
             if (pref2 >= 0)
-                xvisit_all(pref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) { co2[r] = 0; });
+                xvisit_all(pref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, xr, [&](int32_t r) { co2[r] = 0; });
             ref2 = q >= nw ? (nw == 1 ? prev : out[q - nw]) : -1;
             if (ref2 >= 0) {
                 cp2 = nb_of(ref2);
-                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {
+                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, xr, [&](int32_t r) {
                     if (r != prev && !is_placed(placed, r)) atomicAdd(cc2 + r, 1);
                 });
             }
@@ -678,7 +705,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
             }
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
-        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, score);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, xr, score);
         if constexpr (TWOREF) {
             if (ref2 >= 0) {
                 // T2 ∩ class b0: b0 = |b| of the first unplaced row of the (|b|, r) order
@@ -698,7 +725,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                 const int32_t ptr = s_ptr;
                 const uint32_t b0 = ptr < n ? nb_of((int32_t)o[ptr]) : 0xffffffffu;
                 __syncthreads();   // everyone has read s_ptr before warp 0 may rewrite it below
-                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, [&](int32_t r) {
+                xvisit_all(ref2, sig_ptr, sig_blk, bptr, brow, pre2, bst2, wsum, win, mw, xr, [&](int32_t r) {
                     if (r != prev && !is_placed(placed, r) && nb_of(r) == b0) {
                         const Key k = keyof(r);
                         if (key_less(k, best)) best = k;
@@ -853,9 +880,21 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
              : k_chain_x<C_CTA, PT>;                                    // HYBRID_1 = C_CTA over segments
     };
     auto kern = wide ? pick(int64_t{}) : pick(int32_t{});
+    DevBuf xr;
+#ifdef SPMM_EXP_NO_XRANGE   // A/B variant: binary searches inside the greedy steps (round 2 before k_xrange)
+    if (false) {
+#else
+    if (nwin > 1 && sig.S > 0) {
+#endif
+        SPMM_TRY(xr.alloc(sig.S * sizeof(int2), s));
+        k_xrange<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M, bptr.as<int32_t>(),
+                                                    brow.as<int32_t>(), win.as<int32_t>(), xr.as<int2>());
+        SPMM_CUDA(cudaGetLastError());
+    }
     kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
-                                                win.as<int32_t>(), ord.as<uint32_t>(), nnz, p.nt, p.nw,
+                                                win.as<int32_t>(), xr.p ? xr.as<int2>() : nullptr,
+                                                ord.as<uint32_t>(), nnz, p.nt, p.nw,
                                                 placed.as<uint32_t>(), cnt.as<int32_t>(), cnt.as<int32_t>() + M,
                                                 mode == C_H22 ? cnt.as<int32_t>() + 2 * M : nullptr,
                                                 mode == C_H22 ? cnt.as<int32_t>() + 3 * M : nullptr, perm);
