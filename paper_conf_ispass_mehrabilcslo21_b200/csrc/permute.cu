@@ -14,6 +14,7 @@
 // Every argmin is over a total order ending in the original row id, so the result is deterministic
 // and bit-identical to the oracle (DESIGN.md §"Readings").
 #include "internal.cuh"
+#include <type_traits>
 #include <algorithm>
 #include <cstdlib>
 #include <vector>
@@ -434,17 +435,38 @@ __global__ void k_blk_fill(const int32_t *sig_ptr, const int32_t *blk, int64_t M
             brow[bptr[b] + atomicAdd(&bcur[b], 1)] = (int32_t)r;
         }
 }
-// multi-window: posting entries keyed by (block, window of the row), so each block's list holds every
-// window's rows contiguously and a window's CTA visits only its own (two binary searches per list)
-__global__ void k_blk_win_keys(const int32_t *sig_ptr, const int32_t *blk, int64_t M, const int32_t *win,
-                               uint64_t *keys, uint32_t *vals) {
+// multi-window: posting entries keyed by (window of the row, block), so a window's posting lists are one contiguous
+// chunk, list by list (rows ascending within a list: the sort is stable over entries in row order); the values are
+// the entry ids t, the entry's row goes to erow[t]
+__global__ void k_blk_win_keys(const int32_t *sig_ptr, const int32_t *blk, int64_t M, const int32_t *win, int bb,
+                               uint64_t *keys, uint32_t *vals, int32_t *erow) {
     const int lane = threadIdx.x & 31;
     for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M;
          r += ((int64_t)gridDim.x * blockDim.x) >> 5)
         for (int32_t t = sig_ptr[r] + lane; t < sig_ptr[r + 1]; t += 32) {
-            keys[t] = ((uint64_t)(uint32_t)blk[t] << 32) | (uint32_t)win[r];
-            vals[t] = (uint32_t)r;
+            keys[t] = ((uint64_t)(uint32_t)win[r] << bb) | (uint32_t)blk[t];
+            vals[t] = (uint32_t)t;
+            erow[t] = (int32_t)r;
         }
+}
+// runs of equal (window, block) keys = the window sub-lists: flag[i] = 1 at the first entry of a run
+__global__ void k_run_flags(const uint64_t *keys, int64_t S, int32_t *flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = (i == 0 || keys[i] != keys[i - 1]) ? 1 : 0;
+}
+__global__ void k_run_starts(const int32_t *flag, const int32_t *pos, int64_t S, int32_t *rstart) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S; i += (int64_t)gridDim.x * blockDim.x)
+        if (flag[i]) rstart[pos[i]] = (int32_t)i;
+}
+// per sorted entry i (entry id e = vals[i]): xr[e] = its run [start, end), brow[i] = its row
+__global__ void k_xr_fill(const uint32_t *vals, const int32_t *flag, const int32_t *pos, const int32_t *rstart,
+                          const int32_t *erow, int64_t S, int2 *xr, int32_t *brow) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S; i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t e = vals[i];
+        const int32_t rid = pos[i] + flag[i] - 1;
+        xr[e] = make_int2(rstart[rid], rstart[rid + 1]);
+        brow[i] = erow[e];
+    }
 }
 __global__ void k_xkeys(const int32_t *sig_ptr, const int32_t *nnz, int64_t M, int32_t nt, int with_wl, uint64_t *keys,
                         uint32_t *vals) {
@@ -483,33 +505,7 @@ __device__ __forceinline__ Key xblock_argmin(Key k, Key *red) {
 }
 
 // prefix of the posting-list lengths of blocks sig_blk[c0 .. c0+nb) into pre[0..nb], list starts into bst[]
-// mwin >= 0: lists sorted by window; only window mwin's sub-range [first win >= mwin, first win > mwin)
-__device__ __forceinline__ int32_t lower_win(const int32_t *brow, const int32_t *win, int32_t lo, int32_t hi, int32_t w) {
-    while (lo < hi) {
-        const int32_t mid = (lo + hi) >> 1;
-        if (win[brow[mid]] < w) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-// Multi-window chains: the sub-range of each signature entry's posting list that lies in its own row's window
-// (the lists are sorted by window), found once per entry here -- two binary searches per entry, independent, so the
-// whole pass runs at memory throughput -- instead of inside every greedy step, where the searches of the reference
-// row's blocks were a chain of ~2 log2(list) dependent loads on the step's critical path.  Warp per row.
-__global__ void k_xrange(const int32_t *sig_ptr, const int32_t *sig_blk, int64_t M, const int32_t *bptr,
-                         const int32_t *brow, const int32_t *win, int2 *xr) {
-    const int lane = threadIdx.x & 31;
-    for (int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < M;
-         r += ((int64_t)gridDim.x * blockDim.x) >> 5) {
-        const int32_t w = win[r];
-        for (int32_t e = sig_ptr[r] + lane; e < sig_ptr[r + 1]; e += 32) {
-            const int32_t b = sig_blk[e];
-            const int32_t a = lower_win(brow, win, bptr[b], bptr[b + 1], w);
-            xr[e] = make_int2(a, lower_win(brow, win, a, bptr[b + 1], w + 1));
-        }
-    }
-}
-
+// mwin >= 0 (multi-window): only the window's sub-range of each list, xr[entry] = [start, end) (k_xr_fill)
 template <class PT>
 __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *bptr, int32_t c0, int32_t nb,
                                         PT *pre, int32_t *bst, PT *wsum, const int32_t *brow = nullptr,
@@ -519,7 +515,7 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
     int32_t len = 0;
     if (tid < nb) {
         int32_t a, e;
-        if (mwin >= 0 && xr) {                  // the window's sub-range, precomputed per signature entry (k_xrange)
+        if (mwin >= 0) {                        // the window's sub-range of the list (k_xr_fill)
             const int2 v = __ldg(xr + c0 + tid);
             a = v.x;
             e = v.y;
@@ -527,10 +523,6 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
             const int32_t b = sig_blk[c0 + tid];
             a = bptr[b];
             e = bptr[b + 1];
-            if (mwin >= 0) {
-                a = lower_win(brow, win, a, e, mwin);
-                e = lower_win(brow, win, a, e, mwin + 1);
-            }
         }
         len = e - a;
         bst[tid] = a;
@@ -560,8 +552,8 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
 
 // visit every entry of the posting lists described by (pre, bst, nb): f(row)
 // PT: prefix type -- int32 when 1024 x the longest posting list fits (the host checks), else int64
-template <class PT, class F>
-__device__ __forceinline__ void xvisit(const PT *pre, const int32_t *bst, int32_t nb, const int32_t *brow, F f) {
+template <class PT, class IT, class F>
+__device__ __forceinline__ void xvisit(const PT *pre, const int32_t *bst, int32_t nb, const IT *brow, F f) {
     const PT T = pre[nb];
     for (PT e = threadIdx.x; e < T; e += XCH_THREADS) {
         int lo = 0, hi = nb - 1;
@@ -570,19 +562,22 @@ __device__ __forceinline__ void xvisit(const PT *pre, const int32_t *bst, int32_
             if (pre[mid] <= e) lo = mid;
             else hi = mid - 1;
         }
-        f(__ldg(brow + bst[lo] + (e - pre[lo])));
+        f((int32_t)__ldg(brow + bst[lo] + (e - pre[lo])));
     }
 }
 
 // all entries of row r0's lists, chunked by XCH_THREADS blocks (re-derives the prefix; barriers inside)
-template <class PT, class F>
+// IT = int32_t: brow holds row ids (and serves the binary searches when xr is NULL); IT = uint16_t: window-local
+// row indices (k_chain_xl, xr required)
+template <class PT, class IT, class F>
 __device__ __forceinline__ void xvisit_all(int32_t r0, const int32_t *sig_ptr, const int32_t *sig_blk,
-                                           const int32_t *bptr, const int32_t *brow, PT *pre, int32_t *bst,
+                                           const int32_t *bptr, const IT *brow, PT *pre, int32_t *bst,
                                            PT *wsum, const int32_t *win, int32_t mwin, const int2 *xr, F f) {
     const int32_t bs = sig_ptr[r0], be = sig_ptr[r0 + 1];
     for (int32_t c0 = bs; c0 < be; c0 += XCH_THREADS) {
         const int32_t nb = min(XCH_THREADS, be - c0);
-        xprefix(sig_blk, bptr, c0, nb, pre, bst, wsum, brow, win, mwin, xr);
+        xprefix(sig_blk, bptr, c0, nb, pre, bst, wsum,
+                std::is_same<IT, int32_t>::value ? reinterpret_cast<const int32_t *>(brow) : nullptr, win, mwin, xr);
         xvisit(pre, bst, nb, brow, f);
         __syncthreads();
     }
@@ -811,6 +806,198 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     }
 }
 
+// k_chain_xl: k_chain_x for windows of at most XL_MAX rows (every windowed chain policy but HYBRID_2_2) with the
+// window held in shared memory.  The posting-list entries carry the row's index inside its window (bloc, 16 bit),
+// so the per-step state -- the |b_r ∩ b_ref| counters, the placed flags, |b_r|, wl_r, the row ids and the
+// (|b|, [wl,] r) order -- is indexed locally: the count pass is a shared-memory atomic, the score pass and the u*
+// search read shared memory, where k_chain_x makes global atomics and L2 round trips on every step's critical path.
+// Same definitions, same keys, same argmin as k_chain_x (DESIGN.md §6 "exact chains"): bit-identical permutations.
+constexpr int XL_MAX = 4096;
+constexpr size_t XL_SMEM = (size_t)XL_MAX * (4 * 4 + 2 * 4) + XL_MAX / 8;   // r, nb, wl, o, cnt[2]; placed bits
+
+__global__ void k_lpos(const int32_t *base, const int32_t *seg, int64_t W, int64_t M, const int32_t *win,
+                       int32_t *lpos) {
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < M; q += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t r = base[q], w = win[r];
+        lpos[r] = (int32_t)(q - (seg ? (int64_t)seg[w] : (int64_t)w * W));
+    }
+}
+__global__ void k_bloc(const int32_t *brow, int64_t S, const int32_t *lpos, uint16_t *bloc) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S; i += (int64_t)gridDim.x * blockDim.x)
+        bloc[i] = (uint16_t)lpos[brow[i]];
+}
+
+template <int MODE, class PT>
+__global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base, const int32_t *seg, int64_t W,
+                                                             int64_t M, const int32_t *sig_ptr,
+                                                             const int32_t *sig_blk, const int32_t *bptr,
+                                                             const uint16_t *bloc, const int2 *xr,
+                                                             const uint32_t *ord, const int32_t *lpos,
+                                                             const int32_t *nnz, int32_t nt, int32_t nw,
+                                                             int32_t *perm) {
+    extern __shared__ uint32_t xl[];
+    __shared__ PT pre[2][XCH_CACHE + 1];
+    __shared__ int32_t bst[2][XCH_CACHE];
+    __shared__ PT wsum[32];
+    __shared__ Key red[2][XCH_THREADS / 32];
+    __shared__ int32_t s_ptr;
+    const int32_t w = (int32_t)blockIdx.x;
+    const int64_t s0 = seg ? seg[w] : (int64_t)w * W, s1 = seg ? seg[w + 1] : min(s0 + W, M);
+    const int32_t n = (int32_t)(s1 - s0);
+    if (n <= 0) return;
+    int32_t *r_s = reinterpret_cast<int32_t *>(xl);           // local index -> row id
+    uint32_t *nb_s = xl + XL_MAX;                            // |b_r|
+    uint32_t *wl_s = xl + 2 * XL_MAX;                        // wl_r
+    uint32_t *o_s = xl + 3 * XL_MAX;                         // the window's (|b|, [wl,] r) order, local indices
+    int32_t *cnt_s = reinterpret_cast<int32_t *>(xl + 4 * XL_MAX);   // [2][XL_MAX] counters by step parity
+    uint32_t *pl_s = xl + 6 * XL_MAX;                        // placed flags
+    for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
+        const int32_t r = base[s0 + a];
+        r_s[a] = r;
+        nb_s[a] = (uint32_t)(sig_ptr[r + 1] - sig_ptr[r]);
+        wl_s[a] = (uint32_t)((nnz[r] + nt - 1) / nt);
+        o_s[a] = (uint32_t)lpos[ord[s0 + a]];
+        cnt_s[a] = 0;
+        cnt_s[XL_MAX + a] = 0;
+    }
+    for (int32_t a = threadIdx.x; a < (n + 31) / 32; a += XCH_THREADS) pl_s[a] = 0u;
+    __syncthreads();
+    auto placed = [&](int32_t l) -> bool { return (pl_s[l >> 5] >> (l & 31)) & 1u; };
+    int32_t *out = perm + s0;
+    constexpr bool WARPREF = MODE == C_WARP || MODE == C_H23;   // Hamming reference out[q - nw], else prev
+    constexpr bool WLTIE = MODE == C_H21 || MODE == C_H23;      // tie: |wl_r - wl_prev|
+    const int32_t nfirst = WARPREF ? min(n, nw) : 1;
+    Key best;
+    int32_t prev = -1, prev_l = -1, pref = -1;
+    for (int32_t q = 0; q < nfirst; ++q) {
+        best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
+        for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
+            if (q > 0 && placed(a)) continue;
+            const Key c{wl_s[a], 0u, (uint32_t)r_s[a], (uint32_t)a};
+            if (key_less(c, best)) best = c;
+        }
+        const Key w0 = xblock_argmin(best, red[q & 1]);
+        prev = (int32_t)w0.r;
+        prev_l = (int32_t)w0.a;
+        if (threadIdx.x == 0) {
+            out[q] = prev;
+            pl_s[prev_l >> 5] |= 1u << (prev_l & 31);
+            s_ptr = 0;
+        }
+        __syncthreads();
+    }
+    bool cached_pp = false;
+    for (int32_t q = nfirst; q < n; ++q) {
+        const int buf = q & 1;
+        int32_t *cc = cnt_s + buf * XL_MAX, *co = cnt_s + (buf ^ 1) * XL_MAX;
+        const int32_t ref = WARPREF ? (nw == 1 ? prev : out[q - nw]) : prev;
+        const int32_t bs = sig_ptr[ref], be = sig_ptr[ref + 1];
+        const uint32_t cp = (uint32_t)(be - bs);
+        const bool cached = be - bs <= XCH_CACHE;
+        if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, nullptr, nullptr, w, xr);
+        if (pref >= 0) {
+            auto reset = [&](int32_t l) { co[l] = 0; };
+            if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], bloc, reset);
+            else xvisit_all(pref, sig_ptr, sig_blk, bptr, bloc, pre[buf ^ 1], bst[buf ^ 1], wsum, nullptr, w, xr, reset);
+        }
+        auto count = [&](int32_t l) {
+            if (l != prev_l && !placed(l)) atomicAdd(cc + l, 1);
+        };
+        if (cached) xvisit(pre[buf], bst[buf], be - bs, bloc, count);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, bloc, pre[buf], bst[buf], wsum, nullptr, w, xr, count);
+        __syncthreads();
+        const uint32_t wlp = WLTIE ? wl_s[prev_l] : 0u;
+        auto keyof = [&](int32_t l) -> Key {
+            Key k{cp + nb_s[l] - 2u * (uint32_t)cc[l], 0u, (uint32_t)r_s[l], (uint32_t)l};
+            if (WLTIE) {
+                const uint32_t x = wl_s[l];
+                k.k2 = x > wlp ? x - wlp : wlp - x;
+            }
+            return k;
+        };
+        best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
+        auto score = [&](int32_t l) {
+            if (l != prev_l && !placed(l)) {
+                const Key k = keyof(l);
+                if (key_less(k, best)) best = k;
+            }
+        };
+        if (cached) xvisit(pre[buf], bst[buf], be - bs, bloc, score);
+        else xvisit_all(ref, sig_ptr, sig_blk, bptr, bloc, pre[buf], bst[buf], wsum, nullptr, w, xr, score);
+        // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
+        if (threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            int32_t ptr = s_ptr;
+            while (ptr < n) {
+                const bool pl = ptr + lane < n ? placed((int32_t)o_s[ptr + lane]) : false;
+                const unsigned m = __ballot_sync(0xffffffffu, !pl && ptr + lane < n);
+                if (m) { ptr += __ffs(m) - 1; break; }
+                ptr = min(ptr + 32, n);
+            }
+            __syncwarp();
+            if (lane == 0) s_ptr = ptr;
+            if (ptr < n) {
+                if (!WLTIE) {
+                    if (lane == 0) {
+                        const Key k = keyof((int32_t)o_s[ptr]);
+                        if (key_less(k, best)) best = k;
+                    }
+                } else {
+                    const uint32_t b0 = nb_s[o_s[ptr]];
+                    int32_t lo = ptr, hi = n;                     // class end: first index with |b| > b0
+                    while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (nb_s[o_s[mid]] > b0) hi = mid; else lo = mid + 1; }
+                    const int32_t cend = lo;
+                    lo = ptr; hi = cend;                          // lb: first index with wl >= wl_prev
+                    while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (wl_s[o_s[mid]] >= wlp) hi = mid; else lo = mid + 1; }
+                    const int32_t lb = lo;
+                    for (int32_t i = lb; i < cend; i += 32) {      // up: first unplaced in [lb, cend)
+                        const bool ok = i + lane < cend && !placed((int32_t)o_s[i + lane]);
+                        const unsigned m = __ballot_sync(0xffffffffu, ok);
+                        if (m) {
+                            if (lane == 0) {
+                                const Key k = keyof((int32_t)o_s[i + __ffs(m) - 1]);
+                                if (key_less(k, best)) best = k;
+                            }
+                            break;
+                        }
+                    }
+                    int32_t d = -1;                               // down: last unplaced in [ptr, lb)
+                    for (int32_t i = lb - 1; i >= ptr; i -= 32) {
+                        const bool ok = i - lane >= ptr && !placed((int32_t)o_s[i - lane]);
+                        const unsigned m = __ballot_sync(0xffffffffu, ok);
+                        if (m) { d = i - (__ffs(m) - 1); break; }
+                    }
+                    if (d >= 0) {                                 // then the first unplaced of its wl run
+                        const uint32_t wd = wl_s[o_s[d]];
+                        lo = ptr; hi = d;
+                        while (lo < hi) { const int32_t mid = (lo + hi) >> 1; if (wl_s[o_s[mid]] >= wd) hi = mid; else lo = mid + 1; }
+                        for (int32_t i = lo; i <= d; i += 32) {
+                            const bool ok = i + lane <= d && !placed((int32_t)o_s[i + lane]);
+                            const unsigned m = __ballot_sync(0xffffffffu, ok);
+                            if (m) {
+                                if (lane == 0) {
+                                    const Key k = keyof((int32_t)o_s[i + __ffs(m) - 1]);
+                                    if (key_less(k, best)) best = k;
+                                }
+                                break;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        const Key nx = xblock_argmin(best, red[buf]);
+        if (threadIdx.x == 0) {
+            out[q] = (int32_t)nx.r;
+            pl_s[nx.a >> 5] |= 1u << (nx.a & 31);
+        }
+        pref = ref;
+        cached_pp = cached;
+        prev = (int32_t)nx.r;
+        prev_l = (int32_t)nx.a;
+    }
+}
+
 // seg != nullptr: HYBRID_1's nseg segments (positions seg[k] .. seg[k+1]) instead of windows of W
 spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg, int64_t nseg, int64_t W, int64_t M,
                                const Signatures &sig, const int32_t *nnz, const spmm_params &p, int64_t N,
@@ -834,17 +1021,35 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
     }
     SPMM_TRY(exclusive_scan_i32(bcnt.as<int32_t>(), bptr.as<int32_t>(), nblk, nullptr, s));   // bptr[nblk] = S
     SPMM_TRY(brow.alloc(std::max<int64_t>(sig.S, 1) * sizeof(int32_t), s));
+    DevBuf xr;
     if (sig.S > 0 && nwin > 1) {
-        DevBuf ek;
+        DevBuf ek, vals, erow, flag, pos, rstart;
         SPMM_TRY(ek.alloc(sig.S * sizeof(uint64_t), s));
-        k_blk_win_keys<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
-                                                          win.as<int32_t>(), ek.as<uint64_t>(),
-                                                          reinterpret_cast<uint32_t *>(brow.as<int32_t>()));
-        SPMM_CUDA(cudaGetLastError());
-        int bb = 0;
+        SPMM_TRY(vals.alloc(sig.S * sizeof(uint32_t), s));
+        SPMM_TRY(erow.alloc(sig.S * sizeof(int32_t), s));
+        int bb = 0, wb = 0;
         while (bb < 32 && ((uint64_t)nblk >> bb) != 0) ++bb;
-        SPMM_TRY(radix_sort_pairs(ek.as<uint64_t>(), reinterpret_cast<uint32_t *>(brow.as<int32_t>()), sig.S, 0,
-                                  32 + bb, s));
+        while (wb < 32 && ((uint64_t)nwin >> wb) != 0) ++wb;
+        k_blk_win_keys<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
+                                                          win.as<int32_t>(), bb, ek.as<uint64_t>(),
+                                                          vals.as<uint32_t>(), erow.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        SPMM_TRY(radix_sort_pairs(ek.as<uint64_t>(), vals.as<uint32_t>(), sig.S, 0, bb + wb, s));
+        SPMM_TRY(flag.alloc(sig.S * sizeof(int32_t), s));
+        SPMM_TRY(pos.alloc((sig.S + 1) * sizeof(int32_t), s));
+        k_run_flags<<<grid_for(sig.S, 256), 256, 0, s>>>(ek.as<uint64_t>(), sig.S, flag.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
+        int32_t nruns = 0;
+        SPMM_TRY(exclusive_scan_i32(flag.as<int32_t>(), pos.as<int32_t>(), sig.S, &nruns, s));
+        SPMM_TRY(rstart.alloc(((int64_t)nruns + 1) * sizeof(int32_t), s));
+        k_run_starts<<<grid_for(sig.S, 256), 256, 0, s>>>(flag.as<int32_t>(), pos.as<int32_t>(), sig.S,
+                                                          rstart.as<int32_t>());
+        k_set_last<<<1, 1, 0, s>>>(rstart.as<int32_t>(), nruns, (int32_t)sig.S);
+        SPMM_TRY(xr.alloc(sig.S * sizeof(int2), s));
+        k_xr_fill<<<grid_for(sig.S, 256), 256, 0, s>>>(vals.as<uint32_t>(), flag.as<int32_t>(), pos.as<int32_t>(),
+                                                       rstart.as<int32_t>(), erow.as<int32_t>(), sig.S,
+                                                       xr.as<int2>(), brow.as<int32_t>());
+        SPMM_CUDA(cudaGetLastError());
     } else if (sig.S > 0) {
         k_blk_fill<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M,
                                                       bptr.as<int32_t>(), bcur.as<int32_t>(), brow.as<int32_t>());
@@ -880,16 +1085,32 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
              : k_chain_x<C_CTA, PT>;                                    // HYBRID_1 = C_CTA over segments
     };
     auto kern = wide ? pick(int64_t{}) : pick(int32_t{});
-    DevBuf xr;
-#ifdef SPMM_EXP_NO_XRANGE   // A/B variant: binary searches inside the greedy steps (round 2 before k_xrange)
-    if (false) {
+    // windows of at most XL_MAX rows (HYBRID_1's segments are cut at the window size): k_chain_xl
+    const int64_t wmax = seg ? (int64_t)p.window : W;
+#ifdef SPMM_EXP_NO_XL   // A/B variant: k_chain_x with global counters for every window size
+    const bool local = false;
 #else
-    if (nwin > 1 && sig.S > 0) {
+    const bool local = nwin > 1 && sig.S > 0 && mode != C_H22 && wmax > 0 && wmax <= XL_MAX;
 #endif
-        SPMM_TRY(xr.alloc(sig.S * sizeof(int2), s));
-        k_xrange<<<grid_warps(M, 256), 256, 0, s>>>(sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(), M, bptr.as<int32_t>(),
-                                                    brow.as<int32_t>(), win.as<int32_t>(), xr.as<int2>());
+    if (local) {
+        DevBuf lpos, bloc;
+        SPMM_TRY(lpos.alloc(M * sizeof(int32_t), s));
+        SPMM_TRY(bloc.alloc(sig.S * sizeof(uint16_t), s));
+        k_lpos<<<grid_for(M, 256), 256, 0, s>>>(base, seg, W, M, win.as<int32_t>(), lpos.as<int32_t>());
+        k_bloc<<<grid_for(sig.S, 256), 256, 0, s>>>(brow.as<int32_t>(), sig.S, lpos.as<int32_t>(), bloc.as<uint16_t>());
         SPMM_CUDA(cudaGetLastError());
+        auto pickl = [&](auto pt) {
+            using PT = decltype(pt);
+            return mode == C_H21 ? k_chain_xl<C_H21, PT> : mode == C_WARP ? k_chain_xl<C_WARP, PT>
+                 : mode == C_H23 ? k_chain_xl<C_H23, PT> : k_chain_xl<C_CTA, PT>;   // HYBRID_1 = C_CTA
+        };
+        auto kl = wide ? pickl(int64_t{}) : pickl(int32_t{});
+        SPMM_CUDA(cudaFuncSetAttribute(kl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)XL_SMEM));
+        kl<<<(unsigned)nwin, XCH_THREADS, XL_SMEM, s>>>(base, seg, W, M, sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(),
+                                                        bptr.as<int32_t>(), bloc.as<uint16_t>(), xr.as<int2>(),
+                                                        ord.as<uint32_t>(), lpos.as<int32_t>(), nnz, p.nt, p.nw, perm);
+        SPMM_CUDA(cudaGetLastError());
+        return SPMM_OK;
     }
     kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
