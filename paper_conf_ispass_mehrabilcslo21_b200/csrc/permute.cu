@@ -813,7 +813,8 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
 // search read shared memory, where k_chain_x makes global atomics and L2 round trips on every step's critical path.
 // Same definitions, same keys, same argmin as k_chain_x (DESIGN.md §6 "exact chains"): bit-identical permutations.
 constexpr int XL_MAX = 4096;
-constexpr size_t XL_SMEM = (size_t)XL_MAX * (4 * 4 + 2 * 4) + XL_MAX / 8;   // r, nb, wl, o, cnt[2]; placed bits
+// r, nb, wl, o (u32), cnt[2] (i32), placed bits, touched lists[2] (u16)
+constexpr size_t XL_SMEM = (size_t)XL_MAX * (4 * 4 + 2 * 4) + XL_MAX / 8 + (size_t)XL_MAX * 2 * 2;
 
 __global__ void k_lpos(const int32_t *base, const int32_t *seg, int64_t W, int64_t M, const int32_t *win,
                        int32_t *lpos) {
@@ -851,6 +852,10 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
     uint32_t *o_s = xl + 3 * XL_MAX;                         // the window's (|b|, [wl,] r) order, local indices
     int32_t *cnt_s = reinterpret_cast<int32_t *>(xl + 4 * XL_MAX);   // [2][XL_MAX] counters by step parity
     uint32_t *pl_s = xl + 6 * XL_MAX;                        // placed flags
+    // the distinct rows a step's count pass touched (its candidate set T, listed on first touch): the score pass
+    // and the next step's counter reset walk this list instead of re-walking the posting lists
+    uint16_t *tl_s = reinterpret_cast<uint16_t *>(pl_s + XL_MAX / 32);   // [2][XL_MAX]
+    __shared__ int32_t s_nt[2];
     for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
         const int32_t r = base[s0 + a];
         r_s[a] = r;
@@ -861,6 +866,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         cnt_s[XL_MAX + a] = 0;
     }
     for (int32_t a = threadIdx.x; a < (n + 31) / 32; a += XCH_THREADS) pl_s[a] = 0u;
+    if (threadIdx.x < 2) s_nt[threadIdx.x] = 0;
     __syncthreads();
     auto placed = [&](int32_t l) -> bool { return (pl_s[l >> 5] >> (l & 31)) & 1u; };
     int32_t *out = perm + s0;
@@ -868,7 +874,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
     constexpr bool WLTIE = MODE == C_H21 || MODE == C_H23;      // tie: |wl_r - wl_prev|
     const int32_t nfirst = WARPREF ? min(n, nw) : 1;
     Key best;
-    int32_t prev = -1, prev_l = -1, pref = -1;
+    int32_t prev = -1, prev_l = -1;
     for (int32_t q = 0; q < nfirst; ++q) {
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
         for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
@@ -886,7 +892,6 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         }
         __syncthreads();
     }
-    bool cached_pp = false;
     for (int32_t q = nfirst; q < n; ++q) {
         const int buf = q & 1;
         int32_t *cc = cnt_s + buf * XL_MAX, *co = cnt_s + (buf ^ 1) * XL_MAX;
@@ -894,14 +899,15 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         const int32_t bs = sig_ptr[ref], be = sig_ptr[ref + 1];
         const uint32_t cp = (uint32_t)(be - bs);
         const bool cached = be - bs <= XCH_CACHE;
+        uint16_t *tl = tl_s + buf * XL_MAX, *tlo = tl_s + (buf ^ 1) * XL_MAX;
+        // the previous step's touched rows: reset their counters (other buffer); this step's list restarts (every
+        // reader of s_nt[buf] -- step q-1's reset -- is behind the barriers of step q-1's passes)
+        for (int32_t i = threadIdx.x; i < s_nt[buf ^ 1]; i += XCH_THREADS) co[tlo[i]] = 0;
+        if (threadIdx.x == 0) s_nt[buf] = 0;
+        __syncthreads();
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, nullptr, nullptr, w, xr);
-        if (pref >= 0) {
-            auto reset = [&](int32_t l) { co[l] = 0; };
-            if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], bloc, reset);
-            else xvisit_all(pref, sig_ptr, sig_blk, bptr, bloc, pre[buf ^ 1], bst[buf ^ 1], wsum, nullptr, w, xr, reset);
-        }
         auto count = [&](int32_t l) {
-            if (l != prev_l && !placed(l)) atomicAdd(cc + l, 1);
+            if (l != prev_l && !placed(l) && atomicAdd(cc + l, 1) == 0) tl[atomicAdd(&s_nt[buf], 1)] = (uint16_t)l;
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, bloc, count);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, bloc, pre[buf], bst[buf], wsum, nullptr, w, xr, count);
@@ -922,8 +928,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
                 if (key_less(k, best)) best = k;
             }
         };
-        if (cached) xvisit(pre[buf], bst[buf], be - bs, bloc, score);
-        else xvisit_all(ref, sig_ptr, sig_blk, bptr, bloc, pre[buf], bst[buf], wsum, nullptr, w, xr, score);
+        for (int32_t i = threadIdx.x; i < s_nt[buf]; i += XCH_THREADS) score((int32_t)tl[i]);
         // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
         if (threadIdx.x < 32) {
             const int lane = threadIdx.x;
@@ -991,8 +996,6 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
             out[q] = (int32_t)nx.r;
             pl_s[nx.a >> 5] |= 1u << (nx.a & 31);
         }
-        pref = ref;
-        cached_pp = cached;
         prev = (int32_t)nx.r;
         prev_l = (int32_t)nx.a;
     }
