@@ -535,17 +535,15 @@ __device__ __forceinline__ void xprefix(const int32_t *sig_blk, const int32_t *b
     }
     if (lane == 31) wsum[wid] = x;
     __syncthreads();
-    if (wid == 0) {
-        PT w = wsum[lane];
+    // every warp scans the 32 warp totals itself (one barrier fewer than a warp-0 scan + broadcast)
+    PT w = wsum[lane];
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const PT y = __shfl_up_sync(0xffffffffu, w, o);
-            if (lane >= o) w += y;
-        }
-        wsum[lane] = w;
+    for (int o = 1; o < 32; o <<= 1) {
+        const PT y = __shfl_up_sync(0xffffffffu, w, o);
+        if (lane >= o) w += y;
     }
-    __syncthreads();
-    pre[tid + 1] = x + (wid ? wsum[wid - 1] : 0);
+    const PT off = __shfl_sync(0xffffffffu, w, (wid + 31) & 31);
+    pre[tid + 1] = x + (wid ? off : 0);
     if (tid == 0) pre[0] = 0;
     __syncthreads();
 }
@@ -903,8 +901,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         // the previous step's touched rows: reset their counters (other buffer); this step's list restarts (every
         // reader of s_nt[buf] -- step q-1's reset -- is behind the barriers of step q-1's passes)
         for (int32_t i = threadIdx.x; i < s_nt[buf ^ 1]; i += XCH_THREADS) co[tlo[i]] = 0;
-        if (threadIdx.x == 0) s_nt[buf] = 0;
-        __syncthreads();
+        if (threadIdx.x == 0) s_nt[buf] = 0;   // ordered before the count pass by xprefix's barriers
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, nullptr, nullptr, w, xr);
         auto count = [&](int32_t l) {
             if (l != prev_l && !placed(l) && atomicAdd(cc + l, 1) == 0) tl[atomicAdd(&s_nt[buf], 1)] = (uint16_t)l;
