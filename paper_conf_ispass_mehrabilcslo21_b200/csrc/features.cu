@@ -121,29 +121,66 @@ __global__ void k_popcount_rows(const uint32_t *Dmap, int64_t words, unsigned lo
     if ((threadIdx.x & 31) == 0) atomicAdd(&D[blockIdx.x], c);
 }
 
-// adjacent-vector distance: Hamming(p, p+1) = |b_p| + |b_{p+1}| - 2|common|, merge of the two sorted
-// (non-decreasing, duplicated) block sequences; thread per pair
+// adjacent-vector distance: Hamming(p, p+1) = |b_p| + |b_{p+1}| - 2|common|.  Pairs whose rows hold at most
+// ADJ_SHORT nnz together: thread per pair, merge of the two sorted (non-decreasing, duplicated) block sequences.
+// Longer pairs (power-law hub rows, up to 10^5 nnz): warp per pair -- the lanes take the distinct blocks of the
+// shorter row (run starts) and binary-search each in the longer row's columns -- so no single thread walks a hub row.
+constexpr int32_t ADJ_SHORT = 256;
+__device__ __forceinline__ int32_t adj_common_merge(const OrigCSR &A, int64_t p, int32_t bw) {
+    int32_t i = A.begin(p), ie = A.end(p), j = A.begin(p + 1), je = A.end(p + 1);
+    int32_t common = 0;
+    while (i < ie && j < je) {
+        const int32_t x = A.col(i) / bw, y = A.col(j) / bw;
+        if (x == y) {
+            ++common;
+            while (i < ie && A.col(i) / bw == x) ++i;
+            while (j < je && A.col(j) / bw == y) ++j;
+        } else if (x < y) {
+            ++i;
+        } else {
+            ++j;
+        }
+    }
+    return common;
+}
 __global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk_row, Stats *st) {
+    const int lane = threadIdx.x & 31;
     for (int64_t p0 = (int64_t)blockIdx.x * blockDim.x; p0 < M - 1; p0 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t p = p0 + threadIdx.x;
         long long hd = 0;
         const bool in = p < M - 1;
+        bool lng = false;
+        int32_t b0 = 0, e0 = 0, b1 = 0, e1 = 0;
         if (in) {
-            int32_t i = A.begin(p), ie = A.end(p), j = A.begin(p + 1), je = A.end(p + 1);
-            int32_t common = 0;
-            while (i < ie && j < je) {
-                const int32_t x = A.col(i) / bw, y = A.col(j) / bw;
-                if (x == y) {
-                    ++common;
-                    while (i < ie && A.col(i) / bw == x) ++i;
-                    while (j < je && A.col(j) / bw == y) ++j;
-                } else if (x < y) {
-                    ++i;
-                } else {
-                    ++j;
+            b0 = A.begin(p); e0 = A.end(p); b1 = A.begin(p + 1); e1 = A.end(p + 1);
+            lng = (e0 - b0) + (e1 - b1) > ADJ_SHORT;
+            if (!lng) hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * adj_common_merge(A, p, bw);
+        }
+        // the warp's long pairs, one after another, all lanes together
+        unsigned todo = __ballot_sync(0xffffffffu, lng);
+        while (todo) {
+            const int src = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const int32_t sb0 = __shfl_sync(0xffffffffu, b0, src), se0 = __shfl_sync(0xffffffffu, e0, src);
+            const int32_t sb1 = __shfl_sync(0xffffffffu, b1, src), se1 = __shfl_sync(0xffffffffu, e1, src);
+            const bool first_short = se0 - sb0 <= se1 - sb1;
+            const int32_t sb = first_short ? sb0 : sb1, se = first_short ? se0 : se1;   // scanned row
+            const int32_t tb = first_short ? sb1 : sb0, te = first_short ? se1 : se0;   // searched row
+            int32_t c = 0;
+            for (int32_t i = sb + lane; i < se; i += 32) {
+                const int32_t x = A.col(i) / bw;
+                if (i > sb && A.col(i - 1) / bw == x) continue;   // not the first column of its block
+                int32_t lo = tb, hi = te;                           // first column with block >= x
+                while (lo < hi) {
+                    const int32_t mid = (lo + hi) >> 1;
+                    if (A.col(mid) / bw < x) lo = mid + 1;
+                    else hi = mid;
                 }
+                c += lo < te && A.col(lo) / bw == x;
             }
-            hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * common;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+            if (lane == src) hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * c;
         }
         warp_stats(st, hd, in);
     }
