@@ -804,7 +804,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     }
 }
 
-// k_chain_xl: k_chain_x for windows of at most XL_MAX rows (every windowed chain policy but HYBRID_2_2) with the
+// k_chain_xl: k_chain_x for windows of at most XL_MAX rows (every windowed chain policy) with the
 // window held in shared memory.  The posting-list entries carry the row's index inside its window (bloc, 16 bit),
 // so the per-step state -- the |b_r ∩ b_ref| counters, the placed flags, |b_r|, wl_r, the row ids and the
 // (|b|, [wl,] r) order -- is indexed locally: the count pass is a shared-memory atomic, the score pass and the u*
@@ -813,6 +813,8 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
 constexpr int XL_MAX = 4096;
 // r, nb, wl, o (u32), cnt[2] (i32), placed bits, touched lists[2] (u16)
 constexpr size_t XL_SMEM = (size_t)XL_MAX * (4 * 4 + 2 * 4) + XL_MAX / 8 + (size_t)XL_MAX * 2 * 2;
+// HYBRID_2_2's second reference: counters[2] (i32) and touched lists[2] (u16)
+constexpr size_t XL_SMEM_H22 = XL_SMEM + (size_t)XL_MAX * (2 * 4 + 2 * 2);
 
 __global__ void k_lpos(const int32_t *base, const int32_t *seg, int64_t W, int64_t M, const int32_t *win,
                        int32_t *lpos) {
@@ -840,6 +842,13 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
     __shared__ PT wsum[32];
     __shared__ Key red[2][XCH_THREADS / 32];
     __shared__ int32_t s_ptr;
+    // HYBRID_2_2: key (ham(r, prev), q >= nw ? ham(r, out[q - nw]) : 0, r) -- a second reference ref2 with
+    // its own counters and touched list; the argmin lies in T1 ∪ (T2 ∩ class b0) ∪ {u*}
+    constexpr bool TWOREF = MODE == C_H22;
+    constexpr int C2 = TWOREF ? XCH_CACHE : 1;
+    __shared__ PT pre2[C2 + 1];
+    __shared__ int32_t bst2[C2];
+    __shared__ int32_t s_nt2[2];
     const int32_t w = (int32_t)blockIdx.x;
     const int64_t s0 = seg ? seg[w] : (int64_t)w * W, s1 = seg ? seg[w + 1] : min(s0 + W, M);
     const int32_t n = (int32_t)(s1 - s0);
@@ -854,6 +863,8 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
     // and the next step's counter reset walk this list instead of re-walking the posting lists
     uint16_t *tl_s = reinterpret_cast<uint16_t *>(pl_s + XL_MAX / 32);   // [2][XL_MAX]
     __shared__ int32_t s_nt[2];
+    int32_t *cnt2_s = reinterpret_cast<int32_t *>(tl_s + 2 * XL_MAX);   // [2][XL_MAX] (HYBRID_2_2 only)
+    uint16_t *tl2_s = reinterpret_cast<uint16_t *>(cnt2_s + 2 * XL_MAX);  // [2][XL_MAX] (HYBRID_2_2 only)
     for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
         const int32_t r = base[s0 + a];
         r_s[a] = r;
@@ -862,9 +873,13 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         o_s[a] = (uint32_t)lpos[ord[s0 + a]];
         cnt_s[a] = 0;
         cnt_s[XL_MAX + a] = 0;
+        if (TWOREF) {
+            cnt2_s[a] = 0;
+            cnt2_s[XL_MAX + a] = 0;
+        }
     }
     for (int32_t a = threadIdx.x; a < (n + 31) / 32; a += XCH_THREADS) pl_s[a] = 0u;
-    if (threadIdx.x < 2) s_nt[threadIdx.x] = 0;
+    if (threadIdx.x < 2) s_nt[threadIdx.x] = s_nt2[threadIdx.x] = 0;
     __syncthreads();
     auto placed = [&](int32_t l) -> bool { return (pl_s[l >> 5] >> (l & 31)) & 1u; };
     int32_t *out = perm + s0;
@@ -902,12 +917,33 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
         // reader of s_nt[buf] -- step q-1's reset -- is behind the barriers of step q-1's passes)
         for (int32_t i = threadIdx.x; i < s_nt[buf ^ 1]; i += XCH_THREADS) co[tlo[i]] = 0;
         if (threadIdx.x == 0) s_nt[buf] = 0;   // ordered before the count pass by xprefix's barriers
+        int32_t *cc2 = cnt2_s + buf * XL_MAX;
+        uint16_t *tl2 = tl2_s + buf * XL_MAX;
+        if constexpr (TWOREF) {
+            int32_t *co2 = cnt2_s + (buf ^ 1) * XL_MAX;
+            const uint16_t *tl2o = tl2_s + (buf ^ 1) * XL_MAX;
+            for (int32_t i = threadIdx.x; i < s_nt2[buf ^ 1]; i += XCH_THREADS) co2[tl2o[i]] = 0;
+            if (threadIdx.x == 0) s_nt2[buf] = 0;
+        }
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, nullptr, nullptr, w, xr);
         auto count = [&](int32_t l) {
             if (l != prev_l && !placed(l) && atomicAdd(cc + l, 1) == 0) tl[atomicAdd(&s_nt[buf], 1)] = (uint16_t)l;
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, bloc, count);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, bloc, pre[buf], bst[buf], wsum, nullptr, w, xr, count);
+        int32_t ref2 = -1;
+        uint32_t cp2 = 0;
+        if constexpr (TWOREF) {
+            ref2 = q >= nw ? (nw == 1 ? prev : out[q - nw]) : -1;
+            if (ref2 >= 0) {
+                cp2 = (uint32_t)(sig_ptr[ref2 + 1] - sig_ptr[ref2]);
+                __syncthreads();   // pre2 / bst2 / wsum of a previous pass are free (xvisit_all re-derives them)
+                xvisit_all(ref2, sig_ptr, sig_blk, bptr, bloc, pre2, bst2, wsum, nullptr, w, xr, [&](int32_t l) {
+                    if (l != prev_l && !placed(l) && atomicAdd(cc2 + l, 1) == 0)
+                        tl2[atomicAdd(&s_nt2[buf], 1)] = (uint16_t)l;
+                });
+            }
+        }
         __syncthreads();
         const uint32_t wlp = WLTIE ? wl_s[prev_l] : 0u;
         auto keyof = [&](int32_t l) -> Key {
@@ -916,6 +952,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
                 const uint32_t x = wl_s[l];
                 k.k2 = x > wlp ? x - wlp : wlp - x;
             }
+            if (TWOREF && ref2 >= 0) k.k2 = cp2 + nb_s[l] - 2u * (uint32_t)cc2[l];
             return k;
         };
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
@@ -926,6 +963,34 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_xl(const int32_t *base
             }
         };
         for (int32_t i = threadIdx.x; i < s_nt[buf]; i += XCH_THREADS) score((int32_t)tl[i]);
+        if constexpr (TWOREF) {
+            if (ref2 >= 0) {
+                // T2 ∩ class b0: b0 = |b| of the first unplaced row of the (|b|, r) order
+                if (threadIdx.x < 32) {
+                    const int lane = threadIdx.x;
+                    int32_t ptr = s_ptr;
+                    while (ptr < n) {
+                        const bool pl = ptr + lane < n ? placed((int32_t)o_s[ptr + lane]) : false;
+                        const unsigned m = __ballot_sync(0xffffffffu, !pl && ptr + lane < n);
+                        if (m) { ptr += __ffs(m) - 1; break; }
+                        ptr = min(ptr + 32, n);
+                    }
+                    __syncwarp();
+                    if (lane == 0) s_ptr = ptr;
+                }
+                __syncthreads();
+                const int32_t ptr = s_ptr;
+                const uint32_t b0 = ptr < n ? nb_s[o_s[ptr]] : 0xffffffffu;
+                __syncthreads();   // everyone has read s_ptr before warp 0 may rewrite it below
+                for (int32_t i = threadIdx.x; i < s_nt2[buf]; i += XCH_THREADS) {
+                    const int32_t l = (int32_t)tl2[i];
+                    if (l != prev_l && !placed(l) && nb_s[l] == b0) {
+                        const Key k = keyof(l);
+                        if (key_less(k, best)) best = k;
+                    }
+                }
+            }
+        }
         // u*: the first unplaced row of the (|b|, [wl,] r) order (placed rows before s_ptr stay placed)
         if (threadIdx.x < 32) {
             const int lane = threadIdx.x;
@@ -1090,7 +1155,7 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
 #ifdef SPMM_EXP_NO_XL   // A/B variant: k_chain_x with global counters for every window size
     const bool local = false;
 #else
-    const bool local = nwin > 1 && sig.S > 0 && mode != C_H22 && wmax > 0 && wmax <= XL_MAX;
+    const bool local = nwin > 1 && sig.S > 0 && wmax > 0 && wmax <= XL_MAX;
 #endif
     if (local) {
         DevBuf lpos, bloc;
@@ -1102,11 +1167,13 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
         auto pickl = [&](auto pt) {
             using PT = decltype(pt);
             return mode == C_H21 ? k_chain_xl<C_H21, PT> : mode == C_WARP ? k_chain_xl<C_WARP, PT>
-                 : mode == C_H23 ? k_chain_xl<C_H23, PT> : k_chain_xl<C_CTA, PT>;   // HYBRID_1 = C_CTA
+                 : mode == C_H23 ? k_chain_xl<C_H23, PT> : mode == C_H22 ? k_chain_xl<C_H22, PT>
+                 : k_chain_xl<C_CTA, PT>;                                   // HYBRID_1 = C_CTA
         };
         auto kl = wide ? pickl(int64_t{}) : pickl(int32_t{});
-        SPMM_CUDA(cudaFuncSetAttribute(kl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)XL_SMEM));
-        kl<<<(unsigned)nwin, XCH_THREADS, XL_SMEM, s>>>(base, seg, W, M, sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(),
+        const size_t xls = mode == C_H22 ? XL_SMEM_H22 : XL_SMEM;
+        SPMM_CUDA(cudaFuncSetAttribute(kl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)xls));
+        kl<<<(unsigned)nwin, XCH_THREADS, xls, s>>>(base, seg, W, M, sig.ptr.as<int32_t>(), sig.blk.as<int32_t>(),
                                                         bptr.as<int32_t>(), bloc.as<uint16_t>(), xr.as<int2>(),
                                                         ord.as<uint32_t>(), lpos.as<int32_t>(), nnz, p.nt, p.nw, perm);
         SPMM_CUDA(cudaGetLastError());
