@@ -405,6 +405,12 @@ spmm_status launch_chain(int mode, const int32_t *base, const int32_t *seg, int6
 // count pass, so they need no pass of their own.
 constexpr int XCH_THREADS = 1024;
 constexpr int XCH_CACHE = XCH_THREADS;   // posting-list prefix of up to 1024 blocks kept in smem per step
+constexpr int XT_CAP = 8192;             // k_chain_x: touched rows listed per step (dynamic smem, 2 buffers)
+#ifdef SPMM_EXP_NO_XT   // A/B variant: no touched list in k_chain_x (score and reset re-walk the posting lists)
+constexpr int32_t XT_USE = -1;
+#else
+constexpr int32_t XT_USE = XT_CAP;
+#endif
 
 __global__ void k_win_of(const int32_t *base, int64_t M, int64_t W, int32_t *win) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < M; q += (int64_t)gridDim.x * blockDim.x)
@@ -601,6 +607,10 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     __shared__ PT wsum[32];
     __shared__ Key red[2][XCH_THREADS / 32];
     __shared__ int32_t s_ptr;
+    // the distinct rows a step's count pass touched (its T; up to XT_CAP, listed on first touch): the score pass and
+    // the next step's counter reset walk it instead of re-walking the posting lists (re-walk when it overflowed)
+    extern __shared__ int32_t xt_s[];   // [2][XT_CAP]
+    __shared__ int32_t s_nt[2];
     const int32_t w = (int32_t)blockIdx.x;
     // window w = positions [s0, s1) of the pre-order: fixed windows of W, or HYBRID_1's segments (seg)
     const int64_t s0 = seg ? seg[w] : (int64_t)w * W, s1 = seg ? seg[w + 1] : min(s0 + W, M);
@@ -621,6 +631,7 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     const int32_t nfirst = WARPREF ? min(n, nw) : 1;
     Key best;
     int32_t prev = -1, pprev = -1, pref = -1, pref2 = -1;
+    if (threadIdx.x < 2) s_nt[threadIdx.x] = 0;   // ordered by the first rows' barriers
     for (int32_t q = 0; q < nfirst; ++q) {
         best = Key{0xffffffffu, 0xffffffffu, 0xffffffffu, 0u};
         for (int32_t a = threadIdx.x; a < n; a += XCH_THREADS) {
@@ -642,6 +653,11 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
     for (int32_t q = nfirst; q < n; ++q) {
         const int buf = q & 1;
         int32_t *cc = buf ? cnt1 : cnt0, *co = buf ? cnt0 : cnt1;
+        int32_t *xt = xt_s + buf * XT_CAP;
+        const int32_t *xto = xt_s + (buf ^ 1) * XT_CAP;
+        const int32_t nto = s_nt[buf ^ 1];   // the previous step's touched count (> XT_CAP: overflowed)
+        __syncthreads();                     // everyone has read s_nt[buf ^ 1] / s_nt[buf] of earlier steps
+        if (threadIdx.x == 0) s_nt[buf] = 0;
         // the row Hamming distances are taken to; out[q - 1] is written by thread 0 after the previous step's
         // last barrier, so nw == 1 reads it from the register copy prev (as k_chain does)
         const int32_t ref = WARPREF ? (nw == 1 ? prev : out[q - nw]) : prev;
@@ -652,13 +668,18 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
         // step's prefix lives in the other buffer
         if (cached) xprefix(sig_blk, bptr, bs, be - bs, pre[buf], bst[buf], wsum, brow, win, mw, xr);
         // reset the previous step's counters (other buffer), then count |b_r ∩ b_ref|
-        if (pref >= 0) {
+        if (pref >= 0 && nto <= XT_USE) {
+            for (int32_t i = threadIdx.x; i < nto; i += XCH_THREADS) co[xto[i]] = 0;
+        } else if (pref >= 0) {
             auto reset = [&](int32_t r) { co[r] = 0; };
             if (cached_pp) xvisit(pre[buf ^ 1], bst[buf ^ 1], sig_ptr[pref + 1] - sig_ptr[pref], brow, reset);
             else xvisit_all(pref, sig_ptr, sig_blk, bptr, brow, pre[buf ^ 1], bst[buf ^ 1], wsum, win, mw, xr, reset);
         }
         auto count = [&](int32_t r) {
-            if (r != prev && !is_placed(placed, r)) atomicAdd(cc + r, 1);
+            if (r != prev && !is_placed(placed, r) && atomicAdd(cc + r, 1) == 0) {
+                const int32_t i = atomicAdd(&s_nt[buf], 1);
+                if (i < XT_USE) xt[i] = r;
+            }
         };
         if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, count);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, xr, count);
@@ -697,7 +718,9 @@ __global__ void __launch_bounds__(XCH_THREADS, 1) k_chain_x(const int32_t *base,
                 if (key_less(k, best)) best = k;
             }
         };
-        if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
+        const int32_t nt1 = s_nt[buf];
+        if (nt1 <= XT_USE) for (int32_t i = threadIdx.x; i < nt1; i += XCH_THREADS) score(xt[i]);
+        else if (cached) xvisit(pre[buf], bst[buf], be - bs, brow, score);
         else xvisit_all(ref, sig_ptr, sig_blk, bptr, brow, pre[buf], bst[buf], wsum, win, mw, xr, score);
         if constexpr (TWOREF) {
             if (ref2 >= 0) {
@@ -1179,7 +1202,9 @@ spmm_status launch_chain_exact(int mode, const int32_t *base, const int32_t *seg
         SPMM_CUDA(cudaGetLastError());
         return SPMM_OK;
     }
-    kern<<<(unsigned)nwin, XCH_THREADS, 0, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
+    const size_t xts = 2 * XT_CAP * sizeof(int32_t);
+    SPMM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)xts));
+    kern<<<(unsigned)nwin, XCH_THREADS, xts, s>>>(base, seg, W, M, nwin > 1 ? 1 : 0, sig.ptr.as<int32_t>(),
                                                 sig.blk.as<int32_t>(), bptr.as<int32_t>(), brow.as<int32_t>(),
                                                 win.as<int32_t>(), xr.p ? xr.as<int2>() : nullptr,
                                                 ord.as<uint32_t>(), nnz, p.nt, p.nw,

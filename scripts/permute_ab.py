@@ -26,7 +26,7 @@ for pol in {policies!r}:
     ts = []
     for rep in range(3):
         torch.cuda.synchronize(); t0 = time.perf_counter()
-        bench.permute_spec(h, pol, 1024)
+        bench.permute_spec(h, pol, {window})
         torch.cuda.synchronize(); ts.append((time.perf_counter() - t0) * 1e3)
     perm = h.perm()
     res[pol] = {{"ms": sorted(ts)[1], "all_ms": ts, "sha": hashlib.sha256(perm.tobytes()).hexdigest()[:16]}}
@@ -39,6 +39,7 @@ def main():
     ap.add_argument("--define", action="append", required=True)
     ap.add_argument("--configs", default="c3")
     ap.add_argument("--policies", default="cta_aware,hybrid_2_1")
+    ap.add_argument("--window", type=int, default=1024)
     args = ap.parse_args()
     from paper_conf_ispass_mehrabilcslo21_b200 import _build
     lib_b = _build.build_variant(args.define, "_".join(d.lower() for d in args.define))
@@ -47,7 +48,7 @@ def main():
     for c in args.configs.split(","):
         r = {}
         for name, lib in (("product", ""), ("variant", lib_b)):
-            p = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policies=pols)],
+            p = subprocess.run([sys.executable, "-c", CHILD.format(root=ROOT, lib=lib, config=c, policies=pols, window=args.window)],
                                capture_output=True, text=True, timeout=3600)
             line = [l for l in p.stdout.splitlines() if l.startswith("{")]
             if not line:
@@ -57,7 +58,7 @@ def main():
                         "identical": r["product"].get(pol, {}).get("sha") == r["variant"].get(pol, {}).get("sha")}
                   for pol in pols}
         print(c, json.dumps(out[c]), flush=True)
-    print(json.dumps({"defines": args.define, "results": out}))
+    print(json.dumps({"defines": args.define, "window": args.window, "results": out}))
 
 
 if __name__ == "__main__":
