@@ -1,5 +1,5 @@
-"""GPU parity of the inverted-index chain builder (k_chain_x): paper-exact greedy chains
-over windows above 32768 rows, up to the whole matrix (W = 0).
+"""GPU parity of the inverted-index chain builders (k_chain_xl for windows of <= 4096 rows, k_chain_x above, up to
+the whole matrix): paper-exact greedy chains (W = 0).
 
 Small sizes: forced onto the inverted-index builder (SPMM_CHAIN_EXACT=1) and compared bit-exact with the
 oracle (oracle.c, O(W^2) brute force of the definition) for CTA_AWARE and HYBRID_2_1, whole-matrix and
@@ -145,3 +145,29 @@ def test_exact_whole_matrix_c2(policy):
     h.close()
     assert np.array_equal(np.sort(perm), np.arange(a.M))
     check_sampled_steps(a, perm, policy, samples=40)
+
+
+def _hub_matrix(M, N, seed):
+    """2-3 random columns per row plus one column (0) shared by every row: every greedy step touches every
+    unplaced row of its window through block 0's posting list."""
+    rng = np.random.default_rng(seed)
+    rows = [sorted({0, *rng.choice(np.arange(1, N), size=int(rng.integers(2, 4)), replace=False).tolist()})
+            for _ in range(M)]
+    return syn.from_lists(M, N, rows)
+
+
+@pytest.mark.parametrize("window,M,policies", [
+    (8192, 2 * 8192 + 1000, ("cta_aware", "hybrid_2_1")),        # k_chain_x, multi-window, ragged last window
+    (16384, 16384 + 3000, ("cta_aware", "hybrid_2_2")),          # > 8192 touched rows per step: list overflow path
+])
+def test_exact_builder_large_windows(exact_builder, window, M, policies):
+    """Windows above k_chain_xl's 4096 rows go to k_chain_x, whose per-step touched-row list (8192 rows) falls back
+    to re-walking the posting lists when a step touches more rows: both paths against the oracle."""
+    a = _hub_matrix(M, 30000, 2107)
+    h = pkg.SpMM.from_csr(a)
+    for policy in policies:
+        h.permute(policy, window=window)
+        got = h.perm()
+        ref = oracle.permute(a, policy, window=window)
+        assert np.array_equal(got, ref), (policy, window, int(np.argmax(got != ref)))
+    h.close()
