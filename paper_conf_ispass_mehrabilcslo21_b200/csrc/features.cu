@@ -126,6 +126,7 @@ __global__ void k_popcount_rows(const uint32_t *Dmap, int64_t words, unsigned lo
 // Longer pairs (power-law hub rows, up to 10^5 nnz): warp per pair -- the lanes take the distinct blocks of the
 // shorter row (run starts) and binary-search each in the longer row's columns -- so no single thread walks a hub row.
 constexpr int32_t ADJ_SHORT = 256;
+constexpr int32_t ADJ_HUGE = 2048;   // both rows longer: the pair goes to k_adjacent_huge (a CTA per pair)
 __device__ __forceinline__ int32_t adj_common_merge(const OrigCSR &A, int64_t p, int32_t bw) {
     int32_t i = A.begin(p), ie = A.end(p), j = A.begin(p + 1), je = A.end(p + 1);
     int32_t common = 0;
@@ -143,7 +144,8 @@ __device__ __forceinline__ int32_t adj_common_merge(const OrigCSR &A, int64_t p,
     }
     return common;
 }
-__global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk_row, Stats *st) {
+__global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk_row, Stats *st, int64_t *huge,
+                           unsigned long long *n_huge) {
     const int lane = threadIdx.x & 31;
     for (int64_t p0 = (int64_t)blockIdx.x * blockDim.x; p0 < M - 1; p0 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t p = p0 + threadIdx.x;
@@ -156,6 +158,10 @@ __global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk
             lng = (e0 - b0) + (e1 - b1) > ADJ_SHORT;
             if (!lng) hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * adj_common_merge(A, p, bw);
         }
+        // pairs of two hub rows: deferred to k_adjacent_huge (their statistic is added there)
+        const bool hg = lng && min(e0 - b0, e1 - b1) > ADJ_HUGE;
+        if (hg) huge[atomicAdd(n_huge, 1ULL)] = p;
+        lng = lng && !hg;
         // the warp's long pairs, one after another, all lanes together
         unsigned todo = __ballot_sync(0xffffffffu, lng);
         while (todo) {
@@ -182,7 +188,44 @@ __global__ void k_adjacent(OrigCSR A, int64_t M, int32_t bw, const int32_t *nblk
             for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
             if (lane == src) hd = (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * c;
         }
-        warp_stats(st, hd, in);
+        warp_stats(st, hd, in && !hg);
+    }
+}
+
+// the deferred pairs of two rows above ADJ_HUGE nnz: a CTA per pair, its threads take the shorter row's distinct
+// blocks and binary-search them in the longer row
+__global__ void k_adjacent_huge(OrigCSR A, int32_t bw, const int32_t *nblk_row, const int64_t *huge,
+                                const unsigned long long *n_huge, Stats *st) {
+    __shared__ int32_t part[32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (unsigned long long k = blockIdx.x; k < *n_huge; k += gridDim.x) {
+        const int64_t p = huge[k];
+        const int32_t b0 = A.begin(p), e0 = A.end(p), b1 = A.begin(p + 1), e1 = A.end(p + 1);
+        const bool first_short = e0 - b0 <= e1 - b1;
+        const int32_t sb = first_short ? b0 : b1, se = first_short ? e0 : e1;
+        const int32_t tb = first_short ? b1 : b0, te = first_short ? e1 : e0;
+        int32_t c = 0;
+        for (int32_t i = sb + (int32_t)threadIdx.x; i < se; i += blockDim.x) {
+            const int32_t x = A.col(i) / bw;
+            if (i > sb && A.col(i - 1) / bw == x) continue;
+            int32_t lo = tb, hi = te;
+            while (lo < hi) {
+                const int32_t mid = (lo + hi) >> 1;
+                if (A.col(mid) / bw < x) lo = mid + 1;
+                else hi = mid;
+            }
+            c += lo < te && A.col(lo) / bw == x;
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+        if (lane == 0) part[wid] = c;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int32_t t = 0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += part[w];
+            stats_add(st, (long long)nblk_row[p] + nblk_row[p + 1] - 2LL * t);
+        }
+        __syncthreads();
     }
 }
 
@@ -240,9 +283,17 @@ spmm_status compute_features(spmm_ctx *h, bool current_order, const spmm_params 
     k_stats_u32<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(nblk, 256), 148 * 16)), 256, 0, s>>>(
         req.as<unsigned int>(), nblk, 1, S + 2);
     k_popcount_rows<<<nw, 256, 0, s>>>(dmap.as<uint32_t>(), words, dd.as<unsigned long long>());
-    if (M > 1)
+    DevBuf huge;
+    if (M > 1) {
+        // room for every pair whose rows both exceed ADJ_HUGE nnz (at most nnz / ADJ_HUGE of them) + the counter
+        const int64_t cap = h->nnz / ADJ_HUGE + 2;
+        SPMM_TRY(huge.alloc((size_t)(cap + 1) * sizeof(int64_t), s));
+        unsigned long long *n_huge = reinterpret_cast<unsigned long long *>(huge.as<int64_t>() + cap);
+        SPMM_CUDA(cudaMemsetAsync(n_huge, 0, sizeof(unsigned long long), s));
         k_adjacent<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(M, 256), 148 * 16)), 256, 0, s>>>(
-            A, M, bw, nbr.as<int32_t>(), S + 3);
+            A, M, bw, nbr.as<int32_t>(), S + 3, huge.as<int64_t>(), n_huge);
+        k_adjacent_huge<<<148 * 4, 256, 0, s>>>(A, bw, nbr.as<int32_t>(), huge.as<int64_t>(), n_huge, S + 3);
+    }
     SPMM_CUDA(cudaGetLastError());
     Stats hs[4];
     std::vector<unsigned long long> hwl(nw), htt(nw), hdd(nw);
